@@ -1,0 +1,117 @@
+"""O2 pointer B+tree: structure and results under insert/delete sequences, pinned by O1 /
+O6 (std::map) and the textbook invariants; Fig 3 / Fig 10 statistics (weak)."""
+import numpy as np
+import pytest
+
+import harmonia_gen as gen
+
+
+@pytest.mark.parametrize("F", [4, 5, 8, 16, 64, 128])
+def test_insert_delete_sequences(orc, F):
+    rng = np.random.default_rng(F)
+    universe = gen.random_keys(4000, seed=100 + F, bits=20)
+    t = orc.BPlusTree(F)
+    ref = {}
+    for step in range(6000):
+        k = int(universe[rng.integers(universe.shape[0])])
+        if rng.random() < 0.6:
+            v = int(rng.integers(1 << 62))
+            assert t.insert(k, v) == (0 if k in ref else 1)
+            ref[k] = v
+        else:
+            assert t.erase(k) == (1 if k in ref else 0)
+            ref.pop(k, None)
+        if step % 500 == 0:
+            assert t.check() == 0, step
+    assert t.check() == 0
+    assert len(t) == len(ref)
+    ks = np.array(sorted(ref), dtype=np.uint64)
+    vs = np.array([ref[int(k)] for k in ks], dtype=np.uint64)
+    dk, dv = t.dump()
+    assert np.array_equal(dk, ks) and np.array_equal(dv, vs)
+    q = np.concatenate([universe, gen.edge_queries(ks)])
+    assert np.array_equal(t.search(q), orc.sorted_search(ks, vs, q))
+
+
+def test_delete_everything(orc):
+    keys = gen.uniform_keys(3000)
+    t = orc.BPlusTree(8)
+    t.insert_many(keys, gen.values_for(keys))
+    assert t.height > 2
+    for k in np.random.default_rng(1).permutation(keys):
+        assert t.erase(k) == 1
+        assert t.erase(k) == 0
+    assert len(t) == 0 and t.height == 1 and t.check() == 0
+
+
+def test_height_bounds(orc):
+    # a B+tree of n records and fanout F has height between log_F and log_{ceil(F/2)} (+1)
+    import math
+
+    for F in (8, 16, 64):
+        n = 20000
+        keys = gen.uniform_keys(n)
+        t = orc.BPlusTree(F)
+        t.insert_many(keys[np.random.default_rng(F).permutation(n)], keys)
+        h = t.height
+        assert math.ceil(math.log(n / (F - 1), F)) + 1 <= h <= math.ceil(math.log(n / (F // 2), F // 2)) + 2
+
+
+def test_update_map_matches_bptree(orc):
+    keys = gen.uniform_keys(5000)
+    vals = gen.values_for(keys)
+    m = orc.UpdateMap(keys, vals)
+    t = orc.BPlusTree(16)
+    t.insert_many(keys, vals)
+    for b in range(3):
+        ops, ks, vs = gen.update_ops(keys, 2000, insert_frac=0.05, delete_frac=0.05, seed=gen.SEED_OPS + b)
+        m.apply(ops, ks, vs)
+        for o, k, v in zip(ops.tolist(), ks.tolist(), vs.tolist()):
+            if o == 0:
+                t.insert(k, v)
+            else:
+                t.erase(k)
+        mk, mv = m.dump()
+        tk, tv = t.dump()
+        assert np.array_equal(mk, tk) and np.array_equal(mv, tv)
+        assert t.check() == 0
+
+
+def test_update_map_semantics(orc):
+    # C-A18: batch order, last op per key wins, delete of missing key is a no-op
+    m = orc.UpdateMap(np.array([10, 20], dtype=np.uint64), np.array([1, 2], dtype=np.uint64))
+    ops = np.array([0, 0, 1, 1, 0, 0], dtype=np.uint8)
+    ks = np.array([15, 10, 20, 99, 15, 20], dtype=np.uint64)
+    vs = np.array([5, 6, 0, 0, 7, 8], dtype=np.uint64)
+    assert m.apply(ops, ks, vs) == 3
+    k, v = m.dump()
+    assert k.tolist() == [10, 15, 20] and v.tolist() == [6, 7, 8]
+
+
+def test_fig10_front_half_weak(orc):
+    """Fig 10: ~80 % of queries resolve in the front half of a node when nodes are
+    about half full.  Statistical and weak (T9): an insertion-built tree (~69 % fill)
+    resolves well above half in the front half; the fully packed layout does not."""
+    for F in (16, 64, 128):
+        keys = gen.uniform_keys(1 << 15)
+        t = orc.BPlusTree(F)
+        t.insert_many(keys[np.random.default_rng(F).permutation(keys.shape[0])], keys)
+        nodes, entries = t.level_stats()
+        fill = float(entries[-1]) / float(nodes[-1]) / (F - 1)
+        assert 0.6 < fill < 0.8, fill   # random-order insertion: ~ln 2 occupancy
+        c = t.quarter_stats(gen.uniform_queries(keys, 4000))
+        front = (c[0] + c[1]) / c.sum()
+        assert front > 0.6, (F, front)
+
+
+def test_fig3_comparisons_weak(orc):
+    """Fig 3: height-4 fanout-8 tree, per-level comparisons average near 4 with a
+    large spread between min and max."""
+    keys = gen.uniform_keys(700)
+    t = orc.BPlusTree(8)
+    t.insert_many(keys[np.random.default_rng(3).permutation(keys.shape[0])], keys)
+    c = t.comparisons(gen.uniform_queries(keys, 100))
+    avg = c.mean(axis=0)
+    assert np.all(avg > 1.5) and np.all(avg < 6.5)
+    assert c.shape[1] == 4  # height 4 as in the paper's setting
+    assert np.all(c.max(axis=0)[1:] - c.min(axis=0)[1:] >= 3)  # below the (small) root

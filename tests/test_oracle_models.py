@@ -1,0 +1,102 @@
+"""O5 models: Eq 2, PSA order, NTG step model (Fig 9), Eq 3/4 size choice, Fig 2
+transaction closed forms.  Pinned by the paper's stated values (tests/golden)."""
+import numpy as np
+
+import harmonia_gen as gen
+from conftest import golden_kv, golden_lines
+
+
+def test_eq2_paper_value(orc):
+    for ln in golden_lines("eq2.txt"):
+        B, T, K, N = (int(x) for x in ln.split())
+        assert orc.psa_bits(B, T, K) == N
+
+
+def test_eq2_equals_log2_T_over_K(orc):
+    # Eq 2 simplifies to N = log2(T / K); for powers of two it is exact
+    for lt in range(4, 33):
+        assert orc.psa_bits(64, 2.0 ** lt, 16) == max(0, lt - 4)
+    assert orc.psa_bits(64, 10, 16) == 0
+
+
+def test_fig5_fig7_psa_order(orc):
+    g = golden_kv("fig5_fig7.txt")
+    q = np.array([int(x) for x in g["input"].split()], dtype=np.uint64)
+    exp = [int(x) for x in g["sorted"].split()]
+    # with enough bits PSA is a full (stable) sort over the key span [0, 63]
+    perm = orc.psa_order(q, 64, 0, 63)
+    assert q[perm].tolist() == exp
+    # with fewer bits only the top bits order the batch: 1 and 2 share bucket 0 with 2 bits
+    perm2 = orc.psa_order(q, 2, 0, 63)
+    assert q[perm2].tolist() == [2, 1, 20, 35]  # stable inside a bucket
+
+
+def test_psa_bucket_monotone_and_span(orc):
+    keys = gen.uniform_keys(1 << 12)
+    lo, hi = int(keys[0]), int(keys[-1])
+    qs = np.sort(gen.uniform_queries(keys, 2000, miss_frac=0.5))
+    b = [orc.psa_bucket(int(x), 10, lo, hi) for x in qs]
+    assert all(x <= y for x, y in zip(b, b[1:]))
+    assert max(b) < 1 << 10 and len(set(b)) > 500
+    # a common prefix is skipped (C-A11): keys inside [2^40, 2^40 + 2^20) use bits 19..10
+    base = 1 << 40
+    assert orc.psa_bucket(base, 10, base, base + (1 << 20) - 1) == 0
+    assert orc.psa_bucket(base + (1 << 20) - 1, 10, base, base + (1 << 20) - 1) == 1023
+    assert orc.psa_bucket(0, 10, base, base + 5) == 0  # clamped
+
+
+def test_fig9_ntg_steps(orc):
+    for ln in golden_lines("fig9.txt"):
+        F, gs, kpl, r, steps = (int(x) for x in ln.split())
+        assert orc.ntg_steps(r, F - 1, gs, kpl) == steps
+
+
+def test_ntg_steps_brute(orc):
+    # steps = index of the step holding the first key > q, capped by the steps covering cnt
+    for cnt in range(1, 40):
+        for gs in (1, 2, 4, 8):
+            for kpl in (1, 2):
+                w = gs * kpl
+                for r in range(cnt + 1):
+                    s, covered = 0, 0
+                    while covered < cnt:
+                        s += 1
+                        covered += w
+                        if r < covered:
+                            break
+                    assert orc.ntg_steps(r, cnt, gs, kpl) == s
+
+
+def test_fig2_closed_forms(orc):
+    g = golden_kv("fig2.txt")
+    F, h, W = int(g["fanout"]), int(g["height"]), int(g["queries_per_warp"])
+    # full fanout-8 tree of height 4: 1, 8, 64, 512 nodes; 512 * 7 records
+    n = (F - 1) * F ** (h - 1)
+    keys = np.arange(n, dtype=np.uint64) * np.uint64(3)
+    lay = orc.layout_build(keys, keys, F, 1.0)
+    assert lay.h == h
+    # worst: the 4 queries of a warp sit under 4 different level-1 subtrees
+    sub = n // F
+    worst = np.array([keys[i * sub * 2] for i in range(W)], dtype=np.uint64)
+    assert abs(lay.warp_transactions(worst, W) - float(g["worst"])) < 1e-12
+    best = np.repeat(keys[17], W)
+    assert abs(lay.warp_transactions(best, W) - float(g["best"])) < 1e-12
+    # uniform random queries land between the two, near the worst case (paper: 97 %)
+    u = lay.warp_transactions(gen.uniform_queries(keys, 4000), W)
+    assert float(g["best"]) < u < float(g["worst"]) and u / float(g["worst"]) > 0.85
+
+
+def test_eq4_narrowing(orc):
+    """Eq 3/4: with PSA-ordered queries, narrowing keeps paying; with a fully
+    random order at large fanout the per-warp max steps grow faster than 2x."""
+    keys = gen.uniform_keys(1 << 16)
+    lay = orc.layout_build(keys, keys, 64, 1.0)
+    q = gen.uniform_queries(keys, 2000)
+    s32 = lay.ntg_warp_steps(q, 32, kpl=2)
+    s16 = lay.ntg_warp_steps(q, 16, kpl=2)
+    s2 = lay.ntg_warp_steps(q, 2, kpl=2)
+    assert s32 <= s16 <= s2
+    g_sorted = lay.ntg_choose_gs(np.sort(q), 32, kpl=2)
+    g_rand = lay.ntg_choose_gs(q, 32, kpl=2)
+    assert 2 <= g_rand <= 32 and 2 <= g_sorted <= 32
+    assert g_sorted <= g_rand  # sorted batches tolerate narrower groups
