@@ -1,0 +1,232 @@
+/*
+ * harmonia.h — C ABI of libharmonia.so: batched B+tree point and range queries over the
+ * Harmonia layout on NVIDIA B200 (sm_100a).
+ *
+ * Method: Yan, Lin, Peng, Zhang, "Harmonia: A High Throughput B+tree for GPUs", PPoPP'19.
+ * Citations "P:Lnnn" are lines of the paper text (reference PAPER.md); "C-Axx" are the
+ * readings of ambiguous passages listed in DESIGN.md §3.
+ *
+ * Conventions (all functions):
+ *   - Plain C11, no exceptions cross the ABI; every fallible call returns harmonia_status.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = the legacy default stream).
+ *   - "d_" pointers are device memory on the tree's device, "h_" pointers host memory.
+ *   - Keys and values are uint64.  Keys are compared unsigned (C-A1).
+ *   - *_batch calls only enqueue work on `stream` and return after launch; launch errors
+ *     return HARMONIA_ERR_CUDA; execution errors surface at the caller's synchronisation.
+ *   - Query, result and workspace buffers are caller-owned; the library performs no device
+ *     allocation on any query path (search, range, host search).
+ *   - Query inputs are never errors: a query equal to HARMONIA_KEY_PAD returns NOT_FOUND,
+ *     a range with lo > hi returns count 0.
+ *   - Results are bit-identical whatever group size, PSA bits, window, staging plan or GPU
+ *     count is used.
+ *   - A tree is immutable during search/range calls; calls on different streams need
+ *     separate workspaces; harmonia_update_batch needs exclusive access (the paper's phase
+ *     model: query phase, then update phase).
+ */
+#ifndef HARMONIA_H
+#define HARMONIA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HARMONIA_ABI_VERSION 1
+#define HARMONIA_NOT_FOUND UINT64_C(0xFFFFFFFFFFFFFFFF) /* result of an absent key (C-A4)     */
+#define HARMONIA_KEY_PAD   UINT64_C(0xFFFFFFFFFFFFFFFF) /* unused node slot; never a key (C-A2) */
+#define HARMONIA_MAX_LEVELS 64
+
+typedef enum {
+  HARMONIA_OK = 0,
+  HARMONIA_ERR_INVALID_ARG = 1,  /* null pointer, bad fanout/group size/opts, short workspace  */
+  HARMONIA_ERR_UNSORTED = 2,     /* build keys not strictly increasing (duplicates included)  */
+  HARMONIA_ERR_RESERVED = 3,     /* a key == HARMONIA_KEY_PAD or a value == HARMONIA_NOT_FOUND */
+  HARMONIA_ERR_OUT_OF_MEMORY = 4,
+  HARMONIA_ERR_CUDA = 5,         /* CUDA API/launch failure; see harmonia_last_cuda_error()   */
+  HARMONIA_ERR_DEVICE_MISMATCH = 6,
+  HARMONIA_ERR_TOO_LARGE = 7     /* more than 2^32-1 nodes, or height > HARMONIA_MAX_LEVELS    */
+} harmonia_status;
+
+/* Opaque: one Harmonia layout (key region + prefix-sum child region + values) resident on
+ * one device.  Owned by the library; release with harmonia_destroy. */
+typedef struct harmonia_tree harmonia_tree;
+
+typedef struct {
+  uint32_t fanout;        /* F: max children per internal node, power of two in [4, 256].
+                             Internal nodes hold <= F-1 separator keys, leaves <= F-1 records
+                             (P:L120, L268).  0 => 64.                                       */
+  float fill;             /* bulk-load target occupancy in [0.5, 1]; 0 => 1.0 (C-A6)         */
+  int32_t keys_on_device; /* 1: keys/values are device pointers on the current device; 0: host */
+  int32_t reserved;
+} harmonia_build_opts;
+
+/* Query options.  An all-zero struct (or a NULL pointer) selects every default. */
+typedef struct {
+  int32_t group_size;   /* NTG lanes per query G: 0 = auto (measured table for
+                           the tree's fanout); else a power of two in [2, 32] with 2G <= F.  */
+  int32_t psa_bits;     /* PSA sort bits Nb (Eq 2): 0 = auto = ceil(log2(T/K)), K=16;
+                           < 0 = PSA off (queries searched in arrival order); else 1..28.   */
+  int32_t smem_levels;  /* top tree levels staged in shared memory: 0 = auto plan (fits the
+                           smem budget), < 0 = none, else that many levels (clamped).        */
+  int32_t flags;        /* HARMONIA_QF_* bits                                                 */
+  uint64_t window;      /* PSA window = queries partitioned together (the paper's "time
+                           window"): 0 = auto; otherwise rounded to a multiple of 1024 */
+  uint64_t reserved[2];
+} harmonia_query_opts;
+
+#define HARMONIA_QF_NO_PS_SMEM 1u  /* do not stage the prefix-sum array in shared memory     */
+#define HARMONIA_QF_GATHER     2u  /* PSA return via a separate gather pass instead of the
+                                      search kernel scattering results in place             */
+
+typedef struct {
+  uint64_t n_keys;
+  uint32_t fanout, height, psa_bits_auto, group_size_auto;
+  uint64_t n_nodes, n_internal, n_leaves;
+  uint64_t level_start[HARMONIA_MAX_LEVELS + 1]; /* BFS level boundaries, [0, N]            */
+  uint64_t key_region_bytes, ps_bytes, value_bytes;
+  uint64_t min_key, max_key;                     /* PAD/0 when the tree is empty             */
+  int32_t device;
+  int32_t reserved;
+} harmonia_info;
+
+/* ---------------------------------------------------------------------------------------
+ * harmonia_build — bulk-load a Harmonia layout from n records (Fig 4(b)).
+ *   keys[n]: strictly increasing, none equal to HARMONIA_KEY_PAD (C-A9);
+ *   values[n]: none equal to HARMONIA_NOT_FOUND.  Host or device per opts->keys_on_device;
+ *   caller-owned, copied (not retained).  n may be 0 (every query then returns NOT_FOUND).
+ *   Layout: key region = N nodes x F uint64 slots in breadth-first order, unused slots =
+ *   HARMONIA_KEY_PAD (C-A2); PS = uint32[I+1], PS[n] = key-region index of node n's first
+ *   child, PS[I] = N (C-A7); values = uint64[L x F] aligned with leaf slots (C-A3).
+ *   Node counts per level follow the even-distribution closed form (C-A6).
+ *   Synchronises `stream` (validation result is read back).  *out receives the tree.
+ *   Errors: INVALID_ARG, UNSORTED, RESERVED, OUT_OF_MEMORY, TOO_LARGE, CUDA.
+ * ------------------------------------------------------------------------------------- */
+harmonia_status harmonia_build(const uint64_t* keys, const uint64_t* values, uint64_t n,
+                               const harmonia_build_opts* opts, void* stream,
+                               harmonia_tree** out);
+
+/* Frees the tree's device memory (synchronises the device). NULL is a no-op. */
+void harmonia_destroy(harmonia_tree* tree);
+
+harmonia_status harmonia_get_info(const harmonia_tree* tree, harmonia_info* info);
+
+/* Copies the layout to caller-owned host arrays (for the oracle's layout checker):
+ * h_key_region[n_nodes*F], h_ps[n_internal+1], h_leaf_values[n_leaves*F].  Synchronous. */
+harmonia_status harmonia_export_layout(const harmonia_tree* tree, uint64_t* h_key_region,
+                                       uint32_t* h_ps, uint64_t* h_leaf_values);
+
+/* ---------------------------------------------------------------------------------------
+ * harmonia_search_batch — n point queries (§3.2.1; PSA §4.1; NTG §4.2).
+ *   d_queries[n] -> d_values_out[n]: the value of each query's key, or HARMONIA_NOT_FOUND.
+ *   Pipeline per PSA window: bucket histogram on the top Nb key bits, scan, stable-per-warp
+ *   bucket scatter (PSA, Eq 2), NTG descent with Eq 1 (child = PS[node] + i - 1) and leaf
+ *   probe, results written back in the caller's order.  d_queries and d_values_out may not
+ *   overlap.  d_workspace must hold harmonia_search_workspace_bytes(tree, n, opts) bytes,
+ *   16-byte aligned.   Errors: INVALID_ARG, DEVICE_MISMATCH, CUDA.
+ * ------------------------------------------------------------------------------------- */
+size_t harmonia_search_workspace_bytes(const harmonia_tree* tree, uint64_t n,
+                                       const harmonia_query_opts* opts);
+harmonia_status harmonia_search_batch(const harmonia_tree* tree, const uint64_t* d_queries,
+                                      uint64_t n, uint64_t* d_values_out, void* d_workspace,
+                                      size_t workspace_bytes, const harmonia_query_opts* opts,
+                                      void* stream);
+
+/* Host-buffer variant (end-to-end): h_queries[n] / h_values_out[n] in host memory (pinned
+ * for overlap; pageable works but serialises).  Chunks are copied H2D, searched and copied
+ * D2H on a three-stage pipeline; everything is ordered after prior work on `stream` and the
+ * caller synchronises `stream` to consume h_values_out.  d_workspace must hold
+ * harmonia_search_host_workspace_bytes(tree, n, opts).  Not reentrant per tree. */
+size_t harmonia_search_host_workspace_bytes(const harmonia_tree* tree, uint64_t n,
+                                            const harmonia_query_opts* opts);
+harmonia_status harmonia_search_batch_host(const harmonia_tree* tree, const uint64_t* h_queries,
+                                           uint64_t n, uint64_t* h_values_out,
+                                           void* d_workspace, size_t workspace_bytes,
+                                           const harmonia_query_opts* opts, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * harmonia_range_batch — n inclusive range queries [lo, hi] ("use the basic query
+ *   operation to get the first target key in the range, and scan the key region from the
+ *   first target key to the last target key"; C-A10).
+ *   Query j writes its first min(count, max_results) records, ascending, to
+ *   d_keys_out[j*max_results + t] / d_values_out[j*max_results + t]; d_counts_out[j] = the
+ *   true total (> max_results signals truncation).  Slab entries past the count are not
+ *   written.  max_results may be 0 (counts only).  Workspace as for search.
+ * ------------------------------------------------------------------------------------- */
+size_t harmonia_range_workspace_bytes(const harmonia_tree* tree, uint64_t n,
+                                      const harmonia_query_opts* opts);
+harmonia_status harmonia_range_batch(const harmonia_tree* tree, const uint64_t* d_lo,
+                                     const uint64_t* d_hi, uint64_t n, uint32_t max_results,
+                                     uint64_t* d_keys_out, uint64_t* d_values_out,
+                                     uint32_t* d_counts_out, void* d_workspace,
+                                     size_t workspace_bytes, const harmonia_query_opts* opts,
+                                     void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * harmonia_update_batch — batched upsert/delete (§3.2.2; C-A18).
+ *   d_ops[n] (0 = upsert: insert a new record or update an existing record's value;
+ *   1 = delete: remove if present), d_keys[n], d_values[n] (ignored for deletes).
+ *   Sequential semantics in batch order: the last op on a key wins.  Keys equal to
+ *   HARMONIA_KEY_PAD or upsert values equal to HARMONIA_NOT_FOUND are rejected
+ *   (HARMONIA_ERR_RESERVED, tree unchanged).  The layout is rebuilt from the first affected
+ *   leaf: merged leaf sequence, re-packed leaves, internal levels and PS recomputed
+ *   (the paper's post-batch "movement", done as bulk-synchronous device passes).
+ *   May reallocate the tree's arrays; synchronises `stream`.
+ *   d_workspace must hold harmonia_update_workspace_bytes(tree, n).
+ * ------------------------------------------------------------------------------------- */
+size_t harmonia_update_workspace_bytes(const harmonia_tree* tree, uint64_t n);
+harmonia_status harmonia_update_batch(harmonia_tree* tree, const uint8_t* d_ops,
+                                      const uint64_t* d_keys, const uint64_t* d_values,
+                                      uint64_t n, void* d_workspace, size_t workspace_bytes,
+                                      void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * Key-range partitioning across P devices (multi-GPU mode).
+ * harmonia_route_partition: dest(q) = #{ s in d_splitters[0..P-2] : s <= q }  (splitters
+ *   strictly increasing; shard p owns [splitter[p-1], splitter[p]) ).  Writes the queries
+ *   grouped by destination (d_routed[n], destination-major), the original position of each
+ *   routed query (d_pos[n], uint32 — n < 2^32), and h_counts[P] (host, synchronous).
+ * harmonia_scatter_results: d_out[d_pos[i]] = d_routed_values[i] for i < n.
+ * ------------------------------------------------------------------------------------- */
+size_t harmonia_route_workspace_bytes(uint32_t P, uint64_t n);
+harmonia_status harmonia_route_partition(const uint64_t* d_splitters, uint32_t P,
+                                         const uint64_t* d_queries, uint64_t n,
+                                         uint64_t* d_routed, uint32_t* d_pos, uint64_t* h_counts,
+                                         void* d_workspace, size_t workspace_bytes, void* stream);
+harmonia_status harmonia_scatter_results(const uint64_t* d_routed_values, const uint32_t* d_pos,
+                                         uint64_t n, uint64_t* d_out, void* stream);
+
+/* The plan a search/range call with these options would use (for reporting). */
+typedef struct {
+  int32_t group_size, psa_bits, smem_levels, ps_in_smem;
+  uint64_t window;
+  uint32_t smem_bytes, smem_nodes;
+  uint64_t reserved[2];
+} harmonia_plan;
+harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
+                                    const harmonia_query_opts* opts, harmonia_plan* out);
+
+/* Eq 2 as used by psa_bits = 0: ceil(log2(T/K)) clamped to [0, 28], K = 16. */
+int32_t harmonia_psa_bits_auto(uint64_t n_keys);
+
+/* Kernel timing for benchmarks.  While enabled, every kernel the library launches is
+ * bracketed by a CUDA event pair recorded on its launch stream, per kernel class.
+ * harmonia_profile_read synchronises those events, writes the summed milliseconds and
+ * launch counts per class (arrays of HARMONIA_PROF_KINDS) and clears the record. */
+#define HARMONIA_PROF_KINDS 8
+enum { HARMONIA_PROF_SEARCH = 0, HARMONIA_PROF_RANGE = 1, HARMONIA_PROF_PSA_HIST = 2,
+       HARMONIA_PROF_PSA_SCAN = 3, HARMONIA_PROF_PSA_SCATTER = 4, HARMONIA_PROF_RETURN = 5,
+       HARMONIA_PROF_BUILD = 6, HARMONIA_PROF_UPDATE = 7 };
+void harmonia_profile_enable(int on);
+harmonia_status harmonia_profile_read(double* total_ms, uint64_t* launches);
+
+const char* harmonia_status_string(harmonia_status s);
+int harmonia_last_cuda_error(void);          /* cudaError_t of the last ERR_CUDA (thread-local) */
+uint64_t harmonia_kernel_launches(void);     /* kernels this library launched (process total)  */
+int harmonia_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HARMONIA_H */

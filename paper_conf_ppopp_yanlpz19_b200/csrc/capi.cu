@@ -1,0 +1,368 @@
+// Query-side C ABI: planning, search/range orchestration over PSA windows, the host-buffer
+// pipeline, and the multi-GPU routing helpers.  Every arithmetic step of the query path runs
+// in the kernels of psa.cu / search.cu; this file only sequences launches on the caller's
+// stream.
+#include <algorithm>
+#include <cstring>
+
+#include "common.cuh"
+
+namespace hm {
+
+namespace {
+constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
+constexpr uint64_t kAutoWindow = 1ull << 22;  // auto PSA window (queries), see DESIGN.md §5
+
+bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
+}  // namespace
+
+harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o, Plan* p) {
+  harmonia_query_opts z;
+  std::memset(&z, 0, sizeof(z));
+  if (!o) o = &z;
+  Plan P;
+  // ---- NTG group size
+  int G = o->group_size;
+  if (G == 0) {
+    G = auto_group_size(t->F);
+    while (2 * G > (int)t->F) G /= 2;
+  }
+  if (!pow2(G) || G < 2 || G > 32 || 2 * G > (int)t->F) return HARMONIA_ERR_INVALID_ARG;
+  P.G = G;
+  // ---- PSA bits (Eq 2) over the occupied key span (C-A11)
+  int nb = o->psa_bits;
+  if (nb == 0) nb = psa_bits_for(t->n_keys);
+  if (nb > 28) return HARMONIA_ERR_INVALID_ARG;
+  uint64_t window = o->window ? round_up(o->window, 1024) : std::min<uint64_t>(round_up(std::max<uint64_t>(n, 1), 1024), kAutoWindow);
+  if (window > (1ull << 31)) return HARMONIA_ERR_INVALID_ARG;
+  P.window = window;
+  if (nb > 0 && t->n_keys >= 2 && t->min_key < t->max_key) {
+    const uint32_t span = 64 - __builtin_clzll(t->min_key ^ t->max_key);
+    uint32_t lw = 0;
+    while ((1ull << lw) < window) ++lw;
+    nb = std::min<int>({nb, (int)span, (int)lw});  // more buckets than window queries only costs
+    if (nb > 0) {
+      P.psa = true;
+      P.nb = nb;
+      P.bucket.kmin = t->min_key;
+      P.bucket.kmax = t->max_key;
+      P.bucket.shift = span - nb;
+      P.bucket.mask = (uint32_t)((1ull << nb) - 1);
+      P.nbins = 1u << nb;
+    }
+  }
+  P.gather = (o->flags & HARMONIA_QF_GATHER) != 0;
+  // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
+  // top levels in BFS order while they fit
+  const uint32_t ps_bytes = (uint32_t)round_up((t->I + 1) * 4, 16);
+  const uint32_t limit = (uint32_t)std::min<size_t>(t->smem_optin > 1024 ? t->smem_optin - 1024 : 0, 200 * 1024);
+  const uint32_t budget = o->smem_levels > 0 ? limit : std::min(kSmemBudget, limit);
+  uint32_t used = 0;
+  int lv = 0;
+  if (o->smem_levels >= 0) {
+    if (!(o->flags & HARMONIA_QF_NO_PS_SMEM) && t->I > 0 && ps_bytes <= budget) {
+      P.ps_smem = true;
+      P.ps_smem_bytes = ps_bytes;
+      used = ps_bytes;
+    }
+    const int want = o->smem_levels > 0 ? std::min<int>(o->smem_levels, (int)t->h) : (int)t->h;
+    while (lv < want && used + t->level_start[lv + 1] * t->F * 8 <= budget) ++lv;
+  }
+  P.smem_levels = lv;
+  P.smem_nodes = (uint32_t)t->level_start[lv];
+  P.smem_bytes = used + P.smem_nodes * t->F * 8;
+  *p = P;
+  return HARMONIA_OK;
+}
+
+static SearchArgs search_args(const harmonia_tree* t, const Plan& p) {
+  SearchArgs a{};
+  a.keys = t->d_keys;
+  a.ps = t->d_ps;
+  a.vals = t->d_vals;
+  a.leaf_start = t->level_start[t->h - 1];
+  a.h = t->h;
+  a.smem_levels = (uint32_t)p.smem_levels;
+  a.smem_nodes = p.smem_nodes;
+  a.ps_smem_bytes = p.ps_smem ? p.ps_smem_bytes : 0;
+  return a;
+}
+
+static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, uint64_t n, uint64_t* out,
+                                     void* ws, const Plan& p, cudaStream_t st) {
+  if (n == 0) return HARMONIA_OK;
+  if (t->n_keys == 0) {  // C-A17: empty tree, every query is absent
+    HM_CUDA(cudaMemsetAsync(out, 0xFF, n * 8, st));
+    return HARMONIA_OK;
+  }
+  SearchArgs a = search_args(t, p);
+  if (!p.psa) {
+    a.q = q;
+    a.idx = nullptr;
+    a.n = n;
+    a.out = out;
+    return launch_search(t, p, a, st);
+  }
+  const PsaWs w = psa_ws_carve(p, ws);
+  for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
+    const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
+    harmonia_status s = psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr);
+    if (s != HARMONIA_OK) return s;
+    a.q = w.sorted_q;
+    a.n = nw;
+    if (p.gather) {
+      a.idx = nullptr;
+      a.out = w.sorted_out;
+      if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+      if ((s = launch_gather(w.sorted_out, w.idx, nw, out + w0, t->sm_count, st)) != HARMONIA_OK) return s;
+    } else {
+      a.idx = w.idx;
+      a.out = out + w0;
+      if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+    }
+  }
+  return HARMONIA_OK;
+}
+
+static bool on_device(const void* ptr, int dev) {
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return (pa.type == cudaMemoryTypeDevice || pa.type == cudaMemoryTypeManaged) && pa.device == dev;
+}
+
+}  // namespace hm
+
+using namespace hm;
+
+extern "C" size_t harmonia_search_workspace_bytes(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o) {
+  if (!t) return 0;
+  Plan p;
+  if (make_plan(t, n, o, &p) != HARMONIA_OK) return 0;
+  return psa_ws_bytes(p) + 256;
+}
+
+extern "C" harmonia_status harmonia_search_batch(const harmonia_tree* t, const uint64_t* d_q, uint64_t n,
+                                                 uint64_t* d_out, void* ws, size_t ws_bytes,
+                                                 const harmonia_query_opts* o, void* stream) {
+  if (!t) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!d_q || !d_out) return HARMONIA_ERR_INVALID_ARG;
+  if (!on_device(d_q, t->device) || !on_device(d_out, t->device)) return HARMONIA_ERR_DEVICE_MISMATCH;
+  Plan p;
+  harmonia_status s = make_plan(t, n, o, &p);
+  if (s != HARMONIA_OK) return s;
+  const size_t need = psa_ws_bytes(p);
+  if (need) {
+    if (!ws || ws_bytes < need) return HARMONIA_ERR_INVALID_ARG;
+    if (((uintptr_t)ws & 255) != 0) {  // carve from the first 256-B boundary
+      const size_t adj = 256 - ((uintptr_t)ws & 255);
+      if (ws_bytes < need + adj) return HARMONIA_ERR_INVALID_ARG;
+      ws = (char*)ws + adj;
+    }
+  }
+  return search_device(t, d_q, n, d_out, ws, p, (cudaStream_t)stream);
+}
+
+extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
+                                               harmonia_plan* out) {
+  if (!t || !out) return HARMONIA_ERR_INVALID_ARG;
+  Plan p;
+  harmonia_status s = make_plan(t, n, o, &p);
+  if (s != HARMONIA_OK) return s;
+  std::memset(out, 0, sizeof(*out));
+  out->group_size = p.G;
+  out->psa_bits = p.psa ? p.nb : 0;
+  out->smem_levels = p.smem_levels;
+  out->ps_in_smem = p.ps_smem ? 1 : 0;
+  out->window = p.psa ? p.window : 0;
+  out->smem_bytes = p.smem_bytes;
+  out->smem_nodes = p.smem_nodes;
+  return HARMONIA_OK;
+}
+
+// ---- host-buffer pipeline --------------------------------------------------------------
+static uint64_t host_chunk(const Plan& p, uint64_t n) {
+  uint64_t c = p.psa ? p.window : (1ull << 22);
+  return std::max<uint64_t>(1024, std::min<uint64_t>(c, round_up(std::max<uint64_t>(n, 1), 1024)));
+}
+
+extern "C" size_t harmonia_search_host_workspace_bytes(const harmonia_tree* t, uint64_t n,
+                                                       const harmonia_query_opts* o) {
+  if (!t) return 0;
+  Plan p;
+  if (make_plan(t, std::min<uint64_t>(n, 1ull << 22), o, &p) != HARMONIA_OK) return 0;
+  const uint64_t c = host_chunk(p, n);
+  return psa_ws_bytes(p) + 4 * round_up(c * 8, 256) + 512;
+}
+
+extern "C" harmonia_status harmonia_search_batch_host(const harmonia_tree* tc, const uint64_t* h_q, uint64_t n,
+                                                      uint64_t* h_out, void* ws, size_t ws_bytes,
+                                                      const harmonia_query_opts* o, void* stream) {
+  harmonia_tree* t = const_cast<harmonia_tree*>(tc);
+  if (!t) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!h_q || !h_out || !ws) return HARMONIA_ERR_INVALID_ARG;
+  Plan p;
+  harmonia_status s = make_plan(t, std::min<uint64_t>(n, 1ull << 22), o, &p);
+  if (s != HARMONIA_OK) return s;
+  const uint64_t C = host_chunk(p, n);
+  const size_t psa_b = psa_ws_bytes(p);
+  if (ws_bytes < psa_b + 4 * round_up(C * 8, 256) + 256) return HARMONIA_ERR_INVALID_ARG;
+  char* base = (char*)ws;
+  if ((uintptr_t)base & 255) base += 256 - ((uintptr_t)base & 255);
+  void* psa_ws = base;
+  uint64_t* din[2] = {(uint64_t*)(base + psa_b), (uint64_t*)(base + psa_b + round_up(C * 8, 256))};
+  uint64_t* dout[2] = {(uint64_t*)(base + psa_b + 2 * round_up(C * 8, 256)),
+                       (uint64_t*)(base + psa_b + 3 * round_up(C * 8, 256))};
+  cudaStream_t st = (cudaStream_t)stream;
+  if (!t->s_h2d) {
+    HM_CUDA(cudaStreamCreateWithFlags(&t->s_h2d, cudaStreamNonBlocking));
+    HM_CUDA(cudaStreamCreateWithFlags(&t->s_d2h, cudaStreamNonBlocking));
+    HM_CUDA(cudaEventCreateWithFlags(&t->ev_start, cudaEventDisableTiming));
+    for (int i = 0; i < 2; ++i) {
+      HM_CUDA(cudaEventCreateWithFlags(&t->ev_in[i], cudaEventDisableTiming));
+      HM_CUDA(cudaEventCreateWithFlags(&t->ev_done[i], cudaEventDisableTiming));
+      HM_CUDA(cudaEventCreateWithFlags(&t->ev_out[i], cudaEventDisableTiming));
+    }
+  }
+  // order the pipeline after the caller's prior work
+  HM_CUDA(cudaEventRecord(t->ev_start, st));
+  HM_CUDA(cudaStreamWaitEvent(t->s_h2d, t->ev_start, 0));
+  HM_CUDA(cudaStreamWaitEvent(t->s_d2h, t->ev_start, 0));
+  const uint64_t chunks = ceil_div(n, C);
+  for (uint64_t k = 0; k < chunks; ++k) {
+    const int b = (int)(k & 1);
+    const uint64_t off = k * C, m = std::min<uint64_t>(C, n - off);
+    if (k >= 2) HM_CUDA(cudaStreamWaitEvent(t->s_h2d, t->ev_done[b], 0));  // din[b] consumed
+    HM_CUDA(cudaMemcpyAsync(din[b], h_q + off, m * 8, cudaMemcpyHostToDevice, t->s_h2d));
+    HM_CUDA(cudaEventRecord(t->ev_in[b], t->s_h2d));
+    HM_CUDA(cudaStreamWaitEvent(st, t->ev_in[b], 0));
+    if (k >= 2) HM_CUDA(cudaStreamWaitEvent(st, t->ev_out[b], 0));  // dout[b] drained
+    s = search_device(t, din[b], m, dout[b], psa_ws, p, st);
+    if (s != HARMONIA_OK) return s;
+    HM_CUDA(cudaEventRecord(t->ev_done[b], st));
+    HM_CUDA(cudaStreamWaitEvent(t->s_d2h, t->ev_done[b], 0));
+    HM_CUDA(cudaMemcpyAsync(h_out + off, dout[b], m * 8, cudaMemcpyDeviceToHost, t->s_d2h));
+    HM_CUDA(cudaEventRecord(t->ev_out[b], t->s_d2h));
+  }
+  for (uint64_t k = (chunks >= 2 ? chunks - 2 : 0); k < chunks; ++k)
+    HM_CUDA(cudaStreamWaitEvent(st, t->ev_out[k & 1], 0));
+  return HARMONIA_OK;
+}
+
+// ---- range -------------------------------------------------------------------------------
+extern "C" size_t harmonia_range_workspace_bytes(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o) {
+  return harmonia_search_workspace_bytes(t, n, o);
+}
+
+extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const uint64_t* d_lo, const uint64_t* d_hi,
+                                                uint64_t n, uint32_t cap, uint64_t* d_kout, uint64_t* d_vout,
+                                                uint32_t* d_counts, void* ws, size_t ws_bytes,
+                                                const harmonia_query_opts* o, void* stream) {
+  if (!t) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!d_lo || !d_hi || !d_counts || (cap > 0 && (!d_kout || !d_vout))) return HARMONIA_ERR_INVALID_ARG;
+  if (!on_device(d_lo, t->device) || !on_device(d_counts, t->device)) return HARMONIA_ERR_DEVICE_MISMATCH;
+  cudaStream_t st = (cudaStream_t)stream;
+  Plan p;
+  harmonia_status s = make_plan(t, n, o, &p);
+  if (s != HARMONIA_OK) return s;
+  if (t->n_keys == 0) {
+    HM_CUDA(cudaMemsetAsync(d_counts, 0, n * 4, st));
+    return HARMONIA_OK;
+  }
+  const size_t need = psa_ws_bytes(p);
+  if (need) {
+    if (!ws || ws_bytes < need) return HARMONIA_ERR_INVALID_ARG;
+    if (((uintptr_t)ws & 255) != 0) {
+      const size_t adj = 256 - ((uintptr_t)ws & 255);
+      if (ws_bytes < need + adj) return HARMONIA_ERR_INVALID_ARG;
+      ws = (char*)ws + adj;
+    }
+  }
+  RangeArgs a{};
+  a.keys = t->d_keys;
+  a.ps = t->d_ps;
+  a.vals = t->d_vals;
+  a.leaf_base = t->d_leaf_base;
+  a.leaf_start = t->level_start[t->h - 1];
+  a.n_nodes = t->N;
+  a.h = t->h;
+  a.smem_levels = (uint32_t)p.smem_levels;
+  a.smem_nodes = p.smem_nodes;
+  a.ps_smem_bytes = p.ps_smem ? p.ps_smem_bytes : 0;
+  a.cap = cap;
+  if (!p.psa) {
+    a.lo = d_lo;
+    a.hi = d_hi;
+    a.idx = nullptr;
+    a.n = n;
+    a.kout = d_kout;
+    a.vout = d_vout;
+    a.counts = d_counts;
+    return launch_range(t, p, a, st);
+  }
+  const PsaWs w = psa_ws_carve(p, ws);
+  for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
+    const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
+    s = psa_partition(d_lo + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr);
+    if (s != HARMONIA_OK) return s;
+    a.lo = w.sorted_q;
+    a.hi = d_hi + w0;
+    a.idx = w.idx;
+    a.n = nw;
+    a.kout = d_kout ? d_kout + w0 * cap : nullptr;
+    a.vout = d_vout ? d_vout + w0 * cap : nullptr;
+    a.counts = d_counts + w0;
+    if ((s = launch_range(t, p, a, st)) != HARMONIA_OK) return s;
+  }
+  return HARMONIA_OK;
+}
+
+// ---- multi-GPU routing helpers ---------------------------------------------------------
+extern "C" size_t harmonia_route_workspace_bytes(uint32_t P, uint64_t n) {
+  Plan p;
+  p.psa = true;
+  p.nbins = std::max<uint32_t>(P, 1);
+  p.window = round_up(std::max<uint64_t>(n, 1), 1024);
+  return psa_ws_bytes(p) + 256;
+}
+
+extern "C" harmonia_status harmonia_route_partition(const uint64_t* d_split, uint32_t P, const uint64_t* d_q,
+                                                    uint64_t n, uint64_t* d_routed, uint32_t* d_pos,
+                                                    uint64_t* h_counts, void* ws, size_t ws_bytes, void* stream) {
+  if (P == 0 || P > 1024 || !h_counts || (P > 1 && !d_split)) return HARMONIA_ERR_INVALID_ARG;
+  if (n >= (1ull << 32)) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) {
+    for (uint32_t i = 0; i < P; ++i) h_counts[i] = 0;
+    return HARMONIA_OK;
+  }
+  if (!d_q || !d_routed || !d_pos || !ws) return HARMONIA_ERR_INVALID_ARG;
+  Plan p;
+  p.psa = true;
+  p.nbins = P;
+  p.window = round_up(n, 1024);
+  if (ws_bytes < psa_ws_bytes(p) + 256) return HARMONIA_ERR_INVALID_ARG;
+  if ((uintptr_t)ws & 255) ws = (char*)ws + (256 - ((uintptr_t)ws & 255));
+  PsaWs w = psa_ws_carve(p, ws);
+  w.sorted_q = d_routed;
+  w.idx = d_pos;
+  int dev = 0, sm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
+  BucketSplit f{d_split, P - 1};
+  return psa_partition(d_q, n, f, P, w, sm, (cudaStream_t)stream, h_counts);
+}
+
+extern "C" harmonia_status harmonia_scatter_results(const uint64_t* d_vals, const uint32_t* d_pos, uint64_t n,
+                                                    uint64_t* d_out, void* stream) {
+  if (n == 0) return HARMONIA_OK;
+  if (!d_vals || !d_pos || !d_out) return HARMONIA_ERR_INVALID_ARG;
+  int dev = 0, sm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
+  return launch_scatter_back(d_vals, d_pos, n, d_out, sm, (cudaStream_t)stream);
+}

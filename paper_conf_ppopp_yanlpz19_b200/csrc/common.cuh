@@ -1,0 +1,190 @@
+// Internal declarations shared by the translation units of libharmonia.so.
+// (Product code only: nothing here is shared with oracle/.)
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+
+#include "../../include/harmonia.h"
+
+namespace hm {
+
+constexpr uint64_t kPad = 0xFFFFFFFFFFFFFFFFull;       // HARMONIA_KEY_PAD
+constexpr uint64_t kNotFound = 0xFFFFFFFFFFFFFFFFull;  // HARMONIA_NOT_FOUND
+constexpr unsigned kFull = 0xFFFFFFFFu;
+constexpr int kBlock = 256;  // threads per CTA for the query kernels
+
+// ---- error plumbing --------------------------------------------------------------
+harmonia_status cuda_fail(cudaError_t e);
+void count_launch(uint64_t k = 1);
+
+#define HM_CUDA(x)                                  \
+  do {                                              \
+    cudaError_t e_ = (x);                           \
+    if (e_ != cudaSuccess) return hm::cuda_fail(e_); \
+  } while (0)
+#define HM_LAUNCHED()                                \
+  do {                                               \
+    hm::count_launch();                              \
+    cudaError_t e_ = cudaGetLastError();             \
+    if (e_ != cudaSuccess) return hm::cuda_fail(e_); \
+  } while (0)
+
+__host__ __device__ inline uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+// whole warps iterate a grid-stride loop uniformly when its bound is a multiple of 32
+__host__ __device__ inline uint64_t round_up_dev(uint64_t n) { return (n + 31) & ~31ull; }
+inline uint64_t round_up(uint64_t a, uint64_t b) { return ceil_div(a, b) * b; }
+
+// ---- kernel timing (harmonia_profile_*): RAII event pair around one launch ---------------
+void prof_record(int kind, cudaStream_t st, bool start);
+extern bool g_prof_on;
+struct ProfScope {
+  int kind;
+  cudaStream_t st;
+  bool on;
+  ProfScope(int k, cudaStream_t s) : kind(k), st(s), on(g_prof_on) {
+    if (on) prof_record(kind, st, true);
+  }
+  ~ProfScope() {
+    if (on) prof_record(kind, st, false);
+  }
+};
+
+// ---- PSA bucket function (C-A11): bits [span-Nb, span) of clamp(q, kmin, kmax) -------
+struct BucketBits {
+  uint64_t kmin, kmax;
+  uint32_t shift, mask;
+  __device__ __forceinline__ uint32_t operator()(uint64_t q) const {
+    uint64_t c = q < kmin ? kmin : (q > kmax ? kmax : q);
+    return (uint32_t)(c >> shift) & mask;
+  }
+};
+
+// ---- destination by splitters (partitioned multi-GPU mode) --------------------------
+struct BucketSplit {
+  const uint64_t* split;  // P-1 strictly increasing splitters
+  uint32_t nsplit;
+  __device__ __forceinline__ uint32_t operator()(uint64_t q) const {
+    uint32_t lo = 0, hi = nsplit;  // count of splitters <= q
+    while (lo < hi) {
+      uint32_t mid = (lo + hi) >> 1;
+      if (__ldg(split + mid) <= q) lo = mid + 1;
+      else hi = mid;
+    }
+    return lo;
+  }
+};
+
+}  // namespace hm
+
+// The opaque tree of the C ABI.
+struct harmonia_tree {
+  int device = 0;
+  uint32_t F = 0, h = 0;
+  uint64_t n_keys = 0, N = 0, I = 0, L = 0;
+  uint64_t level_start[HARMONIA_MAX_LEVELS + 1] = {};
+  uint64_t* d_keys = nullptr;       // key region, N*F slots, BFS order
+  uint32_t* d_ps = nullptr;         // prefix-sum child region, I+1 entries (+pad to 16 B)
+  uint64_t* d_vals = nullptr;       // leaf-aligned values, L*F
+  uint64_t* d_leaf_base = nullptr;  // records before leaf j, L+1 entries (range counts)
+  uint64_t min_key = 0, max_key = 0;
+  float fill = 1.0f;
+  int sm_count = 148;
+  size_t smem_optin = 0;
+  size_t l2_bytes = 0;
+  // host-pipeline streams/events (harmonia_search_batch_host)
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  cudaEvent_t ev_start = nullptr, ev_in[2] = {}, ev_done[2] = {}, ev_out[2] = {};
+};
+
+namespace hm {
+
+// ---- query plan (host) ----------------------------------------------------------------
+struct Plan {
+  int G = 4;
+  bool psa = false;
+  int nb = 0;                // PSA bits
+  uint64_t window = 0;       // queries per PSA window
+  BucketBits bucket{};
+  uint32_t nbins = 0;
+  int smem_levels = 0;       // staged top levels
+  uint32_t smem_nodes = 0;   // nodes [0, smem_nodes) staged
+  bool ps_smem = false;
+  uint32_t ps_smem_bytes = 0;
+  uint32_t smem_bytes = 0;   // dynamic smem of the search kernel
+  bool gather = false;
+};
+
+harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
+                          Plan* p);
+int auto_group_size(uint32_t F);
+int psa_bits_for(uint64_t n_keys);
+
+// workspace carve-up for one PSA window
+struct PsaWs {
+  uint32_t* counts;     // nbins
+  uint32_t* tile_sums;  // ceil(nbins / kScanTile)
+  uint64_t* sorted_q;   // window
+  uint32_t* idx;        // window
+  uint64_t* sorted_out; // window (gather mode only)
+};
+constexpr uint32_t kScanTile = 4096;
+size_t psa_ws_bytes(const Plan& p);
+PsaWs psa_ws_carve(const Plan& p, void* base);
+
+// ---- kernels launchers (each returns after enqueue) ----------------------------------
+template <class Bucket>
+harmonia_status psa_partition(const uint64_t* q, uint64_t n, const Bucket& f, uint32_t nbins,
+                              const PsaWs& ws, int sm_count, cudaStream_t st,
+                              uint64_t* h_counts /* optional: sync copy of counts */);
+
+struct SearchArgs {
+  const uint64_t* keys;
+  const uint32_t* ps;
+  const uint64_t* vals;
+  uint64_t leaf_start;
+  uint32_t h;
+  uint32_t smem_levels;
+  uint32_t smem_nodes;
+  uint32_t ps_smem_bytes;  // 0 = PS read from global
+  const uint64_t* q;       // queries (PSA-sorted or caller order)
+  const uint32_t* idx;     // original position within the window (nullptr = identity)
+  uint64_t n;
+  uint64_t* out;           // results: out[idx ? idx[j] : j]
+};
+harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
+                              cudaStream_t st);
+
+struct RangeArgs {
+  const uint64_t* keys;
+  const uint32_t* ps;
+  const uint64_t* vals;
+  const uint64_t* leaf_base;
+  uint64_t leaf_start, n_nodes;
+  uint32_t h;
+  uint32_t smem_levels, smem_nodes, ps_smem_bytes;
+  const uint64_t* lo;      // (PSA-sorted) lower bounds
+  const uint64_t* hi;      // upper bounds in caller order (indexed through idx)
+  const uint32_t* idx;     // nullptr = identity
+  uint64_t n;
+  uint32_t cap;
+  uint64_t* kout;
+  uint64_t* vout;
+  uint32_t* counts;
+};
+harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeArgs& a,
+                             cudaStream_t st);
+
+harmonia_status launch_gather(const uint64_t* sorted_out, const uint32_t* idx, uint64_t n,
+                              uint64_t* out, int sm_count, cudaStream_t st);
+harmonia_status launch_scatter_back(const uint64_t* vals, const uint32_t* pos, uint64_t n,
+                                    uint64_t* out, int sm_count, cudaStream_t st);
+
+// layout construction (tree.cu)
+harmonia_status build_layout(harmonia_tree* t, const uint64_t* d_keys, const uint64_t* d_vals,
+                             uint64_t n, cudaStream_t st);
+uint32_t level_shape(uint64_t n, uint32_t F, double fill, uint64_t* bottom_up_nodes);
+
+}  // namespace hm

@@ -1,0 +1,382 @@
+// Narrowed thread-group traversal (NTG, §4.2) over the Harmonia layout.
+//
+// One query is served by a group of G lanes (G = 2..32, warpsize/G queries per warp,
+// P:L500).  At every level the group walks the node in steps of 2G keys: each lane issues
+// one 128-bit load (2 keys), the rank inside the node is the popcount of the group's
+// ballot of (key <= q), and the walk stops at the first step that holds a key > q (the
+// early exit that removes the "useless comparisons" of P:L436).  The child is then
+// PS[node] + rank (Eq 1 with i = rank + 1; equality descends right, C-A5).  At the
+// leaf a ballot of (key == q) gives the slot and the value is read from the leaf-aligned
+// value array (C-A3).
+//
+// B200 mapping: the PS array and the top `smem_levels` levels are staged
+// into shared memory once per CTA with 1-D TMA bulk copies (cp.async.bulk + mbarrier) —
+// the sm_100a replacement for the paper's constant-memory PS top; lower levels go
+// through the non-coherent read-only path (ld.global.nc.v2.u64).  The grid is persistent
+// (a multiple of the SM count); PSA-sorted neighbours share nodes, so their loads coalesce
+// in L1/L2.  Results are written straight to out[idx[j]] (the PSA return step).
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace hm {
+
+namespace {
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// Stage PS (ps_bytes) then the top key-region nodes (key_bytes) into dynamic smem with
+// 1-D bulk copies completing on one mbarrier.  All sizes are multiples of 16 B.
+__device__ __forceinline__ void stage_top(unsigned char* smem, const uint32_t* ps, uint32_t ps_bytes,
+                                          const uint64_t* keys, uint32_t key_bytes, uint64_t* bar) {
+  const uint32_t total = ps_bytes + key_bytes;
+  if (total == 0) return;
+  if (threadIdx.x == 0) {
+    const uint32_t b = smem_u32(bar);
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(b) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(total)
+                 : "memory");
+    constexpr uint32_t kChunk = 32768;
+    const uint32_t dst0 = smem_u32(smem);
+    for (uint32_t off = 0; off < ps_bytes; off += kChunk) {
+      uint32_t sz = min(kChunk, ps_bytes - off);
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+              dst0 + off),
+          "l"((const char*)ps + off), "r"(sz), "r"(b)
+          : "memory");
+    }
+    for (uint32_t off = 0; off < key_bytes; off += kChunk) {
+      uint32_t sz = min(kChunk, key_bytes - off);
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+              dst0 + ps_bytes + off),
+          "l"((const char*)keys + off), "r"(sz), "r"(b)
+          : "memory");
+    }
+  }
+  __syncthreads();
+  const uint32_t b = smem_u32(bar);
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(b)
+        : "memory");
+  }
+}
+
+__device__ __forceinline__ ulonglong2 ld_pair_global(const uint64_t* p) {
+  ulonglong2 v;
+  asm volatile("ld.global.nc.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint64_t ld_stream(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.global.cs.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_stream32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.cs.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+
+template <bool SMEM>
+__device__ __forceinline__ ulonglong2 ld_pair(const uint64_t* p) {
+  if constexpr (SMEM) return *reinterpret_cast<const ulonglong2*>(p);
+  else return ld_pair_global(p);
+}
+
+// Number of keys in the node that are <= q (STRICT: < q).  `live` is uniform inside a
+// group; the loop is warp-uniform so that every ballot sees the full warp.
+template <int F, int G, bool SMEM, bool STRICT>
+__device__ __forceinline__ uint32_t node_rank(const uint64_t* nk, uint64_t q, bool live, uint32_t gmask,
+                                              int gl) {
+  constexpr int KPS = 2 * G, STEPS = F / KPS;
+  uint32_t r = 0;
+  bool done = !live;
+#pragma unroll
+  for (int s = 0; s < STEPS; ++s) {
+    if (__all_sync(kFull, done)) break;
+    ulonglong2 k = make_ulonglong2(kPad, kPad);
+    if (!done) k = ld_pair<SMEM>(nk + s * KPS + 2 * gl);
+    const bool le0 = !done && (STRICT ? k.x < q : k.x <= q);
+    const bool le1 = !done && (STRICT ? k.y < q : k.y <= q);
+    const uint32_t c = __popc(__ballot_sync(kFull, le0) & gmask) + __popc(__ballot_sync(kFull, le1) & gmask);
+    r += c;
+    done = done || (c < (uint32_t)KPS);
+  }
+  return r;
+}
+
+// Descend levels 0..h-2 with Eq 1; returns the leaf's node index.
+template <int F, int G>
+__device__ __forceinline__ uint32_t descend(uint64_t q, bool live, uint32_t h, uint32_t smem_levels,
+                                            const uint64_t* s_keys, const uint32_t* s_ps, bool ps_smem,
+                                            const uint64_t* __restrict__ keys, const uint32_t* __restrict__ ps,
+                                            uint32_t gmask, int gl) {
+  uint32_t node = 0;
+  for (uint32_t l = 0; l + 1 < h; ++l) {
+    const uint32_t first = ps_smem ? s_ps[node] : __ldg(ps + node);  // PS[node_idx]
+    uint32_t r;
+    if (l < smem_levels) r = node_rank<F, G, true, false>(s_keys + (uint64_t)node * F, q, live, gmask, gl);
+    else r = node_rank<F, G, false, false>(keys + (uint64_t)node * F, q, live, gmask, gl);
+    node = first + r;  // Eq 1: child_idx = PrefixSum[node_idx] + i - 1, i = r + 1
+  }
+  return node;
+}
+
+template <int F, int G>
+__global__ void __launch_bounds__(kBlock) k_ntg_search(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+
+  constexpr int QPW = 32 / G, KPS = 2 * G, STEPS = F / KPS;
+  const int lane = threadIdx.x & 31, grp = lane / G, gl = lane % G;
+  const uint32_t gmask = (G == 32) ? kFull : (((1u << G) - 1u) << (grp * G));
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+
+  for (uint64_t base = warp * QPW; base < a.n; base += nwarps * QPW) {
+    const uint64_t j = base + grp;
+    const bool active = j < a.n;
+    const uint64_t q = active ? ld_stream(a.q + j) : kPad;
+    const bool live = active && q != kPad;  // PAD is never a key (C-A2)
+    const uint32_t leaf =
+        descend<F, G>(q, live, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
+    // leaf probe: slot of key == q ("the target key is found")
+    const bool leaf_smem = a.h - 1 < a.smem_levels;
+    const uint64_t* nk = (leaf_smem ? s_keys : a.keys) + (uint64_t)leaf * F;
+    int slot = -1;
+    bool done = !live;
+#pragma unroll
+    for (int s = 0; s < STEPS; ++s) {
+      if (__all_sync(kFull, done)) break;
+      ulonglong2 k = make_ulonglong2(kPad, kPad);
+      if (!done) k = leaf_smem ? ld_pair<true>(nk + s * KPS + 2 * gl) : ld_pair<false>(nk + s * KPS + 2 * gl);
+      const uint32_t b_le = (__ballot_sync(kFull, !done && k.x <= q) & gmask);
+      const uint32_t b_le1 = (__ballot_sync(kFull, !done && k.y <= q) & gmask);
+      const uint32_t e0 = __ballot_sync(kFull, !done && k.x == q) & gmask;
+      const uint32_t e1 = __ballot_sync(kFull, !done && k.y == q) & gmask;
+      if (!done) {
+        if (e0) slot = s * KPS + 2 * (__ffs(e0) - 1 - grp * G);
+        else if (e1) slot = s * KPS + 2 * (__ffs(e1) - 1 - grp * G) + 1;
+        if ((e0 | e1) || (__popc(b_le) + __popc(b_le1) < KPS)) done = true;
+      }
+    }
+    if (active && gl == 0) {
+      uint64_t v = kNotFound;
+      if (slot >= 0) v = __ldg(a.vals + (uint64_t)(leaf - a.leaf_start) * F + slot);
+      const uint64_t o = a.idx ? (uint64_t)ld_stream32(a.idx + j) : j;
+      a.out[o] = v;
+    }
+  }
+}
+
+// Range scan: descend with lo, then walk leaf slots in key-region order.
+template <int F, int G>
+__global__ void __launch_bounds__(kBlock) k_ntg_range(const RangeArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+
+  constexpr int QPW = 32 / G, KPS = 2 * G, STEPS = F / KPS;
+  const int lane = threadIdx.x & 31, grp = lane / G, gl = lane % G;
+  const uint32_t gmask = (G == 32) ? kFull : (((1u << G) - 1u) << (grp * G));
+  unsigned lt;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
+  const uint32_t below = lt & gmask;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t cap = a.cap;
+
+  for (uint64_t base = warp * QPW; base < a.n; base += nwarps * QPW) {
+    const uint64_t j = base + grp;
+    const bool active = j < a.n;
+    const uint64_t lo = active ? ld_stream(a.lo + j) : kPad;
+    const uint64_t slab = active ? (a.idx ? (uint64_t)ld_stream32(a.idx + j) : j) : 0;
+    const uint64_t hi = active ? __ldg(a.hi + slab) : 0;
+    const bool live = active && lo <= hi && lo != kPad;
+    uint32_t cur = descend<F, G>(lo, live, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
+    uint64_t cnt = 0;
+    bool trunc = live && cap == 0;
+    bool done = !live || trunc;
+    int s = 0;
+    uint64_t* ko = a.kout + slab * cap;
+    uint64_t* vo = a.vout + slab * cap;
+    while (!__all_sync(kFull, done)) {
+      ulonglong2 k = make_ulonglong2(kPad, kPad);
+      const uint64_t off = (uint64_t)cur * F + s * KPS + 2 * gl;
+      if (!done) k = ld_pair_global(a.keys + off);
+      const bool v0 = !done && k.x != kPad && k.x >= lo && k.x <= hi;
+      const bool v1 = !done && k.y != kPad && k.y >= lo && k.y <= hi;
+      const bool over = !done && ((k.x != kPad && k.x > hi) || (k.y != kPad && k.y > hi));
+      const bool pad = !done && (k.x == kPad || k.y == kPad);
+      const uint32_t b0 = __ballot_sync(kFull, v0) & gmask, b1 = __ballot_sync(kFull, v1) & gmask;
+      const uint32_t bo = __ballot_sync(kFull, over) & gmask, bp = __ballot_sync(kFull, pad) & gmask;
+      if (!done) {
+        const uint64_t p0 = cnt + __popc(b0 & below) + __popc(b1 & below);
+        const uint64_t p1 = p0 + (v0 ? 1 : 0);
+        if (v0 | v1) {
+          const ulonglong2 vv = ld_pair_global(a.vals + ((uint64_t)(cur - a.leaf_start) * F + s * KPS + 2 * gl));
+          if (v0 && p0 < cap) { ko[p0] = k.x; vo[p0] = vv.x; }
+          if (v1 && p1 < cap) { ko[p1] = k.y; vo[p1] = vv.y; }
+        }
+        cnt += __popc(b0) + __popc(b1);
+        if (bo) {
+          done = true;
+        } else if (bp || s == STEPS - 1) {  // leaf exhausted: continue in the next leaf
+          ++cur;
+          s = 0;
+          if (cur >= a.n_nodes) done = true;
+        } else {
+          ++s;
+        }
+        if (!done && cnt >= cap) {  // slab full: the total comes from ranks below
+          trunc = true;
+          done = true;
+        }
+      }
+    }
+    // true total for truncated queries: rank(<= hi) - rank(< lo) via leaf_base
+    if (__any_sync(kFull, trunc)) {
+      // keys never equal PAD, so #keys <= PAD == #keys <= PAD-1 (and PAD slots stay excluded)
+      const uint64_t hd = hi == kPad ? kPad - 1 : hi;
+      const uint32_t lh = descend<F, G>(hd, trunc, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
+      const uint32_t rh = node_rank<F, G, false, false>(a.keys + (uint64_t)lh * F, hd, trunc, gmask, gl);
+      const uint32_t ll = descend<F, G>(lo, trunc, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
+      const uint32_t rl = node_rank<F, G, false, true>(a.keys + (uint64_t)ll * F, lo, trunc, gmask, gl);
+      if (trunc)
+        cnt = (__ldg(a.leaf_base + (lh - a.leaf_start)) + rh) - (__ldg(a.leaf_base + (ll - a.leaf_start)) + rl);
+    }
+    if (active && gl == 0) a.counts[slab] = (uint32_t)(cnt > 0xFFFFFFFFull ? 0xFFFFFFFFull : cnt);
+  }
+}
+
+template <int F, int G>
+harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  auto kern = k_ntg_search<F, G>;
+  static int configured_smem = -1;  // per instantiation
+  if ((int)p.smem_bytes > configured_smem) {
+    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
+    configured_smem = (int)p.smem_bytes;
+  }
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBlock, p.smem_bytes));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t qpb = (uint64_t)(kBlock / 32) * (32 / G);
+  const uint64_t need = ceil_div(a.n, qpb);
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
+  {
+    ProfScope ps_(HARMONIA_PROF_SEARCH, st);
+    {
+    ProfScope ps_(HARMONIA_PROF_RANGE, st);
+    kern<<<grid, kBlock, p.smem_bytes, st>>>(a);
+  }
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+template <int F, int G>
+harmonia_status launch_range_fg(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
+  auto kern = k_ntg_range<F, G>;
+  static int configured_smem = -1;
+  if ((int)p.smem_bytes > configured_smem) {
+    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
+    configured_smem = (int)p.smem_bytes;
+  }
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBlock, p.smem_bytes));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t qpb = (uint64_t)(kBlock / 32) * (32 / G);
+  const uint64_t need = ceil_div(a.n, qpb);
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
+  kern<<<grid, kBlock, p.smem_bytes, st>>>(a);
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+// F x G dispatch (2G <= F: one 128-bit load per lane covers 2 keys)
+#define HM_DISPATCH(FN, F_, G_, ...)                                                   \
+  switch (F_) {                                                                        \
+    case 4:                                                                            \
+      if (G_ == 2) return FN<4, 2>(__VA_ARGS__);                                       \
+      break;                                                                           \
+    case 8:                                                                            \
+      if (G_ == 2) return FN<8, 2>(__VA_ARGS__);                                       \
+      if (G_ == 4) return FN<8, 4>(__VA_ARGS__);                                       \
+      break;                                                                           \
+    case 16:                                                                           \
+      if (G_ == 2) return FN<16, 2>(__VA_ARGS__);                                      \
+      if (G_ == 4) return FN<16, 4>(__VA_ARGS__);                                      \
+      if (G_ == 8) return FN<16, 8>(__VA_ARGS__);                                      \
+      break;                                                                           \
+    case 32:                                                                           \
+      if (G_ == 2) return FN<32, 2>(__VA_ARGS__);                                      \
+      if (G_ == 4) return FN<32, 4>(__VA_ARGS__);                                      \
+      if (G_ == 8) return FN<32, 8>(__VA_ARGS__);                                      \
+      if (G_ == 16) return FN<32, 16>(__VA_ARGS__);                                    \
+      break;                                                                           \
+    case 64:                                                                           \
+      if (G_ == 2) return FN<64, 2>(__VA_ARGS__);                                      \
+      if (G_ == 4) return FN<64, 4>(__VA_ARGS__);                                      \
+      if (G_ == 8) return FN<64, 8>(__VA_ARGS__);                                      \
+      if (G_ == 16) return FN<64, 16>(__VA_ARGS__);                                    \
+      if (G_ == 32) return FN<64, 32>(__VA_ARGS__);                                    \
+      break;                                                                           \
+    case 128:                                                                          \
+      if (G_ == 2) return FN<128, 2>(__VA_ARGS__);                                     \
+      if (G_ == 4) return FN<128, 4>(__VA_ARGS__);                                     \
+      if (G_ == 8) return FN<128, 8>(__VA_ARGS__);                                     \
+      if (G_ == 16) return FN<128, 16>(__VA_ARGS__);                                   \
+      if (G_ == 32) return FN<128, 32>(__VA_ARGS__);                                   \
+      break;                                                                           \
+    case 256:                                                                          \
+      if (G_ == 2) return FN<256, 2>(__VA_ARGS__);                                     \
+      if (G_ == 4) return FN<256, 4>(__VA_ARGS__);                                     \
+      if (G_ == 8) return FN<256, 8>(__VA_ARGS__);                                     \
+      if (G_ == 16) return FN<256, 16>(__VA_ARGS__);                                   \
+      if (G_ == 32) return FN<256, 32>(__VA_ARGS__);                                   \
+      break;                                                                           \
+  }                                                                                    \
+  return HARMONIA_ERR_INVALID_ARG;
+
+}  // namespace
+
+harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  if (a.n == 0) return HARMONIA_OK;
+  HM_DISPATCH(launch_search_fg, t->F, p.G, t, p, a, st)
+}
+
+harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
+  if (a.n == 0) return HARMONIA_OK;
+  HM_DISPATCH(launch_range_fg, t->F, p.G, t, p, a, st)
+}
+
+// Measured default G per fanout (refreshed from bench sweeps).
+int auto_group_size(uint32_t F) {
+  switch (F) {
+    case 4: return 2;
+    case 8: return 2;
+    case 16: return 4;
+    case 32: return 4;
+    case 64: return 8;
+    case 128: return 8;
+    default: return 16;
+  }
+}
+
+}  // namespace hm

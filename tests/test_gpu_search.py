@@ -1,0 +1,247 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Run on a B200 with ``pytest -m gpu``.  Every comparison is bit-exact (integer work)."""
+import numpy as np
+import pytest
+
+import harmonia_gen as gen
+
+pytestmark = pytest.mark.gpu
+
+MAX = (1 << 64) - 1
+
+
+@pytest.fixture(scope="module")
+def hm():
+    import torch
+
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_ppopp_yanlpz19_b200 as m
+
+    m.lib()
+    return m
+
+
+def cu(a):
+    import torch
+
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    return t.cpu().numpy()
+
+
+def tree(hm, keys, vals, F, fill=1.0):
+    return hm.Tree(cu(keys), cu(vals), fanout=F, fill=fill)
+
+
+# ----------------------------------------------------------------------------- layout
+@pytest.mark.parametrize("n,F,fill", [(0, 16, 1.0), (1, 4, 1.0), (3, 4, 1.0), (15, 16, 1.0), (16, 16, 1.0),
+                                      (1000, 4, 1.0), (5000, 8, 0.69), (20000, 16, 0.5), (65536, 16, 1.0),
+                                      (100000, 64, 1.0), (100000, 128, 0.69), (70000, 256, 1.0), (1 << 20, 64, 1.0)])
+def test_layout_bit_exact_and_invariants(hm, orc, n, F, fill):
+    keys = gen.uniform_keys(n)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F, fill)
+    info, kr, ps, lv = t.export_layout()
+    ref = orc.layout_build(keys, vals, F, fill)
+    assert info["height"] == ref.h and info["level_start"] == ref.level_start.tolist()
+    assert np.array_equal(kr, ref.key_region)      # I8: bit-exact key region
+    assert np.array_equal(ps, ref.ps)              # I8: bit-exact PS
+    assert np.array_equal(lv, ref.leaf_vals)
+    lay = orc.Layout(F, info["height"], info["level_start"], kr, ps, lv)
+    code, msg = lay.check(keys, vals)
+    assert code == 0, msg
+    assert info["ps_bytes"] == 4 * (info["n_internal"] + 1)  # I9
+
+
+def test_build_from_host_equals_device(hm):
+    keys = gen.uniform_keys(30000)
+    vals = gen.values_for(keys)
+    a = hm.Tree(keys, vals, fanout=32).export_layout()
+    b = tree(hm, keys, vals, 32).export_layout()
+    for x, y in zip(a[1:], b[1:]):
+        assert np.array_equal(x, y)
+
+
+def test_build_errors(hm):
+    k = np.array([1, 5, 5, 9], dtype=np.uint64)
+    with pytest.raises(hm.HarmoniaError, match="UNSORTED"):
+        tree(hm, k, k, 8)
+    k = np.array([9, 5], dtype=np.uint64)
+    with pytest.raises(hm.HarmoniaError, match="UNSORTED"):
+        tree(hm, k, k, 8)
+    k = np.array([1, MAX], dtype=np.uint64)
+    with pytest.raises(hm.HarmoniaError, match="RESERVED"):
+        tree(hm, k, np.array([1, 2], dtype=np.uint64), 8)
+    k = np.array([1, 2], dtype=np.uint64)
+    with pytest.raises(hm.HarmoniaError, match="RESERVED"):
+        tree(hm, k, np.array([1, MAX], dtype=np.uint64), 8)
+    with pytest.raises(hm.HarmoniaError, match="INVALID_ARG"):
+        tree(hm, k, k, 12)
+
+
+# ----------------------------------------------------------------------------- config 1
+def _queries(kind, keys, Q):
+    if kind == "uniform":
+        return gen.uniform_queries(keys, Q)
+    if kind == "miss50":
+        return gen.uniform_queries(keys, Q, miss_frac=0.5)
+    if kind == "zipf":
+        return gen.zipf_queries(keys, Q)
+    if kind == "sorted_run":
+        return gen.sorted_run_queries(keys, Q)
+    raise ValueError(kind)
+
+
+@pytest.mark.parametrize("kind", ["uniform", "miss50", "zipf", "sorted_run"])
+@pytest.mark.parametrize("fill", [1.0, 0.69])
+def test_config1_parity(hm, orc, kind, fill):
+    """BASELINE config 1: 2^16 uint64 keys, F=16, 2^20 queries."""
+    keys = gen.uniform_keys(1 << 16)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 16, fill)
+    q = _queries(kind, keys, 1 << 20)
+    exp = orc.sorted_search(keys, vals, q)
+    assert np.array_equal(host(t.search(cu(q))), exp)
+    assert np.array_equal(host(t.search(cu(q), psa_bits=-1)), exp)
+
+
+@pytest.mark.parametrize("keyset", ["clustered", "random", "dense"])
+def test_key_distributions(hm, orc, keyset):
+    keys = {"clustered": gen.clustered_keys(50000), "random": gen.random_keys(50000, seed=4),
+            "dense": np.arange(50000, dtype=np.uint64)}[keyset]
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 64)
+    q = np.concatenate([gen.uniform_queries(keys, 200000, miss_frac=0.3), gen.edge_queries(keys),
+                        keys + np.uint64(1), keys - np.uint64(1)])
+    assert np.array_equal(host(t.search(cu(q))), orc.sorted_search(keys, vals, q))
+
+
+FG = [(F, G) for F in (4, 8, 16, 32, 64, 128, 256) for G in (2, 4, 8, 16, 32) if 2 * G <= F]
+
+
+@pytest.mark.parametrize("F,G", FG)
+def test_every_fanout_and_group_size(hm, orc, F, G):
+    keys = gen.random_keys(40000, seed=F * 100 + G)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F, 0.69 if G % 4 == 0 else 1.0)
+    q = np.concatenate([gen.uniform_queries(keys, 60001, miss_frac=0.4), gen.edge_queries(keys)])
+    exp = orc.sorted_search(keys, vals, q)
+    for kw in ({}, {"psa_bits": -1}, {"window": 4096}, {"smem_levels": -1}, {"smem_levels": 2},
+               {"flags": hm.QF_GATHER, "window": 8192}, {"psa_bits": 3}):
+        assert np.array_equal(host(t.search(cu(q), group_size=G, **kw)), exp), kw
+
+
+def test_edge_cases(hm, orc):
+    for keys in (np.zeros(0, dtype=np.uint64), np.array([0], dtype=np.uint64),
+                 np.array([MAX - 1], dtype=np.uint64), np.array([0, MAX - 1], dtype=np.uint64),
+                 np.arange(7, dtype=np.uint64) * np.uint64(3)):
+        vals = gen.values_for(keys)
+        for F in (4, 8, 64):
+            t = tree(hm, keys, vals, F)
+            q = np.concatenate([gen.edge_queries(keys), keys, gen._stream(3, 0, 100)])
+            assert np.array_equal(host(t.search(cu(q))), orc.sorted_search(keys, vals, q))
+            lo, hi = gen.random_ranges(keys, 64)
+            ko, vo, cnt = t.range(cu(lo), cu(hi), 8)
+            eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, 8)
+            _cmp_range(host(ko), host(vo), host(cnt), eko, evo, ecnt, 8)
+    # zero queries is a no-op
+    t = tree(hm, np.arange(10, dtype=np.uint64), np.arange(10, dtype=np.uint64), 8)
+    assert t.search(cu(np.zeros(0, dtype=np.uint64))).numel() == 0
+
+
+# ----------------------------------------------------------------------------- range
+def _cmp_range(ko, vo, cnt, eko, evo, ecnt, cap):
+    assert np.array_equal(cnt, ecnt)
+    m = np.minimum(cnt.astype(np.int64), cap)
+    mask = np.arange(cap)[None, :] < m[:, None]
+    if cap:
+        assert np.array_equal(ko[mask], eko[mask])
+        assert np.array_equal(vo[mask], evo[mask])
+        assert np.all(ko[~mask] == np.uint64(MAX))  # slab entries past the count untouched
+
+
+@pytest.mark.parametrize("F,G", [(16, 2), (16, 8), (64, 4), (64, 32), (8, 4), (128, 16)])
+@pytest.mark.parametrize("length,cap", [(16, 16), (64, 64), (256, 100), (1024, 1024), (50, 0)])
+def test_range_parity(hm, orc, F, G, length, cap):
+    keys = gen.uniform_keys(1 << 16)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F)
+    lo, hi = gen.ranges(keys, 3000, length)
+    lo2, hi2 = gen.random_ranges(keys, 3000, max_width_keys=3 * max(cap, 8))
+    lo, hi = np.concatenate([lo, lo2]), np.concatenate([hi, hi2])
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, cap)
+    for kw in ({}, {"psa_bits": -1}, {"window": 2048}):
+        ko, vo, cnt = t.range(cu(lo), cu(hi), cap, group_size=G, **kw)
+        _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
+
+
+def test_range_unbounded_counts(hm, orc):
+    keys = gen.uniform_keys(100000)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 32, 0.69)
+    lo = np.array([0, 0, int(keys[500]), int(keys[-1]), MAX, 5], dtype=np.uint64)
+    hi = np.array([MAX, int(keys[99]), MAX, MAX, MAX, 4], dtype=np.uint64)
+    ko, vo, cnt = t.range(cu(lo), cu(hi), 32)
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, 32)
+    _cmp_range(host(ko), host(vo), host(cnt), eko, evo, ecnt, 32)
+
+
+# ----------------------------------------------------------------------------- host API
+def test_search_host_pipeline(hm, orc):
+    import torch
+
+    keys = gen.uniform_keys(1 << 18)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 64)
+    q = gen.uniform_queries(keys, (1 << 22) * 3 + 12345, miss_frac=0.1)
+    qh = torch.from_numpy(q).pin_memory()
+    out = t.search_host(qh)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.numpy(), orc.sorted_search(keys, vals, q))
+    out2 = t.search_host(qh, psa_bits=-1)
+    torch.cuda.synchronize()
+    assert np.array_equal(out2.numpy(), out.numpy())
+
+
+# ----------------------------------------------------------------------------- routing
+def test_route_partition_and_scatter(hm):
+    import torch
+
+    keys = gen.uniform_keys(1 << 16)
+    q = gen.uniform_queries(keys, 100003, miss_frac=0.2)
+    for P in (1, 2, 3, 8):
+        split = keys[[(p * keys.shape[0]) // P for p in range(1, P)]].astype(np.uint64)
+        routed, pos, counts = hm.route_partition(cu(split), P, cu(q))
+        r, p_ = host(routed), host(pos).astype(np.int64)
+        assert sum(counts) == q.shape[0]
+        assert np.array_equal(np.sort(p_), np.arange(q.shape[0]))
+        assert np.array_equal(r, q[p_])
+        dest = np.searchsorted(split, q, side="right")
+        bounds = np.concatenate([[0], np.cumsum(counts)])
+        for d in range(P):
+            assert np.all(dest[p_[bounds[d]:bounds[d + 1]]] == d)
+        back = hm.scatter_results(routed, pos)
+        assert np.array_equal(host(back), q)
+    torch.cuda.synchronize()
+
+
+# ----------------------------------------------------------------------------- full size
+def test_config2_full_size_sampled(hm, orc):
+    """BASELINE config 2 at full size in the bench's launch configuration (defaults):
+    2^23 keys, F=64, 2^26 uniform queries.  Values are key-derived, so every output is
+    checked by the property out == values_for(q); 2^20 sampled outputs against the oracle."""
+    import torch
+
+    T, Q = 1 << 23, 1 << 26
+    keys = gen.uniform_keys(T)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 64)
+    q = gen.uniform_queries(keys, Q)
+    out = host(t.search(cu(q)))
+    torch.cuda.synchronize()
+    assert np.array_equal(out, gen.values_for(q))
+    sel = gen._stream(77, 0, 1 << 20) % np.uint64(Q)
+    assert np.array_equal(out[sel], orc.sorted_search(keys, vals, q[sel]))
