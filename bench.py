@@ -284,12 +284,38 @@ def main():
     def step():
         t.search(q, out, opts=opts)
 
+    if a.sweep:
+        for spec in a.sweep.split(";"):
+            kw = dict(group_size=a.group_size, psa_bits=a.psa_bits, smem_levels=a.smem_levels, window=a.window,
+                      flags=a.flags)
+            for item in filter(None, spec.split(",")):
+                k, v = item.split("=")
+                kw[k] = int(v)
+            o = hm.make_opts(**kw)
+            for _ in range(3):
+                t.search(q, out, opts=o)
+            torch.cuda.synchronize()
+            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            hm.profile_enable(True)
+            hm.profile_read()
+            s0.record()
+            for _ in range(a.steps):
+                t.search(q, out, opts=o)
+            s1.record()
+            torch.cuda.synchronize()
+            hm.profile_enable(False)
+            pr = hm.profile_read()
+            ms_ = s0.elapsed_time(s1) / a.steps
+            print(json.dumps({"sweep": kw, "gqs": c["Q"] / ms_ / 1e6, "ms": ms_, "plan": t.plan(c["Q"], o),
+                              "kernels_ms_per_step": {k: v[0] / a.steps for k, v in pr.items()}}), flush=True)
+        return
+
     for _ in range(max(3, a.warmup)):
         step()
     torch.cuda.synchronize()
     # property check on this rank's batch: values are key-derived (uniform/zipf hit 100 %)
     sel = np.asarray(gen._stream(99, 0, 1 << 16) % np.uint64(c["Q"]), dtype=np.int64)
-    got = out[torch.from_numpy(sel).to(dev)].cpu().numpy()
+    got = out.view(torch.int64)[torch.from_numpy(sel).to(dev)].cpu().numpy().view(np.uint64)
     parity_ok = bool(np.array_equal(got, gen.values_for(q_np[sel])))
 
     # ---- timed region: K steps, events on the launch stream, max over ranks

@@ -52,6 +52,8 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
     }
   }
   P.gather = (o->flags & HARMONIA_QF_GATHER) != 0;
+  P.kary = (o->flags & HARMONIA_QF_LINEAR) ? 0 : 1;
+  P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
   // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
   // top levels in BFS order while they fit
   const uint32_t ps_bytes = (uint32_t)round_up((t->I + 1) * 4, 16);
@@ -106,7 +108,8 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
   const PsaWs w = psa_ws_carve(p, ws);
   for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
-    harmonia_status s = psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr);
+    harmonia_status s = p.psa_global ? psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
+                                     : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st);
     if (s != HARMONIA_OK) return s;
     a.q = w.sorted_q;
     a.n = nw;
@@ -308,7 +311,8 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   const PsaWs w = psa_ws_carve(p, ws);
   for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
-    s = psa_partition(d_lo + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr);
+    s = p.psa_global ? psa_partition(d_lo + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
+                     : psa_partition2(d_lo + w0, nw, p.bucket, p.nb, w, t->sm_count, st);
     if (s != HARMONIA_OK) return s;
     a.lo = w.sorted_q;
     a.hi = d_hi + w0;

@@ -14,7 +14,9 @@ namespace hm {
 constexpr uint64_t kPad = 0xFFFFFFFFFFFFFFFFull;       // HARMONIA_KEY_PAD
 constexpr uint64_t kNotFound = 0xFFFFFFFFFFFFFFFFull;  // HARMONIA_NOT_FOUND
 constexpr unsigned kFull = 0xFFFFFFFFu;
-constexpr int kBlock = 256;  // threads per CTA for the query kernels
+constexpr int kBlock = 256;        // threads per CTA for the streaming kernels
+constexpr int kQueryBlock = 1024;  // search/range CTAs: 2 per SM, so the staged tree top is
+                                   // duplicated twice per SM and L1 keeps most of its capacity
 
 // ---- error plumbing --------------------------------------------------------------
 harmonia_status cuda_fail(cudaError_t e);
@@ -115,6 +117,8 @@ struct Plan {
   uint32_t ps_smem_bytes = 0;
   uint32_t smem_bytes = 0;   // dynamic smem of the search kernel
   bool gather = false;
+  int kary = 1;              // in-node search: 1 = k-ary NTG, 0 = linear NTG (Fig 9)
+  bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
 };
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
@@ -154,6 +158,8 @@ struct SearchArgs {
   uint64_t n;
   uint64_t* out;           // results: out[idx ? idx[j] : j]
 };
+harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
+                               int sm_count, cudaStream_t st);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
                               cudaStream_t st);
 

@@ -92,47 +92,133 @@ __device__ __forceinline__ ulonglong2 ld_pair(const uint64_t* p) {
   else return ld_pair_global(p);
 }
 
-// Number of keys in the node that are <= q (STRICT: < q).  `live` is uniform inside a
-// group; the loop is warp-uniform so that every ballot sees the full warp.
-template <int F, int G, bool SMEM, bool STRICT>
-__device__ __forceinline__ uint32_t node_rank(const uint64_t* nk, uint64_t q, bool live, uint32_t gmask,
-                                              int gl) {
-  constexpr int KPS = 2 * G, STEPS = F / KPS;
-  uint32_t r = 0;
-  bool done = !live;
-#pragma unroll
-  for (int s = 0; s < STEPS; ++s) {
-    if (__all_sync(kFull, done)) break;
-    ulonglong2 k = make_ulonglong2(kPad, kPad);
-    if (!done) k = ld_pair<SMEM>(nk + s * KPS + 2 * gl);
-    const bool le0 = !done && (STRICT ? k.x < q : k.x <= q);
-    const bool le1 = !done && (STRICT ? k.y < q : k.y <= q);
-    const uint32_t c = __popc(__ballot_sync(kFull, le0) & gmask) + __popc(__ballot_sync(kFull, le1) & gmask);
-    r += c;
-    done = done || (c < (uint32_t)KPS);
+// Predicated 128-bit load that keeps the old register contents when `pred` is false
+// (a single predicated LDG/LDS, no branch around it).
+template <bool SMEM>
+__device__ __forceinline__ void ld_pair_if(ulonglong2& k, const uint64_t* p, bool pred) {
+  if constexpr (SMEM) {
+    const uint32_t a = smem_u32(p);
+    asm("{ .reg .pred q; setp.ne.b32 q, %3, 0; @q ld.shared.v2.u64 {%0, %1}, [%2]; }"
+                 : "+l"(k.x), "+l"(k.y)
+                 : "r"(a), "r"((int)pred));
+  } else {
+    asm("{ .reg .pred q; setp.ne.b32 q, %3, 0; @q ld.global.nc.v2.u64 {%0, %1}, [%2]; }"
+                 : "+l"(k.x), "+l"(k.y)
+                 : "l"(p), "r"((int)pred));
   }
+}
+
+// warp ballot without the compiler's divergence fallback (all 32 lanes always converge here)
+__device__ __forceinline__ unsigned ballot(bool pred) {
+  unsigned r;
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %1, 0; vote.sync.ballot.b32 %0, q, 0xffffffff; }"
+               : "=r"(r)
+               : "r"((int)pred));
   return r;
 }
 
-// Descend levels 0..h-2 with Eq 1; returns the leaf's node index.
-template <int F, int G>
-__device__ __forceinline__ uint32_t descend(uint64_t q, bool live, uint32_t h, uint32_t smem_levels,
+// NTG in-node rank: the number of keys in the node that are <= q (STRICT:
+// < q), for every group whose last-lane bit is set in `act` (a warp-uniform mask).
+// Step s: each lane of the group loads keys [s*2G + 2*gl, +2) with one 128-bit load; the
+// group goes on to step s+1 only if its last key is still <= q (early exit, Fig 9).  A
+// group that has stopped keeps its registers, so its ballot bits in later steps repeat
+// its final step: the rank is (steps-1)*2G + popc of the final two ballots.  EQ also
+// reports whether some key equals q (leaf probe).
+template <int F, int G, bool SMEM, bool STRICT, bool EQ>
+__device__ __forceinline__ uint32_t ntg_rank(const uint64_t* nk, uint64_t q, unsigned act, int grp, int gl,
+                                             uint32_t gmask, bool* found) {
+  constexpr int KPS = 2 * G, STEPS = F / KPS;
+  const unsigned mybit = 1u << (grp * G + G - 1);
+  bool my = (act & mybit) != 0;
+  ulonglong2 k = make_ulonglong2(0, 0);
+  unsigned bx = 0, by = 0, fe = 0;
+  int steps = 0;
+#pragma unroll
+  for (int s = 0; s < STEPS; ++s) {
+    ld_pair_if<SMEM>(k, nk + s * KPS + 2 * gl, my);
+    bx = ballot(STRICT ? k.x < q : k.x <= q);
+    by = ballot(STRICT ? k.y < q : k.y <= q);
+    if constexpr (EQ) fe |= ballot((k.x == q) | (k.y == q));
+    steps += my ? 1 : 0;
+    act &= by;  // groups whose whole step is <= q continue
+    if (act == 0) break;
+    my = (act & mybit) != 0;
+  }
+  if constexpr (EQ) *found = (fe & gmask) != 0;
+  return (uint32_t)((steps - 1) * KPS) + __popc(bx & gmask) + __popc(by & gmask);
+}
+
+// k-ary NTG in-node rank: the same G-lane group, 128-bit loads and
+// ballot/popc rank as the linear walk above, but the group first compares the last key of
+// each of G equal blocks of the span (one coarse step selects the block that holds the
+// rank), recursing until the span fits one contiguous step.  Every query takes the same
+// log_G(F/2G)+1 steps, so there is no early-exit divergence inside the warp (the query
+// divergence of P:L500 disappears) and the comparisons per level drop from O(F/2G) steps
+// to O(log F).  Inactive groups must pass a q that keeps spans inside the node (q = 0).
+template <int S, int G, bool SMEM, bool STRICT, bool EQ>
+struct KaryStep {
+  static __device__ __forceinline__ uint32_t run(const uint64_t* nk, uint32_t base, uint64_t q, int gl,
+                                                 uint32_t gmask, unsigned& fe) {
+    if constexpr (S / 2 <= G) {
+      constexpr int L = S / 2;  // final step: L lanes read the span contiguously
+      ulonglong2 k = make_ulonglong2(kPad, kPad);
+      if constexpr (L < G) ld_pair_if<SMEM>(k, nk + base + 2 * gl, gl < L);
+      else k = ld_pair<SMEM>(nk + base + 2 * gl);
+      const unsigned bx = ballot(STRICT ? k.x < q : k.x <= q);
+      const unsigned by = ballot(STRICT ? k.y < q : k.y <= q);
+      if constexpr (EQ) fe |= ballot((k.x == q) | (k.y == q));
+      return base + __popc(bx & gmask) + __popc(by & gmask);
+    } else {
+      constexpr int B = S / G;  // coarse step: lane gl holds the last two keys of block gl
+      const ulonglong2 k = ld_pair<SMEM>(nk + base + gl * B + (B - 2));
+      const unsigned by = ballot(STRICT ? k.y < q : k.y <= q);
+      if constexpr (EQ) fe |= ballot((k.x == q) | (k.y == q));
+      // blocks whose last key is <= q lie entirely before the rank (the span's last key is
+      // > q, so at most G-1 of them)
+      return KaryStep<B, G, SMEM, STRICT, EQ>::run(nk, base + (uint32_t)__popc(by & gmask) * B, q, gl, gmask, fe);
+    }
+  }
+};
+
+template <int F, int G, bool SMEM, bool STRICT, bool EQ>
+__device__ __forceinline__ uint32_t kary_rank(const uint64_t* nk, uint64_t q, int gl, uint32_t gmask,
+                                              bool* found) {
+  unsigned fe = 0;
+  const uint32_t r = KaryStep<F, G, SMEM, STRICT, EQ>::run(nk, 0, q, gl, gmask, fe);
+  if constexpr (EQ) *found = (fe & gmask) != 0;
+  return r;
+}
+
+// in-node rank dispatch: MODE 0 = linear NTG (Fig 9), MODE 1 = k-ary NTG
+template <int F, int G, int MODE, bool SMEM, bool STRICT, bool EQ>
+__device__ __forceinline__ uint32_t node_rank(const uint64_t* nk, uint64_t q, bool live, unsigned act, int grp,
+                                              int gl, uint32_t gmask, bool* found) {
+  if constexpr (MODE == 0) return ntg_rank<F, G, SMEM, STRICT, EQ>(nk, q, act, grp, gl, gmask, found);
+  else return kary_rank<F, G, SMEM, STRICT, EQ>(nk, live ? q : 0, gl, gmask, found);
+}
+
+// Descend levels 0..h-2 with Eq 1; returns the leaf's node index.  `act` = last-lane bits
+// of the live groups (uniform); non-live groups stay on node indices that are valid.
+template <int F, int G, int MODE>
+__device__ __forceinline__ uint32_t descend(uint64_t q, bool live, unsigned act, uint32_t h, uint32_t smem_levels,
                                             const uint64_t* s_keys, const uint32_t* s_ps, bool ps_smem,
                                             const uint64_t* __restrict__ keys, const uint32_t* __restrict__ ps,
-                                            uint32_t gmask, int gl) {
+                                            int grp, int gl, uint32_t gmask) {
   uint32_t node = 0;
   for (uint32_t l = 0; l + 1 < h; ++l) {
     const uint32_t first = ps_smem ? s_ps[node] : __ldg(ps + node);  // PS[node_idx]
     uint32_t r;
-    if (l < smem_levels) r = node_rank<F, G, true, false>(s_keys + (uint64_t)node * F, q, live, gmask, gl);
-    else r = node_rank<F, G, false, false>(keys + (uint64_t)node * F, q, live, gmask, gl);
-    node = first + r;  // Eq 1: child_idx = PrefixSum[node_idx] + i - 1, i = r + 1
+    if (l < smem_levels)
+      r = node_rank<F, G, MODE, true, false, false>(s_keys + (uint64_t)node * F, q, live, act, grp, gl, gmask, nullptr);
+    else
+      r = node_rank<F, G, MODE, false, false, false>(keys + (uint64_t)node * F, q, live, act, grp, gl, gmask, nullptr);
+    node = first + (live ? r : 0u);  // Eq 1: child_idx = PrefixSum[node_idx] + i - 1, i = r + 1
   }
   return node;
 }
 
-template <int F, int G>
-__global__ void __launch_bounds__(kBlock) k_ntg_search(const SearchArgs a) {
+template <int F, int G, int MODE>
+__global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_search(const SearchArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
   stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
@@ -140,42 +226,31 @@ __global__ void __launch_bounds__(kBlock) k_ntg_search(const SearchArgs a) {
   const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
   const bool ps_smem = a.ps_smem_bytes != 0;
 
-  constexpr int QPW = 32 / G, KPS = 2 * G, STEPS = F / KPS;
+  constexpr int QPW = 32 / G;
   const int lane = threadIdx.x & 31, grp = lane / G, gl = lane % G;
   const uint32_t gmask = (G == 32) ? kFull : (((1u << G) - 1u) << (grp * G));
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
 
   for (uint64_t base = warp * QPW; base < a.n; base += nwarps * QPW) {
     const uint64_t j = base + grp;
     const bool active = j < a.n;
     const uint64_t q = active ? ld_stream(a.q + j) : kPad;
     const bool live = active && q != kPad;  // PAD is never a key (C-A2)
+    const unsigned act = __ballot_sync(kFull, live && gl == G - 1);
     const uint32_t leaf =
-        descend<F, G>(q, live, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
-    // leaf probe: slot of key == q ("the target key is found")
-    const bool leaf_smem = a.h - 1 < a.smem_levels;
-    const uint64_t* nk = (leaf_smem ? s_keys : a.keys) + (uint64_t)leaf * F;
-    int slot = -1;
-    bool done = !live;
-#pragma unroll
-    for (int s = 0; s < STEPS; ++s) {
-      if (__all_sync(kFull, done)) break;
-      ulonglong2 k = make_ulonglong2(kPad, kPad);
-      if (!done) k = leaf_smem ? ld_pair<true>(nk + s * KPS + 2 * gl) : ld_pair<false>(nk + s * KPS + 2 * gl);
-      const uint32_t b_le = (__ballot_sync(kFull, !done && k.x <= q) & gmask);
-      const uint32_t b_le1 = (__ballot_sync(kFull, !done && k.y <= q) & gmask);
-      const uint32_t e0 = __ballot_sync(kFull, !done && k.x == q) & gmask;
-      const uint32_t e1 = __ballot_sync(kFull, !done && k.y == q) & gmask;
-      if (!done) {
-        if (e0) slot = s * KPS + 2 * (__ffs(e0) - 1 - grp * G);
-        else if (e1) slot = s * KPS + 2 * (__ffs(e1) - 1 - grp * G) + 1;
-        if ((e0 | e1) || (__popc(b_le) + __popc(b_le1) < KPS)) done = true;
-      }
-    }
+        descend<F, G, MODE>(q, live, act, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, grp, gl, gmask);
+    // leaf probe ("the target key is found"): r = #keys <= q, hit iff key[r-1] == q
+    bool found = false;
+    uint32_t r;
+    if (leaf_smem)
+      r = node_rank<F, G, MODE, true, false, true>(s_keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, &found);
+    else
+      r = node_rank<F, G, MODE, false, false, true>(a.keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, &found);
     if (active && gl == 0) {
       uint64_t v = kNotFound;
-      if (slot >= 0) v = __ldg(a.vals + (uint64_t)(leaf - a.leaf_start) * F + slot);
+      if (live && found) v = __ldg(a.vals + (uint64_t)(leaf - a.leaf_start) * F + (r - 1));
       const uint64_t o = a.idx ? (uint64_t)ld_stream32(a.idx + j) : j;
       a.out[o] = v;
     }
@@ -183,8 +258,8 @@ __global__ void __launch_bounds__(kBlock) k_ntg_search(const SearchArgs a) {
 }
 
 // Range scan: descend with lo, then walk leaf slots in key-region order.
-template <int F, int G>
-__global__ void __launch_bounds__(kBlock) k_ntg_range(const RangeArgs a) {
+template <int F, int G, int MODE>
+__global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_range(const RangeArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
   stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
@@ -209,7 +284,9 @@ __global__ void __launch_bounds__(kBlock) k_ntg_range(const RangeArgs a) {
     const uint64_t slab = active ? (a.idx ? (uint64_t)ld_stream32(a.idx + j) : j) : 0;
     const uint64_t hi = active ? __ldg(a.hi + slab) : 0;
     const bool live = active && lo <= hi && lo != kPad;
-    uint32_t cur = descend<F, G>(lo, live, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
+    const unsigned act = __ballot_sync(kFull, live && gl == G - 1);
+    uint32_t cur = descend<F, G, MODE>(lo, live, act, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, grp, gl,
+                                 gmask);
     uint64_t cnt = 0;
     bool trunc = live && cap == 0;
     bool done = !live || trunc;
@@ -254,10 +331,15 @@ __global__ void __launch_bounds__(kBlock) k_ntg_range(const RangeArgs a) {
     if (__any_sync(kFull, trunc)) {
       // keys never equal PAD, so #keys <= PAD == #keys <= PAD-1 (and PAD slots stay excluded)
       const uint64_t hd = hi == kPad ? kPad - 1 : hi;
-      const uint32_t lh = descend<F, G>(hd, trunc, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
-      const uint32_t rh = node_rank<F, G, false, false>(a.keys + (uint64_t)lh * F, hd, trunc, gmask, gl);
-      const uint32_t ll = descend<F, G>(lo, trunc, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, gmask, gl);
-      const uint32_t rl = node_rank<F, G, false, true>(a.keys + (uint64_t)ll * F, lo, trunc, gmask, gl);
+      const unsigned tact = __ballot_sync(kFull, trunc && gl == G - 1);
+      const uint32_t lh = descend<F, G, MODE>(hd, trunc, tact, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps,
+                                        grp, gl, gmask);
+      const uint32_t rh =
+          node_rank<F, G, MODE, false, false, false>(a.keys + (uint64_t)lh * F, hd, trunc, tact, grp, gl, gmask, nullptr);
+      const uint32_t ll = descend<F, G, MODE>(lo, trunc, tact, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps,
+                                        grp, gl, gmask);
+      const uint32_t rl =
+          node_rank<F, G, MODE, false, true, false>(a.keys + (uint64_t)ll * F, lo, trunc, tact, grp, gl, gmask, nullptr);
       if (trunc)
         cnt = (__ldg(a.leaf_base + (lh - a.leaf_start)) + rh) - (__ldg(a.leaf_base + (ll - a.leaf_start)) + rl);
     }
@@ -267,24 +349,21 @@ __global__ void __launch_bounds__(kBlock) k_ntg_range(const RangeArgs a) {
 
 template <int F, int G>
 harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
-  auto kern = k_ntg_search<F, G>;
-  static int configured_smem = -1;  // per instantiation
-  if ((int)p.smem_bytes > configured_smem) {
+  auto kern = p.kary ? k_ntg_search<F, G, 1> : k_ntg_search<F, G, 0>;
+  static int configured_smem[2] = {-1, -1};  // per instantiation and mode
+  if ((int)p.smem_bytes > configured_smem[p.kary]) {
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem = (int)p.smem_bytes;
+    configured_smem[p.kary] = (int)p.smem_bytes;
   }
   int per_sm = 0;
-  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBlock, p.smem_bytes));
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kQueryBlock, p.smem_bytes));
   per_sm = std::max(per_sm, 1);
-  const uint64_t qpb = (uint64_t)(kBlock / 32) * (32 / G);
+  const uint64_t qpb = (uint64_t)(kQueryBlock / 32) * (32 / G);
   const uint64_t need = ceil_div(a.n, qpb);
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    {
-    ProfScope ps_(HARMONIA_PROF_RANGE, st);
-    kern<<<grid, kBlock, p.smem_bytes, st>>>(a);
-  }
+    kern<<<grid, kQueryBlock, p.smem_bytes, st>>>(a);
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
@@ -292,19 +371,22 @@ harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const Se
 
 template <int F, int G>
 harmonia_status launch_range_fg(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
-  auto kern = k_ntg_range<F, G>;
-  static int configured_smem = -1;
-  if ((int)p.smem_bytes > configured_smem) {
+  auto kern = p.kary ? k_ntg_range<F, G, 1> : k_ntg_range<F, G, 0>;
+  static int configured_smem[2] = {-1, -1};
+  if ((int)p.smem_bytes > configured_smem[p.kary]) {
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem = (int)p.smem_bytes;
+    configured_smem[p.kary] = (int)p.smem_bytes;
   }
   int per_sm = 0;
-  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBlock, p.smem_bytes));
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kQueryBlock, p.smem_bytes));
   per_sm = std::max(per_sm, 1);
-  const uint64_t qpb = (uint64_t)(kBlock / 32) * (32 / G);
+  const uint64_t qpb = (uint64_t)(kQueryBlock / 32) * (32 / G);
   const uint64_t need = ceil_div(a.n, qpb);
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
-  kern<<<grid, kBlock, p.smem_bytes, st>>>(a);
+  {
+    ProfScope ps_(HARMONIA_PROF_RANGE, st);
+    kern<<<grid, kQueryBlock, p.smem_bytes, st>>>(a);
+  }
   HM_LAUNCHED();
   return HARMONIA_OK;
 }

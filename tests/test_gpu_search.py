@@ -130,7 +130,9 @@ def test_every_fanout_and_group_size(hm, orc, F, G):
     q = np.concatenate([gen.uniform_queries(keys, 60001, miss_frac=0.4), gen.edge_queries(keys)])
     exp = orc.sorted_search(keys, vals, q)
     for kw in ({}, {"psa_bits": -1}, {"window": 4096}, {"smem_levels": -1}, {"smem_levels": 2},
-               {"flags": hm.QF_GATHER, "window": 8192}, {"psa_bits": 3}):
+               {"flags": hm.QF_GATHER, "window": 8192}, {"psa_bits": 3}, {"flags": hm.QF_LINEAR},
+               {"flags": hm.QF_LINEAR, "psa_bits": -1, "smem_levels": 1},
+               {"flags": hm.QF_PSA_GLOBAL}, {"flags": hm.QF_PSA_GLOBAL | hm.QF_LINEAR, "window": 3072}):
         assert np.array_equal(host(t.search(cu(q), group_size=G, **kw)), exp), kw
 
 
@@ -173,7 +175,7 @@ def test_range_parity(hm, orc, F, G, length, cap):
     lo2, hi2 = gen.random_ranges(keys, 3000, max_width_keys=3 * max(cap, 8))
     lo, hi = np.concatenate([lo, lo2]), np.concatenate([hi, hi2])
     eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, cap)
-    for kw in ({}, {"psa_bits": -1}, {"window": 2048}):
+    for kw in ({}, {"psa_bits": -1}, {"window": 2048}, {"flags": hm.QF_LINEAR}):
         ko, vo, cnt = t.range(cu(lo), cu(hi), cap, group_size=G, **kw)
         _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
 
