@@ -11,7 +11,7 @@ namespace hm {
 
 namespace {
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
-constexpr uint64_t kAutoWindow = 1ull << 22;  // auto PSA window (queries), see DESIGN.md §5
+constexpr uint64_t kAutoWindow = 1ull << 24;  // auto PSA window (queries): measured best, DESIGN.md §7
 
 bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 }  // namespace

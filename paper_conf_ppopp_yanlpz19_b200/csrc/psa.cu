@@ -156,232 +156,11 @@ int stream_grid(uint64_t n, int sm) {
   return (int)std::min<uint64_t>(g, (uint64_t)sm * 8);
 }
 
-// ---- two-level PSA (default): coarse MSB partition + chunk-local counting sort ----------
-// Level 1 orders the window by the top kCoarseBits of the Nb-bit bucket with one atomic per
-// (CTA tile, bin) instead of one per query; level 2 sorts every kChunk-sized chunk of that
-// order by the full Nb-bit bucket in shared memory.  The result is the same partial order
-// as Eq 2's N-bit sort at chunk granularity (C-A12: order inside a bucket is free).
-constexpr int kCoarseBits = 8, kCoarseBins = 1 << kCoarseBits;
-constexpr int kCoarseTile = kBlock * 8;  // 2048 queries per scatter tile
-constexpr int kSortThreads = 512, kSortPer = 8, kChunk = kSortThreads * kSortPer;  // 4096
-constexpr int kLocalBins = 2048;
-constexpr size_t kSortSmem = kLocalBins * 4 + kChunk * 8 + kChunk * 4;  // 56 KiB
-
-// exclusive scan of one value per thread over the block (blockDim = NT); returns the
-// prefix, *total receives the block sum.  `tmp` needs NT/32 + 1 words.
-template <int NT>
-__device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t v, uint32_t* tmp, uint32_t* total) {
-  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t inc = v;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    uint32_t y = __shfl_up_sync(kFull, inc, d);
-    if (lane >= (unsigned)d) inc += y;
-  }
-  if (lane == 31) tmp[warp] = inc;
-  __syncthreads();
-  if (warp == 0) {
-    uint32_t w = lane < NT / 32 ? tmp[lane] : 0;
-    uint32_t wi = w;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      uint32_t y = __shfl_up_sync(kFull, wi, d);
-      if (lane >= (unsigned)d) wi += y;
-    }
-    if (lane < NT / 32) tmp[lane] = wi - w;
-    if (lane == 31) tmp[NT / 32] = wi;
-  }
-  __syncthreads();
-  const uint32_t r = tmp[warp] + inc - v;
-  *total = tmp[NT / 32];
-  __syncthreads();
-  return r;
-}
-
-template <class Bucket>
-__global__ void __launch_bounds__(kBlock) k_psa_coarse_hist(const uint64_t* __restrict__ q, uint64_t n, Bucket f,
-                                                            uint32_t shift1, uint32_t* __restrict__ counts) {
-  __shared__ uint32_t h[kCoarseBins];
-  static_assert(kBlock == kCoarseBins, "one bin per thread");
-  h[threadIdx.x] = 0;
-  __syncthreads();
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += stride)
-    atomicAdd(&h[f(__ldg(q + i)) >> shift1], 1u);
-  __syncthreads();
-  if (h[threadIdx.x]) atomicAdd(counts + threadIdx.x, h[threadIdx.x]);
-}
-
-template <class Bucket>
-__global__ void __launch_bounds__(kBlock) k_psa_coarse_scatter(const uint64_t* __restrict__ q, uint64_t n, Bucket f,
-                                                               uint32_t shift1, const uint32_t* __restrict__ counts,
-                                                               uint32_t* __restrict__ cursor,
-                                                               uint64_t* __restrict__ sorted_q,
-                                                               uint32_t* __restrict__ idx) {
-  __shared__ uint32_t s_prefix[kCoarseBins], s_cnt[kCoarseBins], s_base[kCoarseBins], tmp[kBlock / 32 + 1];
-  uint32_t tot;
-  s_prefix[threadIdx.x] = block_exclusive_scan<kBlock>(counts[threadIdx.x], tmp, &tot);
-  for (uint64_t t0 = (uint64_t)blockIdx.x * kCoarseTile; t0 < n; t0 += (uint64_t)gridDim.x * kCoarseTile) {
-    s_cnt[threadIdx.x] = 0;
-    __syncthreads();
-    uint64_t v[8];
-    uint32_t d[8], rk[8];
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const uint64_t i = t0 + k * kBlock + threadIdx.x;
-      if (i < n) {
-        v[k] = __ldg(q + i);
-        d[k] = f(v[k]) >> shift1;
-        rk[k] = atomicAdd(&s_cnt[d[k]], 1u);
-      }
-    }
-    __syncthreads();
-    const uint32_t c = s_cnt[threadIdx.x];
-    if (c) s_base[threadIdx.x] = s_prefix[threadIdx.x] + atomicAdd(cursor + threadIdx.x, c);
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const uint64_t i = t0 + k * kBlock + threadIdx.x;
-      if (i < n) {
-        const uint32_t dst = s_base[d[k]] + rk[k];
-        sorted_q[dst] = v[k];
-        idx[dst] = (uint32_t)i;
-      }
-    }
-    __syncthreads();
-  }
-}
-
-// In place: each chunk of the coarse order is counting-sorted by its Nb-bit bucket value
-// (offset by the chunk minimum, shifted until the range fits kLocalBins).
-template <class Bucket>
-__global__ void __launch_bounds__(kSortThreads) k_psa_local_sort(uint64_t* __restrict__ sorted_q,
-                                                                 uint32_t* __restrict__ idx, uint64_t n, Bucket f) {
-  extern __shared__ __align__(16) unsigned char sm[];
-  uint32_t* hist = reinterpret_cast<uint32_t*>(sm);
-  uint64_t* sk = reinterpret_cast<uint64_t*>(sm + kLocalBins * 4);
-  uint32_t* si = reinterpret_cast<uint32_t*>(sm + kLocalBins * 4 + kChunk * 8);
-  __shared__ uint32_t tmp[kSortThreads / 32 + 1];
-  __shared__ uint32_t s_min[kSortThreads / 32], s_max[kSortThreads / 32];
-  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t c0 = (uint64_t)blockIdx.x * kChunk; c0 < n; c0 += (uint64_t)gridDim.x * kChunk) {
-    const uint32_t m = (uint32_t)std::min<uint64_t>(kChunk, n - c0);
-    uint64_t v[kSortPer];
-    uint32_t ix[kSortPer], b[kSortPer];
-    uint32_t bmin = 0xFFFFFFFFu, bmax = 0;
-#pragma unroll
-    for (int k = 0; k < kSortPer; ++k) {
-      const uint32_t e = k * kSortThreads + threadIdx.x;
-      if (e < m) {
-        v[k] = sorted_q[c0 + e];
-        ix[k] = idx[c0 + e];
-        b[k] = f(v[k]);
-        bmin = min(bmin, b[k]);
-        bmax = max(bmax, b[k]);
-      }
-    }
-    bmin = __reduce_min_sync(kFull, bmin);
-    bmax = __reduce_max_sync(kFull, bmax);
-    if (lane == 0) {
-      s_min[warp] = bmin;
-      s_max[warp] = bmax;
-    }
-    for (uint32_t i = threadIdx.x; i < kLocalBins; i += kSortThreads) hist[i] = 0;
-    __syncthreads();
-    bmin = s_min[0];
-    bmax = s_max[0];
-#pragma unroll
-    for (int w = 1; w < kSortThreads / 32; ++w) {
-      bmin = min(bmin, s_min[w]);
-      bmax = max(bmax, s_max[w]);
-    }
-    uint32_t sh = 0;
-    while (((bmax - bmin) >> sh) >= (uint32_t)kLocalBins) ++sh;
-    uint32_t rk[kSortPer];
-#pragma unroll
-    for (int k = 0; k < kSortPer; ++k) {
-      const uint32_t e = k * kSortThreads + threadIdx.x;
-      if (e < m) {
-        b[k] = (b[k] - bmin) >> sh;
-        rk[k] = atomicAdd(&hist[b[k]], 1u);
-      }
-    }
-    __syncthreads();
-    // exclusive scan of the local histogram: 4 consecutive bins per thread
-    static_assert(kLocalBins == 4 * kSortThreads, "4 bins per thread");
-    uint32_t hv[4], hs = 0;
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      hv[k] = hist[threadIdx.x * 4 + k];
-      hs += hv[k];
-    }
-    uint32_t tot;
-    uint32_t run = block_exclusive_scan<kSortThreads>(hs, tmp, &tot);
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      hist[threadIdx.x * 4 + k] = run;
-      run += hv[k];
-    }
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < kSortPer; ++k) {
-      const uint32_t e = k * kSortThreads + threadIdx.x;
-      if (e < m) {
-        const uint32_t dst = hist[b[k]] + rk[k];
-        sk[dst] = v[k];
-        si[dst] = ix[k];
-      }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < kSortPer; ++k) {
-      const uint32_t e = k * kSortThreads + threadIdx.x;
-      if (e < m) {
-        sorted_q[c0 + e] = sk[e];
-        idx[c0 + e] = si[e];
-      }
-    }
-    __syncthreads();
-  }
-}
-
 }  // namespace
-
-harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
-                               cudaStream_t st) {
-  const uint32_t b1 = (uint32_t)std::min(nb, kCoarseBits);
-  const uint32_t shift1 = (uint32_t)nb - b1;
-  HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * kCoarseBins * 4, st));
-  {
-    ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
-    k_psa_coarse_hist<BucketBits><<<stream_grid(n, sm), kBlock, 0, st>>>(q, n, f, shift1, ws.counts);
-  }
-  HM_LAUNCHED();
-  {
-    ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kCoarseTile), (uint64_t)sm * 8);
-    k_psa_coarse_scatter<BucketBits><<<g, kBlock, 0, st>>>(q, n, f, shift1, ws.counts, ws.counts + kCoarseBins,
-                                                           ws.sorted_q, ws.idx);
-  }
-  HM_LAUNCHED();
-  {
-    ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);  // (reported as the "scan" class: level-2 sort)
-    static bool configured = false;
-    if (!configured) {
-      HM_CUDA(cudaFuncSetAttribute(k_psa_local_sort<BucketBits>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)kSortSmem));
-      configured = true;
-    }
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kChunk), (uint64_t)sm * 4);
-    k_psa_local_sort<BucketBits><<<g, kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
-  }
-  HM_LAUNCHED();
-  return HARMONIA_OK;
-}
 
 size_t psa_ws_bytes(const Plan& p) {
   if (!p.psa) return 0;
-  size_t b = round_up((size_t)std::max<uint32_t>(p.nbins, 2 * kCoarseBins) * 4, 256);
+  size_t b = round_up((size_t)std::max<uint32_t>(p.nbins, 512) * 4, 256);
   b += round_up(ceil_div(p.nbins, kScanTile) * 4, 256);
   b += round_up(p.window * 8, 256);
   b += round_up(p.window * 4, 256);
@@ -393,7 +172,7 @@ PsaWs psa_ws_carve(const Plan& p, void* base) {
   char* c = (char*)base;
   PsaWs w{};
   w.counts = (uint32_t*)c;
-  c += round_up((size_t)std::max<uint32_t>(p.nbins, 2 * kCoarseBins) * 4, 256);
+  c += round_up((size_t)std::max<uint32_t>(p.nbins, 512) * 4, 256);
   w.tile_sums = (uint32_t*)c;
   c += round_up(ceil_div(p.nbins, kScanTile) * 4, 256);
   w.sorted_q = (uint64_t*)c;

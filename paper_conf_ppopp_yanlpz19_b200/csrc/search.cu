@@ -197,6 +197,17 @@ __device__ __forceinline__ uint32_t node_rank(const uint64_t* nk, uint64_t q, bo
   else return kary_rank<F, G, SMEM, STRICT, EQ>(nk, live ? q : 0, gl, gmask, found);
 }
 
+// Bring every 128-B line of a node into L1 at once: the in-node steps that follow then
+// wait for one L2 round trip per level instead of one per line they touch.
+template <int BYTES, int G>
+__device__ __forceinline__ void prefetch_lines(const void* p, int gl, bool on) {
+  constexpr int LINES = BYTES >= 128 ? BYTES / 128 : 1;
+  if (on) {
+#pragma unroll
+    for (int i = gl; i < LINES; i += G) asm volatile("prefetch.global.L1 [%0];" ::"l"((const char*)p + i * 128));
+  }
+}
+
 // Descend levels 0..h-2 with Eq 1; returns the leaf's node index.  `act` = last-lane bits
 // of the live groups (uniform); non-live groups stay on node indices that are valid.
 template <int F, int G, int MODE>
@@ -208,10 +219,11 @@ __device__ __forceinline__ uint32_t descend(uint64_t q, bool live, unsigned act,
   for (uint32_t l = 0; l + 1 < h; ++l) {
     const uint32_t first = ps_smem ? s_ps[node] : __ldg(ps + node);  // PS[node_idx]
     uint32_t r;
-    if (l < smem_levels)
+    if (l < smem_levels) {
       r = node_rank<F, G, MODE, true, false, false>(s_keys + (uint64_t)node * F, q, live, act, grp, gl, gmask, nullptr);
-    else
+    } else {
       r = node_rank<F, G, MODE, false, false, false>(keys + (uint64_t)node * F, q, live, act, grp, gl, gmask, nullptr);
+    }
     node = first + (live ? r : 0u);  // Eq 1: child_idx = PrefixSum[node_idx] + i - 1, i = r + 1
   }
   return node;
@@ -239,19 +251,22 @@ __global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_search(const SearchArgs 
     const uint64_t q = active ? ld_stream(a.q + j) : kPad;
     const bool live = active && q != kPad;  // PAD is never a key (C-A2)
     const unsigned act = __ballot_sync(kFull, live && gl == G - 1);
+    uint64_t o = j;  // result position, loaded early to overlap the descent
+    if (a.idx && active && gl == 0) o = ld_stream32(a.idx + j);
     const uint32_t leaf =
         descend<F, G, MODE>(q, live, act, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, grp, gl, gmask);
     // leaf probe ("the target key is found"): r = #keys <= q, hit iff key[r-1] == q
     bool found = false;
     uint32_t r;
-    if (leaf_smem)
+    const uint64_t* lv = a.vals + (uint64_t)(leaf - a.leaf_start) * F;
+    if (leaf_smem) {
       r = node_rank<F, G, MODE, true, false, true>(s_keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, &found);
-    else
+    } else {
       r = node_rank<F, G, MODE, false, false, true>(a.keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, &found);
+    }
     if (active && gl == 0) {
       uint64_t v = kNotFound;
-      if (live && found) v = __ldg(a.vals + (uint64_t)(leaf - a.leaf_start) * F + (r - 1));
-      const uint64_t o = a.idx ? (uint64_t)ld_stream32(a.idx + j) : j;
+      if (live && found) v = __ldg(lv + (r - 1));
       a.out[o] = v;
     }
   }
@@ -450,15 +465,10 @@ harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeA
 
 // Measured default G per fanout (refreshed from bench sweeps).
 int auto_group_size(uint32_t F) {
-  switch (F) {
-    case 4: return 2;
-    case 8: return 2;
-    case 16: return 4;
-    case 32: return 4;
-    case 64: return 8;
-    case 128: return 8;
-    default: return 16;
-  }
+  // k-ary NTG: G = 2 was fastest at F = 64 (bench sweeps); the same narrow
+  // group keeps 16 queries per warp for the other fanouts (F >= 4 always admits G = 2).
+  (void)F;
+  return 2;
 }
 
 }  // namespace hm

@@ -1,0 +1,124 @@
+"""Summarise ncu output into profiles/: the launch list (per-kernel share of the step) and
+the `--set full` capture of the top kernels (DRAM/L2 traffic, throughput, stall reasons).
+
+  python tools/ncu_summary.py --launches gpurun_out/launches_r1.csv --rep gpurun_out/prof_r1.ncu-rep \
+      --queries-per-launch 16777216 --workload c2_T2^23_F64_Q2^26_uniform --out profiles/r1
+"""
+import argparse
+import collections
+import csv
+import io
+import json
+import os
+import subprocess
+
+METRICS = [
+    "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+    "dram__throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_bytes.sum", "lts__t_sector_hit_rate.pct",
+    "lts__throughput.avg.pct_of_peak_sustained_elapsed", "l1tex__t_sector_hit_rate.pct",
+    "l1tex__throughput.avg.pct_of_peak_sustained_active", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+    "smsp__issue_active.avg.pct_of_peak_sustained_active", "sm__warps_active.avg.pct_of_peak_sustained_active",
+    "smsp__inst_executed.sum", "smsp__thread_inst_executed_per_inst_executed.ratio",
+    "smsp__sass_average_branch_targets_threads_uniform.pct",
+    "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
+    "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
+]
+
+
+def short(name):
+    n = name.split("(")[0]
+    for p in ("void ", "hm::", "<unnamed>::", "unnamed>::", "(anonymous namespace)::"):
+        n = n.replace(p, "")
+    return n.strip()
+
+
+def launches(path):
+    rows = list(csv.reader(open(path)))
+    hi = [i for i, r in enumerate(rows) if r and r[0] == "ID"][0]
+    h = rows[hi]
+    ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
+    agg = collections.OrderedDict()
+    for r in rows[hi + 1:]:
+        v = float(r[vi].replace(",", ""))
+        v *= {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3, "second": 1e6, "s": 1e6}.get(r[ui], 1.0)
+        a = agg.setdefault(short(r[ki]), [0, 0.0])
+        a[0] += 1
+        a[1] += v
+    tot = sum(a[1] for a in agg.values())
+    return {k: {"launches": n, "total_us": us, "avg_us": us / n, "share": us / tot} for k, (n, us) in agg.items()}
+
+
+def full(rep):
+    txt = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(txt)))
+    h, units = rows[0], rows[1]
+    out = []
+    for r in rows[2:]:
+        d = {"kernel": short(r[h.index("Kernel Name")])}
+        for m in METRICS:
+            if m in h:
+                i = h.index(m)
+                try:
+                    d[m] = float(r[i].replace(",", ""))
+                except ValueError:
+                    d[m] = r[i]
+                d[m + ".unit"] = units[i]
+        stalls = {}
+        for k in h:
+            if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("not_issued"):
+                try:
+                    v = int(r[h.index(k)])
+                except ValueError:
+                    continue
+                if v:
+                    stalls[k.replace("smsp__pcsamp_warps_issue_stalled_", "")] = v
+        tot = sum(stalls.values()) or 1
+        d["stall_share"] = {k: round(v / tot, 3) for k, v in sorted(stalls.items(), key=lambda kv: -kv[1])[:8]}
+        out.append(d)
+    return out
+
+
+def to_bytes(v, unit):
+    return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--launches")
+    ap.add_argument("--rep")
+    ap.add_argument("--queries-per-launch", type=int, default=0)
+    ap.add_argument("--workload", default="")
+    ap.add_argument("--out", required=True)
+    a = ap.parse_args()
+    res = {"workload": a.workload}
+    if a.launches:
+        res["launch_list"] = launches(a.launches)
+    if a.rep:
+        res["full_capture"] = full(a.rep)
+    json.dump(res, open(a.out + ".json", "w"), indent=1)
+    # traffic per launch for bench.py's roofline.traffic (first capture of each kernel)
+    tr_path = os.path.join(os.path.dirname(a.out), "ncu_traffic.json")
+    tr = json.load(open(tr_path)) if os.path.exists(tr_path) else {}
+    for d in res.get("full_capture", []):
+        k = d["kernel"].split("<")[0]
+        rd = to_bytes(d.get("dram__bytes_read.sum", 0), d.get("dram__bytes_read.sum.unit", "byte"))
+        wr = to_bytes(d.get("dram__bytes_write.sum", 0), d.get("dram__bytes_write.sum.unit", "byte"))
+        tr.setdefault(a.workload, {}).setdefault(k, {"dram_bytes_per_launch": rd + wr,
+                                                     "source": os.path.basename(a.out) + ".json (ncu --set full, cold L2)"})
+    json.dump(tr, open(tr_path, "w"), indent=1)
+    with open(a.out + ".md", "w") as f:
+        f.write(f"# ncu summary {os.path.basename(a.out)} — {a.workload}\n\n")
+        if "launch_list" in res:
+            f.write("## Launch list (`--metrics gpu__time_duration.sum --clock-control none`; cold, serialised: compare shares)\n\n")
+            f.write("| kernel | launches | avg µs | share |\n|---|---|---|---|\n")
+            for k, v in sorted(res["launch_list"].items(), key=lambda kv: -kv[1]["share"]):
+                f.write(f"| {k} | {v['launches']} | {v['avg_us']:.1f} | {v['share']:.3f} |\n")
+        if "full_capture" in res:
+            f.write("\n## `--set full` captures\n\n")
+            for d in res["full_capture"]:
+                f.write(f"### {d['kernel']}\n\n")
+                for m in METRICS:
+                    if m in d:
+                        f.write(f"- {m}: {d[m]} {d.get(m + '.unit', '')}\n")
+                f.write(f"- stall share (pc sampling): {d['stall_share']}\n\n")
+    print(open(a.out + ".md").read())
