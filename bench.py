@@ -60,6 +60,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--mode", default="replicated", choices=["replicated", "partitioned"])
     ap.add_argument("--sweep", default="", help="comma list of k=v option sets separated by ';' (diagnostics)")
     return ap.parse_args()
 
@@ -258,7 +259,7 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     pg = None
-    if world > 1:
+    if world > 1 or a.mode == "partitioned":
         import torch.distributed as dist
 
         dist.init_process_group("nccl", device_id=dev)
@@ -268,21 +269,37 @@ def main():
         if pg:
             pg.barrier()
 
-    # ---- inputs (synthetic, seeded): identical tree on every rank (replicated mode),
-    # each rank its own slice of the global query stream (weak scaling, no collective)
+    # ---- inputs (synthetic, seeded).  replicated: identical tree on every rank, each rank its
+    # own slice of the global query stream (weak scaling, no collective).  partitioned: rank p
+    # holds the key-quantile shard p; its queries are uniform over the global key set and are
+    # routed to their shards by NCCL all-to-all (the real exchange step).
     keys = gen.uniform_keys(c["T"])
     vals = gen.values_for(keys)
-    t = hm.Tree(torch.from_numpy(keys).to(dev), torch.from_numpy(vals).to(dev), fanout=c["F"], fill=a.fill)
+    opts = hm.make_opts(a.group_size, a.psa_bits, a.smem_levels, a.window, a.flags)
+    pt = None
+    if a.mode == "partitioned":
+        from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree, key_splitters
+
+        sp = key_splitters(keys, world)
+        bnd = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [c["T"]]
+        lk, lv = keys[bnd[rank]:bnd[rank + 1]], vals[bnd[rank]:bnd[rank + 1]]
+        pt = PartitionedTree(torch.from_numpy(lk).to(dev), torch.from_numpy(lv).to(dev), sp, fanout=c["F"],
+                             fill=a.fill, device=dev)
+        t = pt.ops.tree
+    else:
+        t = hm.Tree(torch.from_numpy(keys).to(dev), torch.from_numpy(vals).to(dev), fanout=c["F"], fill=a.fill)
     info = t.info()
     q_np = make_queries(keys, c["Q"], c["dist"], rank)
     q_host = torch.from_numpy(q_np).pin_memory()
     q = q_host.to(dev)
     out = torch.empty_like(q)
-    opts = hm.make_opts(a.group_size, a.psa_bits, a.smem_levels, a.window, a.flags)
     plan = t.plan(c["Q"], opts)
 
     def step():
-        t.search(q, out, opts=opts)
+        if pt is not None:
+            out.copy_(pt.search(q))
+        else:
+            t.search(q, out, opts=opts)
 
     if a.sweep:
         for spec in a.sweep.split(";"):
@@ -349,7 +366,15 @@ def main():
     e2e = None
     if not a.no_e2e:
         out_host = torch.empty(c["Q"], dtype=torch.uint64, pin_memory=True)
-        t.search_host(q_host, out_host, opts=opts)
+
+        def e2e_step():
+            if pt is not None:  # H2D, routed search, D2H through the same public objects
+                q.copy_(q_host, non_blocking=True)
+                out_host.copy_(pt.search(q), non_blocking=True)
+            else:
+                t.search_host(q_host, out_host, opts=opts)
+
+        e2e_step()
         torch.cuda.synchronize()
         barrier()
         torch.cuda.synchronize()
@@ -357,7 +382,7 @@ def main():
         k2 = max(1, a.e2e_steps)
         h0.record(stream)
         for _ in range(k2):
-            t.search_host(q_host, out_host, opts=opts)
+            e2e_step()
         h1.record(stream)
         torch.cuda.synchronize()
         hms = h0.elapsed_time(h1)
@@ -369,7 +394,9 @@ def main():
         parity_ok = parity_ok and e2e_ok
         e2e = {"value": c["Q"] * world * k2 / (hms / 1e3) / 1e9, "unit": UNIT,
                "h2d_bytes_per_step": int(c["Q"] * 8), "d2h_bytes_per_step": int(c["Q"] * 8),
-               "steps": k2, "ms_per_step": hms / k2, "api": "harmonia_search_batch_host (pinned)"}
+               "steps": k2, "ms_per_step": hms / k2,
+               "api": "PartitionedTree.search + pinned copies" if pt is not None else
+               "harmonia_search_batch_host (pinned)"}
 
     if rank != 0:
         if pg:
@@ -429,7 +456,7 @@ def main():
         "warmup": max(3, a.warmup), "ms_per_step": ms_max / a.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": c["name"], "T": c["T"], "fanout": c["F"], "fill": a.fill, "Q_per_gpu": c["Q"],
-                   "queries": c["dist"], "mode": "replicated" if world > 1 else "single",
+                   "queries": c["dist"], "mode": a.mode if (world > 1 or a.mode == "partitioned") else "single",
                    "l2_flush": "inputs_larger_than_L2 (queries+results %d MiB/GPU > L2 %d MiB)" % (
                        c["Q"] * 16 >> 20, l2_bytes >> 20),
                    "plan": plan, "height": info["height"]},

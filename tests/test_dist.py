@@ -1,0 +1,137 @@
+"""Multi-process (gloo, world_size 2 and 3) tests of the partitioned-mode exchange logic.
+
+The device steps (route / local search / local range / scatter back) are replaced by CPU
+stand-ins built on the oracle, so these tests check the host-side routing, splits, the
+all_to_all exchanges and the reassembly of points and multi-shard ranges against the oracle
+over the *global* key set.  The CUDA ops themselves are checked in tests/test_gpu_*.py."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import harmonia_gen as gen
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+class CpuOps:
+    """Oracle-backed stand-ins for the CUDA steps of PartitionedTree (test only)."""
+
+    def __init__(self, keys, vals, splitters, P):
+        import oracle
+
+        self.orc, self.keys, self.vals = oracle, keys, vals
+        self.split = np.asarray(splitters, dtype=np.uint64)
+        self.P = P
+
+    def route(self, q):
+        qn = q.view(torch.int64).numpy().view(np.uint64)
+        dest = np.searchsorted(self.split, qn, side="right")
+        pos = np.argsort(dest, kind="stable")
+        counts = np.bincount(dest, minlength=self.P).tolist()
+        return (torch.from_numpy(qn[pos].view(np.int64).copy()).view(torch.uint64),
+                torch.from_numpy(pos.astype(np.int64)), counts)
+
+    def search(self, q):
+        qn = q.view(torch.int64).numpy().view(np.uint64)
+        out = self.orc.sorted_search(self.keys, self.vals, qn, 1)
+        return torch.from_numpy(out.view(np.int64).copy()).view(torch.uint64)
+
+    def range(self, lo, hi, cap):
+        ko, vo, cnt = self.orc.sorted_range(self.keys, self.vals, lo.view(torch.int64).numpy().view(np.uint64),
+                                            hi.view(torch.int64).numpy().view(np.uint64), cap, 1)
+        m = lo.numel()
+        if cap:  # untouched slab entries are unspecified; make them PAD like the CUDA path
+            mask = np.arange(cap)[None, :] >= np.minimum(cnt.astype(np.int64), cap)[:, None]
+            ko = ko.reshape(m, cap).copy()
+            vo = vo.reshape(m, cap).copy()
+            ko[mask] = np.uint64(0xFFFFFFFFFFFFFFFF)
+            vo[mask] = np.uint64(0xFFFFFFFFFFFFFFFF)
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy()).view(torch.uint64)
+        return (t(ko) if cap else None), (t(vo) if cap else None), torch.from_numpy(cnt.astype(np.int64))
+
+    def scatter(self, vals, pos):
+        out = torch.empty_like(vals.view(torch.int64))
+        out[pos] = vals.view(torch.int64)
+        return out.view(torch.uint64)
+
+
+def _worker(rank, world, port, T, cap, result_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree, key_splitters
+
+        keys = gen.uniform_keys(T)
+        vals = gen.values_for(keys)
+        sp = key_splitters(keys, world)
+        bounds = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
+        lk, lv = keys[bounds[rank]:bounds[rank + 1]], vals[bounds[rank]:bounds[rank + 1]]
+        ops = CpuOps(lk, lv, sp, world)
+        pt = PartitionedTree(lk, lv, sp, ops=ops)
+        # point queries: hits, misses, edges, splitter keys themselves
+        q = np.concatenate([gen.uniform_queries(keys, 3000 + 17 * rank, seed=gen.SEED_QUERY + rank, miss_frac=0.3),
+                            gen.edge_queries(keys), np.asarray(sp, dtype=np.uint64),
+                            np.asarray(sp, dtype=np.uint64) - np.uint64(1)])
+        qt = torch.from_numpy(q.view(np.int64).copy()).view(torch.uint64)
+        got = pt.search(qt).view(torch.int64).numpy().view(np.uint64)
+        exp = oracle.sorted_search(keys, vals, q)
+        ok_pts = bool(np.array_equal(got, exp))
+        # ranges: short, long (crossing several shards), empty, lo > hi, full span
+        lo1, hi1 = gen.ranges(keys, 200, 40, seed=gen.SEED_RANGE + rank)
+        lo2, hi2 = gen.random_ranges(keys, 200, seed=gen.SEED_RANGE + 7 * rank, max_width_keys=T)
+        lo = np.concatenate([lo1, lo2, [0, 5, int(keys[-1])], np.asarray(sp, dtype=np.uint64)])
+        hi = np.concatenate([hi1, hi2, [(1 << 64) - 1, 4, (1 << 64) - 1],
+                             np.asarray(sp, dtype=np.uint64) + np.uint64(3)])
+        lo, hi = lo.astype(np.uint64), hi.astype(np.uint64)
+        tl = torch.from_numpy(lo.view(np.int64).copy()).view(torch.uint64)
+        th = torch.from_numpy(hi.view(np.int64).copy()).view(torch.uint64)
+        ko, vo, cnt = pt.range(tl, th, cap)
+        eko, evo, ecnt = oracle.sorted_range(keys, vals, lo, hi, cap)
+        ok_rng = bool(np.array_equal(cnt.numpy(), ecnt.astype(np.int64)))
+        if cap:
+            k = ko.view(torch.int64).numpy().view(np.uint64)
+            v = vo.view(torch.int64).numpy().view(np.uint64)
+            m = np.minimum(ecnt.astype(np.int64), cap)
+            mask = np.arange(cap)[None, :] < m[:, None]
+            ok_rng = ok_rng and bool(np.array_equal(k[mask], eko[mask])) and bool(np.array_equal(v[mask], evo[mask]))
+        result_q.put((rank, ok_pts, ok_rng))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,cap", [(2, 16), (3, 0), (3, 64)])
+def test_partitioned_exchange_gloo(world, cap):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, 20000, cap, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, ok_pts, ok_rng in res:
+        assert ok_pts, f"rank {rank}: point results differ from the oracle"
+        assert ok_rng, f"rank {rank}: range results differ from the oracle"
+
+
+def test_splitters_and_slices():
+    from paper_conf_ppopp_yanlpz19_b200.dist import key_splitters
+
+    keys = gen.uniform_keys(1000)
+    sp = key_splitters(keys, 4)
+    assert sp == [int(keys[250]), int(keys[500]), int(keys[750])]
+    assert key_splitters(keys, 1) == []
