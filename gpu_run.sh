@@ -1,3 +1,1 @@
-python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29511 bench.py --gpus 1 --steps 10 --warmup 3 --mode partitioned --no-cpu > gpurun_out/bench_part1.json 2> gpurun_out/bench_part1.err; cat gpurun_out/bench_part1.json | cut -c1-600; tail -3 gpurun_out/bench_part1.err
-python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29512 bench.py --gpus 1 --steps 10 --warmup 3 --no-cpu > gpurun_out/bench_rep1.json 2> gpurun_out/bench_rep1.err; cat gpurun_out/bench_rep1.json | cut -c1-300; tail -3 gpurun_out/bench_rep1.err
-python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29513 bench.py --impl reference --gpus 1 --steps 3 --warmup 1 2>&1 | tail -1 | cut -c1-200
+python -m pytest tests/test_gpu_update.py -m gpu -x -q > gpurun_out/gpu_upd.log 2>&1; tail -30 gpurun_out/gpu_upd.log

@@ -1,15 +1,348 @@
-// Batched update: implemented in a later milestone; the ABI slot is fixed.
+// Batched update (§3.2.2; C-A18) as bulk-synchronous device passes.
+//
+// The paper applies updates on the CPU with two-grained locks, auxiliary nodes for splits and
+// a post-batch "movement" of the key region (Alg 1).  Here the phase model
+// (the update phase has the tree to itself) lets the whole batch be applied at once:
+//   1. validate (no PAD keys, no NOT_FOUND upsert values)            k_upd_validate
+//   2. stable sort of the batch by key (CUB radix sort, positions as payload)
+//   3. last op per key wins (sequential semantics, C-A18)             k_upd_winners + scan
+//   4. extract the current record sequence from the leaves            k_upd_extract
+//   5. classify winners against it: update value in place / delete / insert
+//                                                                     k_upd_classify + scans
+//   6. merge kept records with the inserts (merge path by ranks)       k_upd_merge_*
+//   7. rebuild the layout from the merged sequence (build_layout): the "movement" of P:L314.
+// The affected region of a batch is the leaf suffix from its smallest key; on the GPU
+// re-packing that suffix and the (small) internal levels costs the same passes as the closed
+// form over all leaves, so the layout is rebuilt in full and stays bit-identical to a fresh
+// harmonia_build of the resulting record set (the oracle's closed form, invariant I8).
+#include <cub/cub.cuh>
+
+#include <algorithm>
+
 #include "common.cuh"
 
+namespace hm {
+namespace {
+
+__global__ void k_upd_validate(const uint8_t* __restrict__ ops, const uint64_t* __restrict__ keys,
+                               const uint64_t* __restrict__ vals, uint64_t n, unsigned* flags) {
+  unsigned f = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (keys[i] == kPad) f |= 2u;
+    if (ops[i] == 0 && vals[i] == kNotFound) f |= 2u;
+    if (ops[i] > 1) f |= 4u;
+  }
+  f = __reduce_or_sync(kFull, f);
+  if (f && (threadIdx.x & 31) == 0) atomicOr(flags, f);
+}
+
+__global__ void k_iota(uint32_t* __restrict__ p, uint64_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = (uint32_t)i;
+}
+
+// flag[i] = 1 if sorted entry i is the last op on its key
+__global__ void k_upd_winners(const uint64_t* __restrict__ sk, uint64_t n, uint32_t* __restrict__ flag) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    flag[i] = (i + 1 == n || sk[i + 1] != sk[i]) ? 1u : 0u;
+}
+
+__global__ void k_upd_compact_winners(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ spos,
+                                      const uint32_t* __restrict__ flag, const uint32_t* __restrict__ at, uint64_t n,
+                                      const uint8_t* __restrict__ ops, const uint64_t* __restrict__ vals,
+                                      uint64_t* __restrict__ wk, uint8_t* __restrict__ wop, uint64_t* __restrict__ wv) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (flag[i]) {
+      const uint32_t d = at[i], p = spos[i];
+      wk[d] = sk[i];
+      wop[d] = ops[p];
+      wv[d] = vals[p];
+    }
+  }
+}
+
+// current records in key order: record r lives in leaf j at slot r - leaf_base[j]
+__global__ void k_upd_extract(const uint64_t* __restrict__ kr, const uint64_t* __restrict__ lv,
+                              const uint64_t* __restrict__ leaf_base, uint64_t leaf_start, uint64_t L, uint32_t F,
+                              uint64_t* __restrict__ K, uint64_t* __restrict__ V) {
+  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < L * F; s += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t j = s / F, slot = s % F;
+    const uint64_t b = leaf_base[j], c = leaf_base[j + 1] - b;
+    if (slot < c) {
+      K[b + slot] = kr[(leaf_start + j) * F + slot];
+      V[b + slot] = lv[s];
+    }
+  }
+}
+
+__device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* a, uint64_t n, uint64_t x) {
+  uint64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (a[mid] < x) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// winners vs current records: in-place value update, delete mark, or insert flag
+__global__ void k_upd_classify(const uint64_t* __restrict__ wk, const uint8_t* __restrict__ wop,
+                               const uint64_t* __restrict__ wv, uint64_t nw, const uint64_t* __restrict__ K,
+                               uint64_t* __restrict__ V, uint64_t nk, uint32_t* __restrict__ keep,
+                               uint32_t* __restrict__ ins_flag) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t p = lower_bound_u64(K, nk, wk[i]);
+    const bool exists = p < nk && K[p] == wk[i];
+    uint32_t ins = 0;
+    if (wop[i] == 0) {
+      if (exists) V[p] = wv[i];  // update an existing record's value
+      else ins = 1;              // insert a new record
+    } else if (exists) {
+      keep[p] = 0;               // delete an existing record; a missing key is a no-op
+    }
+    ins_flag[i] = ins;
+  }
+}
+
+__global__ void k_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+// kept record i goes to kpos[i] + #inserts with a smaller key
+__global__ void k_upd_merge_kept(const uint64_t* __restrict__ K, const uint64_t* __restrict__ V,
+                                 const uint32_t* __restrict__ keep, const uint32_t* __restrict__ kpos, uint64_t nk,
+                                 const uint64_t* __restrict__ ik, uint64_t ni, uint64_t* __restrict__ NK,
+                                 uint64_t* __restrict__ NV) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nk; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (keep[i]) {
+      const uint64_t d = kpos[i] + lower_bound_u64(ik, ni, K[i]);
+      NK[d] = K[i];
+      NV[d] = V[i];
+    }
+  }
+}
+
+// insert j goes to j + #kept records with a smaller key
+__global__ void k_upd_merge_ins(const uint64_t* __restrict__ ik, const uint64_t* __restrict__ iv, uint64_t ni,
+                                const uint64_t* __restrict__ K, const uint32_t* __restrict__ kpos, uint64_t nk,
+                                uint64_t* __restrict__ NK, uint64_t* __restrict__ NV) {
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < ni; j += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t p = lower_bound_u64(K, nk, ik[j]);
+    const uint64_t d = j + kpos[p];
+    NK[d] = ik[j];
+    NV[d] = iv[j];
+  }
+}
+
+__global__ void k_upd_compact_ins(const uint64_t* __restrict__ wk, const uint64_t* __restrict__ wv,
+                                  const uint32_t* __restrict__ ins_flag, const uint32_t* __restrict__ ins_at, uint64_t nw,
+                                  uint64_t* __restrict__ ik, uint64_t* __restrict__ iv) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x)
+    if (ins_flag[i]) {
+      ik[ins_at[i]] = wk[i];
+      iv[ins_at[i]] = wv[i];
+    }
+}
+
+int grid_of(uint64_t n, int sm) {
+  return (int)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(std::max<uint64_t>(n, 1), kBlock), (uint64_t)sm * 8));
+}
+
+// workspace layout (byte offsets), for batch n and current record count nk
+struct UpdWs {
+  size_t cub, sk, sk2, pos, pos2, flag, at, wk, wop, wv, K, V, keep, kpos, insf, insat, ik, iv, NK, NV, total;
+};
+
+UpdWs upd_layout(uint64_t n, uint64_t nk, size_t cub_bytes) {
+  UpdWs w{};
+  size_t o = 0;
+  auto take = [&](size_t b) {
+    size_t r = o;
+    o += round_up(std::max<size_t>(b, 1), 256);
+    return r;
+  };
+  w.cub = take(cub_bytes);
+  w.sk = take(n * 8);
+  w.sk2 = take(n * 8);
+  w.pos = take(n * 4);
+  w.pos2 = take(n * 4);
+  w.flag = take((n + 1) * 4);
+  w.at = take((n + 1) * 4);
+  w.wk = take(n * 8);
+  w.wop = take(n);
+  w.wv = take(n * 8);
+  w.K = take(nk * 8);
+  w.V = take(nk * 8);
+  w.keep = take((nk + 1) * 4);
+  w.kpos = take((nk + 1) * 4);
+  w.insf = take((n + 1) * 4);
+  w.insat = take((n + 1) * 4);
+  w.ik = take(n * 8);
+  w.iv = take(n * 8);
+  w.NK = take((nk + n) * 8);
+  w.NV = take((nk + n) * 8);
+  w.total = o;
+  return w;
+}
+
+size_t cub_temp_bytes(uint64_t n, uint64_t nk) {
+  size_t a = 0, b = 0, c = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, a, (const uint64_t*)nullptr, (uint64_t*)nullptr, (const uint32_t*)nullptr,
+                                  (uint32_t*)nullptr, (int)std::max<uint64_t>(n, 1));
+  cub::DeviceScan::ExclusiveSum(nullptr, b, (const uint32_t*)nullptr, (uint32_t*)nullptr,
+                                (int)std::max<uint64_t>(n + 1, 1));
+  cub::DeviceScan::ExclusiveSum(nullptr, c, (const uint32_t*)nullptr, (uint32_t*)nullptr,
+                                (int)std::max<uint64_t>(nk + 1, 1));
+  return std::max({a, b, c});
+}
+
+}  // namespace
+}  // namespace hm
+
+using namespace hm;
+
 extern "C" size_t harmonia_update_workspace_bytes(const harmonia_tree* t, uint64_t n) {
-  (void)t;
-  (void)n;
-  return 0;
+  if (!t) return 0;
+  return upd_layout(n, t->n_keys, cub_temp_bytes(n, t->n_keys)).total + 256;
 }
 
 extern "C" harmonia_status harmonia_update_batch(harmonia_tree* t, const uint8_t* d_ops, const uint64_t* d_keys,
                                                  const uint64_t* d_values, uint64_t n, void* ws, size_t ws_bytes,
                                                  void* stream) {
-  (void)t; (void)d_ops; (void)d_keys; (void)d_values; (void)n; (void)ws; (void)ws_bytes; (void)stream;
-  return HARMONIA_ERR_INVALID_ARG;
+  if (!t) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!d_ops || !d_keys || !d_values || !ws) return HARMONIA_ERR_INVALID_ARG;
+  if (n >= (1ull << 31)) return HARMONIA_ERR_INVALID_ARG;
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint64_t nk = t->n_keys;
+  const size_t cubb = cub_temp_bytes(n, nk);
+  const UpdWs L = upd_layout(n, nk, cubb);
+  char* base = (char*)ws;
+  if ((uintptr_t)base & 255) {
+    const size_t adj = 256 - ((uintptr_t)base & 255);
+    if (ws_bytes < adj) return HARMONIA_ERR_INVALID_ARG;
+    base += adj;
+    ws_bytes -= adj;
+  }
+  if (ws_bytes < L.total) return HARMONIA_ERR_INVALID_ARG;
+  auto P = [&](size_t off) { return (void*)(base + off); };
+  const int sm = t->sm_count;
+  ProfScope prof(HARMONIA_PROF_UPDATE, st);
+
+  // 1. validate
+  unsigned* d_flags = (unsigned*)P(L.flag);
+  HM_CUDA(cudaMemsetAsync(d_flags, 0, 4, st));
+  k_upd_validate<<<grid_of(n, sm), kBlock, 0, st>>>(d_ops, d_keys, d_values, n, d_flags);
+  HM_LAUNCHED();
+  unsigned flags = 0;
+  HM_CUDA(cudaMemcpyAsync(&flags, d_flags, 4, cudaMemcpyDeviceToHost, st));
+  HM_CUDA(cudaStreamSynchronize(st));
+  if (flags & 2u) return HARMONIA_ERR_RESERVED;
+  if (flags & 4u) return HARMONIA_ERR_INVALID_ARG;
+
+  // 2. stable sort by key, batch position as payload
+  uint64_t *sk = (uint64_t*)P(L.sk), *sk2 = (uint64_t*)P(L.sk2);
+  uint32_t *pos = (uint32_t*)P(L.pos), *pos2 = (uint32_t*)P(L.pos2);
+  k_iota<<<grid_of(n, sm), kBlock, 0, st>>>(pos, n);
+  HM_LAUNCHED();
+  size_t cb = cubb;
+  HM_CUDA(cub::DeviceRadixSort::SortPairs(P(L.cub), cb, d_keys, sk2, pos, pos2, (int)n, 0, 64, st));
+  count_launch(4);
+  (void)sk;
+  // 3. winners (last op per key) and their compaction
+  uint32_t *flag = (uint32_t*)P(L.flag), *at = (uint32_t*)P(L.at);
+  k_upd_winners<<<grid_of(n, sm), kBlock, 0, st>>>(sk2, n, flag);
+  HM_LAUNCHED();
+  HM_CUDA(cudaMemsetAsync(flag + n, 0, 4, st));
+  cb = cubb;
+  HM_CUDA(cub::DeviceScan::ExclusiveSum(P(L.cub), cb, flag, at, (int)(n + 1), st));
+  count_launch(2);
+  uint32_t nw32 = 0;
+  HM_CUDA(cudaMemcpyAsync(&nw32, at + n, 4, cudaMemcpyDeviceToHost, st));
+  uint64_t *wk = (uint64_t*)P(L.wk), *wv = (uint64_t*)P(L.wv);
+  uint8_t* wop = (uint8_t*)P(L.wop);
+  k_upd_compact_winners<<<grid_of(n, sm), kBlock, 0, st>>>(sk2, pos2, flag, at, n, d_ops, d_values, wk, wop, wv);
+  HM_LAUNCHED();
+  HM_CUDA(cudaStreamSynchronize(st));
+  const uint64_t nw = nw32;
+
+  // 4. current records
+  uint64_t *K = (uint64_t*)P(L.K), *V = (uint64_t*)P(L.V);
+  if (nk > 0) {
+    k_upd_extract<<<grid_of(t->L * t->F, sm), kBlock, 0, st>>>(t->d_keys, t->d_vals, t->d_leaf_base,
+                                                               t->level_start[t->h - 1], t->L, t->F, K, V);
+    HM_LAUNCHED();
+  }
+  // 5. classify
+  uint32_t *keep = (uint32_t*)P(L.keep), *kpos = (uint32_t*)P(L.kpos);
+  uint32_t *insf = (uint32_t*)P(L.insf), *insat = (uint32_t*)P(L.insat);
+  k_fill_u32<<<grid_of(nk + 1, sm), kBlock, 0, st>>>(keep, nk + 1, 1u);
+  HM_LAUNCHED();
+  HM_CUDA(cudaMemsetAsync(keep + nk, 0, 4, st));
+  HM_CUDA(cudaMemsetAsync(insf + nw, 0, 4, st));
+  k_upd_classify<<<grid_of(nw, sm), kBlock, 0, st>>>(wk, wop, wv, nw, K, V, nk, keep, insf);
+  HM_LAUNCHED();
+  cb = cubb;
+  HM_CUDA(cub::DeviceScan::ExclusiveSum(P(L.cub), cb, keep, kpos, (int)(nk + 1), st));
+  count_launch(2);
+  cb = cubb;
+  HM_CUDA(cub::DeviceScan::ExclusiveSum(P(L.cub), cb, insf, insat, (int)(nw + 1), st));
+  count_launch(2);
+  uint32_t nkeep = 0, nins = 0;
+  HM_CUDA(cudaMemcpyAsync(&nkeep, kpos + nk, 4, cudaMemcpyDeviceToHost, st));
+  HM_CUDA(cudaMemcpyAsync(&nins, insat + nw, 4, cudaMemcpyDeviceToHost, st));
+  uint64_t *ik = (uint64_t*)P(L.ik), *iv = (uint64_t*)P(L.iv);
+  k_upd_compact_ins<<<grid_of(nw, sm), kBlock, 0, st>>>(wk, wv, insf, insat, nw, ik, iv);
+  HM_LAUNCHED();
+  HM_CUDA(cudaStreamSynchronize(st));
+
+  // 6. merge
+  const uint64_t nn = (uint64_t)nkeep + nins;
+  uint64_t *NK = (uint64_t*)P(L.NK), *NV = (uint64_t*)P(L.NV);
+  if (nk > 0) {
+    k_upd_merge_kept<<<grid_of(nk, sm), kBlock, 0, st>>>(K, V, keep, kpos, nk, ik, nins, NK, NV);
+    HM_LAUNCHED();
+  }
+  if (nins > 0) {
+    k_upd_merge_ins<<<grid_of(nins, sm), kBlock, 0, st>>>(ik, iv, nins, K, kpos, nk, NK, NV);
+    HM_LAUNCHED();
+  }
+  // 7. rebuild the layout (new arrays; the old ones are released after the build)
+  harmonia_tree old = *t;
+  t->d_keys = nullptr;
+  t->d_vals = nullptr;
+  t->d_ps = nullptr;
+  t->d_leaf_base = nullptr;
+  harmonia_status s = build_layout(t, NK, NV, nn, st);
+  if (s != HARMONIA_OK) {
+    cudaFree(t->d_keys);
+    cudaFree(t->d_vals);
+    cudaFree(t->d_ps);
+    cudaFree(t->d_leaf_base);
+    t->d_keys = old.d_keys;  // tree unchanged on failure
+    t->d_vals = old.d_vals;
+    t->d_ps = old.d_ps;
+    t->d_leaf_base = old.d_leaf_base;
+    t->h = old.h;
+    t->N = old.N;
+    t->I = old.I;
+    t->L = old.L;
+    t->n_keys = old.n_keys;
+    for (int l = 0; l <= HARMONIA_MAX_LEVELS; ++l) t->level_start[l] = old.level_start[l];
+    return s;
+  }
+  cudaFree(old.d_keys);
+  cudaFree(old.d_vals);
+  cudaFree(old.d_ps);
+  cudaFree(old.d_leaf_base);
+  if (nn > 0) {
+    HM_CUDA(cudaMemcpyAsync(&t->min_key, NK, 8, cudaMemcpyDeviceToHost, st));
+    HM_CUDA(cudaMemcpyAsync(&t->max_key, NK + nn - 1, 8, cudaMemcpyDeviceToHost, st));
+    HM_CUDA(cudaStreamSynchronize(st));
+  } else {
+    t->min_key = kPad;
+    t->max_key = 0;
+  }
+  return HARMONIA_OK;
 }

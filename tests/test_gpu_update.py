@@ -1,0 +1,119 @@
+"""GPU parity of harmonia_update_batch against the std::map update oracle (O6).
+
+After every batch the exported layout must equal the oracle's closed-form layout of the
+resulting record set bit for bit (the update rebuilds the layout), pass the
+invariant checker, and answer point/range queries exactly like the oracle."""
+import numpy as np
+import pytest
+
+import harmonia_gen as gen
+
+pytestmark = pytest.mark.gpu
+MAX = (1 << 64) - 1
+
+
+@pytest.fixture(scope="module")
+def hm():
+    import torch
+
+    assert torch.cuda.is_available()
+    import paper_conf_ppopp_yanlpz19_b200 as m
+
+    m.lib()
+    return m
+
+
+def cu(a):
+    import torch
+
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def check_tree(hm, orc, t, F, ref_keys, ref_vals, probe):
+    info, kr, ps, lv = t.export_layout()
+    lay = orc.layout_build(ref_keys, ref_vals, F, 1.0)
+    assert info["n_keys"] == ref_keys.shape[0]
+    assert np.array_equal(kr, lay.key_region) and np.array_equal(ps, lay.ps) and np.array_equal(lv, lay.leaf_vals)
+    code, msg = orc.Layout(F, info["height"], info["level_start"], kr, ps, lv).check(ref_keys, ref_vals)
+    assert code == 0, msg
+    out = t.search(cu(probe)).cpu().numpy()
+    assert np.array_equal(out, orc.sorted_search(ref_keys, ref_vals, probe))
+    lo, hi = gen.random_ranges(ref_keys, 500)
+    ko, vo, cnt = t.range(cu(lo), cu(hi), 8)
+    eko, evo, ecnt = orc.sorted_range(ref_keys, ref_vals, lo, hi, 8)
+    assert np.array_equal(cnt.cpu().numpy(), ecnt)
+    m = np.minimum(ecnt.astype(np.int64), 8)
+    mask = np.arange(8)[None, :] < m[:, None]
+    assert np.array_equal(ko.cpu().numpy()[mask], eko[mask]) and np.array_equal(vo.cpu().numpy()[mask], evo[mask])
+
+
+@pytest.mark.parametrize("F", [4, 16, 64])
+def test_update_batches_match_oracle(hm, orc, F):
+    keys = gen.uniform_keys(30000)
+    vals = gen.values_for(keys)
+    t = hm.Tree(cu(keys), cu(vals), fanout=F)
+    ref = orc.UpdateMap(keys, vals)
+    touched = []
+    for b in range(4):
+        ops, ks, vs = gen.update_ops(keys, 8000, insert_frac=0.05 + 0.1 * b, delete_frac=0.05 * b,
+                                     seed=gen.SEED_OPS + 31 * b + F)
+        # repeated keys inside one batch: the last op must win (C-A18)
+        ops = np.concatenate([ops, ops[:500] ^ np.uint8(1)])
+        ks = np.concatenate([ks, ks[:500]])
+        vs = np.concatenate([vs, vs[:500] + np.uint64(7)])
+        t.update(ops, cu(ks), cu(vs))
+        ref.apply(ops, ks, vs)
+        touched.append(ks)
+        rk, rv = ref.dump()
+        probe = np.concatenate([np.concatenate(touched), gen.uniform_queries(rk, 20000, miss_frac=0.3)])
+        check_tree(hm, orc, t, F, rk, rv, probe)
+
+
+def test_update_edge_cases(hm, orc):
+    keys = np.arange(1, 200, dtype=np.uint64) * np.uint64(10)
+    vals = gen.values_for(keys)
+    t = hm.Tree(cu(keys), cu(vals), fanout=8)
+    ref = orc.UpdateMap(keys, vals)
+    # delete everything -> empty tree
+    ops = np.ones(keys.shape[0], dtype=np.uint8)
+    t.update(ops, cu(keys), cu(vals))
+    ref.apply(ops, keys, vals)
+    assert t.info()["n_keys"] == 0
+    q = np.concatenate([keys, gen.edge_queries(keys)])
+    assert np.all(t.search(cu(q)).cpu().numpy() == np.uint64(MAX))
+    # insert into the empty tree, including key 0 and MAX-1
+    ks = np.array([5, 0, MAX - 1, 77, 5], dtype=np.uint64)
+    vs = np.array([1, 2, 3, 4, 9], dtype=np.uint64)
+    ops = np.zeros(5, dtype=np.uint8)
+    t.update(ops, cu(ks), cu(vs))
+    ref.apply(ops, ks, vs)
+    rk, rv = ref.dump()
+    check_tree(hm, orc, t, 8, rk, rv, np.concatenate([ks, gen.edge_queries(rk)]))
+    # reserved key / value -> RESERVED, tree unchanged
+    before = t.export_layout()
+    with pytest.raises(hm.HarmoniaError, match="RESERVED"):
+        t.update(np.zeros(1, dtype=np.uint8), cu(np.array([MAX], dtype=np.uint64)), cu(np.array([1], dtype=np.uint64)))
+    with pytest.raises(hm.HarmoniaError, match="RESERVED"):
+        t.update(np.zeros(1, dtype=np.uint8), cu(np.array([3], dtype=np.uint64)), cu(np.array([MAX], dtype=np.uint64)))
+    after = t.export_layout()
+    for x, y in zip(before[1:], after[1:]):
+        assert np.array_equal(x, y)
+    # delete of a missing key is a no-op; a delete value may be anything
+    t.update(np.ones(1, dtype=np.uint8), cu(np.array([123456], dtype=np.uint64)), cu(np.array([MAX], dtype=np.uint64)))
+    check_tree(hm, orc, t, 8, rk, rv, rk)
+
+
+def test_paper_scale_update_batch(hm, orc):
+    """batches of 4096K ops, 5 % inserts + 95 % updates, on a 2^23-key tree."""
+    keys = gen.uniform_keys(1 << 23)
+    vals = gen.values_for(keys)
+    t = hm.Tree(cu(keys), cu(vals), fanout=64)
+    ops, ks, vs = gen.update_ops(keys, 1 << 22, insert_frac=0.05)
+    t.update(ops, cu(ks), cu(vs))
+    ref = orc.UpdateMap(keys, vals)
+    ref.apply(ops, ks, vs)
+    rk, rv = ref.dump()
+    assert t.info()["n_keys"] == rk.shape[0]
+    sel = gen._stream(5, 0, 1 << 18) % np.uint64(rk.shape[0])
+    probe = np.concatenate([rk[sel], ks[: 1 << 18]])
+    assert np.array_equal(t.search(cu(probe)).cpu().numpy(), orc.sorted_search(rk, rv, probe))
