@@ -71,9 +71,10 @@ def lib():
     """Load libharmonia.so (building it in-tree if it is missing).  Raises if unavailable."""
     global _lib
     if _lib is None:
-        if not os.path.exists(_build.LIB):
+        path = os.environ.get("HARMONIA_LIB") or _build.LIB  # HARMONIA_LIB: an alternative build (experiments)
+        if path == _build.LIB and not os.path.exists(path):
             _build.build()
-        L = C.CDLL(_build.LIB)
+        L = C.CDLL(path)
         sig = {
             "harmonia_build": (C.c_int, [_vp, _vp, _u64, C.POINTER(BuildOpts), _vp, C.POINTER(_vp)]),
             "harmonia_destroy": (None, [_vp]),
