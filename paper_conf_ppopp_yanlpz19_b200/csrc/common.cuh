@@ -159,7 +159,7 @@ struct SearchArgs {
   uint64_t* out;           // results: out[idx ? idx[j] : j]
 };
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
-                               int sm_count, cudaStream_t st);
+                               int sm_count, cudaStream_t st, bool ballot_sort = false);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
                               cudaStream_t st);
 

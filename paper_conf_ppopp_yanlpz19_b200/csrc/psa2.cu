@@ -286,10 +286,14 @@ __global__ void __launch_bounds__(kSortThreads, 2) k_psa2_local_sort(uint64_t* _
   }
 }
 
+constexpr int kLocalBins = 1 << kLocalBits;
+constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12;
+#include "psa2_count_sort.inc"
+
 }  // namespace
 
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
-                               cudaStream_t st) {
+                               cudaStream_t st, bool ballot_sort) {
   const uint32_t b1 = (uint32_t)std::min(nb, kCoarseBits);
   const uint32_t shift1 = (uint32_t)nb - b1;
   HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * kCoarseBins * 4, st));
@@ -311,10 +315,15 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
     static bool configured = false;
     if (!configured) {
       HM_CUDA(cudaFuncSetAttribute(k_psa2_local_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSortSmem));
+      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)kCountSortSmem));
       configured = true;
     }
     const int g = (int)std::min<uint64_t>(ceil_div(n, kChunk), (uint64_t)sm * 4);
-    k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
+    if (ballot_sort)  // two stable LSD passes of ballot multisplit (ablation)
+      k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
+    else              // one counting pass with shared-memory atomics (default, measured faster)
+      k_psa2_count_sort<<<std::max(g, 1), kSortThreads, kCountSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
   }
   HM_LAUNCHED();
   return HARMONIA_OK;

@@ -155,38 +155,36 @@ __device__ __forceinline__ uint32_t ntg_rank(const uint64_t* nk, uint64_t q, uns
 // log_G(F/2G)+1 steps, so there is no early-exit divergence inside the warp (the query
 // divergence of P:L500 disappears) and the comparisons per level drop from O(F/2G) steps
 // to O(log F).  Inactive groups must pass a q that keeps spans inside the node (q = 0).
-template <int S, int G, bool SMEM, bool STRICT, bool EQ>
+template <int S, int G, bool SMEM, bool STRICT>
 struct KaryStep {
   static __device__ __forceinline__ uint32_t run(const uint64_t* nk, uint32_t base, uint64_t q, int gl,
-                                                 uint32_t gmask, unsigned& fe) {
+                                                 uint32_t gmask) {
     if constexpr (S / 2 <= G) {
       constexpr int L = S / 2;  // final step: L lanes read the span contiguously
       ulonglong2 k = make_ulonglong2(kPad, kPad);
-      if constexpr (L < G) ld_pair_if<SMEM>(k, nk + base + 2 * gl, gl < L);
-      else k = ld_pair<SMEM>(nk + base + 2 * gl);
+      if constexpr (L < G) ld_pair_if<SMEM>(k, nk + (base + 2 * gl), gl < L);
+      else k = ld_pair<SMEM>(nk + (base + 2 * gl));
       const unsigned bx = ballot(STRICT ? k.x < q : k.x <= q);
       const unsigned by = ballot(STRICT ? k.y < q : k.y <= q);
-      if constexpr (EQ) fe |= ballot((k.x == q) | (k.y == q));
       return base + __popc(bx & gmask) + __popc(by & gmask);
     } else {
       constexpr int B = S / G;  // coarse step: lane gl holds the last two keys of block gl
-      const ulonglong2 k = ld_pair<SMEM>(nk + base + gl * B + (B - 2));
+      const ulonglong2 k = ld_pair<SMEM>(nk + (base + gl * B + (B - 2)));
       const unsigned by = ballot(STRICT ? k.y < q : k.y <= q);
-      if constexpr (EQ) fe |= ballot((k.x == q) | (k.y == q));
       // blocks whose last key is <= q lie entirely before the rank (the span's last key is
       // > q, so at most G-1 of them)
-      return KaryStep<B, G, SMEM, STRICT, EQ>::run(nk, base + (uint32_t)__popc(by & gmask) * B, q, gl, gmask, fe);
+      return KaryStep<B, G, SMEM, STRICT>::run(nk, base + (uint32_t)__popc(by & gmask) * B, q, gl, gmask);
     }
   }
 };
 
+// (k-ary never needs an equality ballot: the leaf probe re-reads key[r-1] with the value)
 template <int F, int G, bool SMEM, bool STRICT, bool EQ>
 __device__ __forceinline__ uint32_t kary_rank(const uint64_t* nk, uint64_t q, int gl, uint32_t gmask,
                                               bool* found) {
-  unsigned fe = 0;
-  const uint32_t r = KaryStep<F, G, SMEM, STRICT, EQ>::run(nk, 0, q, gl, gmask, fe);
-  if constexpr (EQ) *found = (fe & gmask) != 0;
-  return r;
+  static_assert(!EQ, "k-ary rank has no equality output");
+  (void)found;
+  return KaryStep<F, G, SMEM, STRICT>::run(nk, 0, q, gl, gmask);
 }
 
 // in-node rank dispatch: MODE 0 = linear NTG (Fig 9), MODE 1 = k-ary NTG
@@ -255,18 +253,23 @@ __global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_search(const SearchArgs 
     if (a.idx && active && gl == 0) o = ld_stream32(a.idx + j);
     const uint32_t leaf =
         descend<F, G, MODE>(q, live, act, a.h, a.smem_levels, s_keys, s_ps, ps_smem, a.keys, a.ps, grp, gl, gmask);
-    // leaf probe ("the target key is found"): r = #keys <= q, hit iff key[r-1] == q
-    bool found = false;
+    // leaf probe ("the target key is found"): r = #keys <= q; the key is present iff
+    // key[r-1] == q.  key[r-1] and value[r-1] are read together (one L1 round trip) instead
+    // of carrying an equality ballot through every in-node step.
     uint32_t r;
+    const uint64_t* lk = a.keys + (uint64_t)leaf * F;
     const uint64_t* lv = a.vals + (uint64_t)(leaf - a.leaf_start) * F;
-    if (leaf_smem) {
-      r = node_rank<F, G, MODE, true, false, true>(s_keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, &found);
-    } else {
-      r = node_rank<F, G, MODE, false, false, true>(a.keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, &found);
-    }
+    if (leaf_smem)
+      r = node_rank<F, G, MODE, true, false, false>(s_keys + (uint64_t)leaf * F, q, live, act, grp, gl, gmask, nullptr);
+    else
+      r = node_rank<F, G, MODE, false, false, false>(lk, q, live, act, grp, gl, gmask, nullptr);
     if (active && gl == 0) {
       uint64_t v = kNotFound;
-      if (live && found) v = __ldg(lv + (r - 1));
+      if (live && r > 0) {
+        const uint64_t kk = __ldg(lk + (r - 1));
+        const uint64_t vv = __ldg(lv + (r - 1));
+        if (kk == q) v = vv;
+      }
       a.out[o] = v;
     }
   }
