@@ -188,7 +188,9 @@ extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t 
 
 // ---- host-buffer pipeline --------------------------------------------------------------
 static uint64_t host_chunk(const Plan& p, uint64_t n) {
-  uint64_t c = p.psa ? p.window : (1ull << 22);
+  // 4M-query chunks: the copies (PCIe-bound) dominate, so a deeper pipeline beats larger
+  // PSA windows here
+  uint64_t c = std::min<uint64_t>(p.psa ? p.window : (1ull << 22), 1ull << 22);
   return std::max<uint64_t>(1024, std::min<uint64_t>(c, round_up(std::max<uint64_t>(n, 1), 1024)));
 }
 

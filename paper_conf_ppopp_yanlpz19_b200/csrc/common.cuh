@@ -15,7 +15,14 @@ constexpr uint64_t kPad = 0xFFFFFFFFFFFFFFFFull;       // HARMONIA_KEY_PAD
 constexpr uint64_t kNotFound = 0xFFFFFFFFFFFFFFFFull;  // HARMONIA_NOT_FOUND
 constexpr unsigned kFull = 0xFFFFFFFFu;
 constexpr int kBlock = 256;        // threads per CTA for the streaming kernels
-constexpr int kQueryBlock = 1024;  // search/range CTAs: 2 per SM, so the staged tree top is
+#ifndef HM_QUERY_BLOCK
+#define HM_QUERY_BLOCK 1024
+#endif
+#ifndef HM_QBPSM
+#define HM_QBPSM 2
+#endif
+constexpr int kQueryBlocksPerSM = HM_QBPSM;
+constexpr int kQueryBlock = HM_QUERY_BLOCK;  // search/range CTAs: 2 per SM, so the staged tree top is
                                    // duplicated twice per SM and L1 keeps most of its capacity
 
 // ---- error plumbing --------------------------------------------------------------

@@ -228,7 +228,7 @@ __device__ __forceinline__ uint32_t descend(uint64_t q, bool live, unsigned act,
 }
 
 template <int F, int G, int MODE>
-__global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_search(const SearchArgs a) {
+__global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_search(const SearchArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
   stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
@@ -277,7 +277,7 @@ __global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_search(const SearchArgs 
 
 // Range scan: descend with lo, then walk leaf slots in key-region order.
 template <int F, int G, int MODE>
-__global__ void __launch_bounds__(kQueryBlock, 2) k_ntg_range(const RangeArgs a) {
+__global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(const RangeArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
   stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
