@@ -79,6 +79,7 @@ typedef struct {
 #define HARMONIA_QF_NO_PS_SMEM 1u  /* do not stage the prefix-sum array in shared memory     */
 #define HARMONIA_QF_GATHER     2u  /* PSA return via a separate gather pass instead of the
                                       search kernel scattering results in place             */
+#define HARMONIA_QF_ILP1       16u /* k-ary search with one query per lane group instead of two */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic
                                       per query) instead of the default two-level partition  */
 #define HARMONIA_QF_LINEAR     4u  /* in-node search = the paper's linear NTG walk (Fig 9:

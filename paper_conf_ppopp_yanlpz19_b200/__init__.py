@@ -23,6 +23,7 @@ QF_NO_PS_SMEM = 1
 QF_GATHER = 2
 QF_LINEAR = 4
 QF_PSA_GLOBAL = 8
+QF_ILP1 = 16
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
            6: "DEVICE_MISMATCH", 7: "TOO_LARGE"}
 

@@ -53,6 +53,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   }
   P.gather = (o->flags & HARMONIA_QF_GATHER) != 0;
   P.kary = (o->flags & HARMONIA_QF_LINEAR) ? 0 : 1;
+  P.ilp2 = (o->flags & HARMONIA_QF_ILP1) == 0;
   P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
   // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
   // top levels in BFS order while they fit

@@ -125,6 +125,7 @@ struct Plan {
   uint32_t smem_bytes = 0;   // dynamic smem of the search kernel
   bool gather = false;
   int kary = 1;              // in-node search: 1 = k-ary NTG, 0 = linear NTG (Fig 9)
+  bool ilp2 = true;          // k-ary: two queries per lane group (k_ntg_search2)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
 };
 

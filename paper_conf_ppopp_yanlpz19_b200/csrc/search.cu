@@ -86,6 +86,18 @@ __device__ __forceinline__ uint32_t ld_stream32(const uint32_t* p) {
   return v;
 }
 
+__device__ __forceinline__ uint64_t ld_key_global(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.global.nc.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+// one key (the pivot of a k-ary coarse step): half the L1 wavefront data of a pair load
+template <bool SMEM>
+__device__ __forceinline__ uint64_t ld_key(const uint64_t* p) {
+  if constexpr (SMEM) return *p;
+  else return ld_key_global(p);
+}
+
 template <bool SMEM>
 __device__ __forceinline__ ulonglong2 ld_pair(const uint64_t* p) {
   if constexpr (SMEM) return *reinterpret_cast<const ulonglong2*>(p);
@@ -168,9 +180,9 @@ struct KaryStep {
       const unsigned by = ballot(STRICT ? k.y < q : k.y <= q);
       return base + __popc(bx & gmask) + __popc(by & gmask);
     } else {
-      constexpr int B = S / G;  // coarse step: lane gl holds the last two keys of block gl
-      const ulonglong2 k = ld_pair<SMEM>(nk + (base + gl * B + (B - 2)));
-      const unsigned by = ballot(STRICT ? k.y < q : k.y <= q);
+      constexpr int B = S / G;  // coarse step: lane gl reads the last key of block gl (pivot)
+      const uint64_t kp = ld_key<SMEM>(nk + (base + gl * B + (B - 1)));
+      const unsigned by = ballot(STRICT ? kp < q : kp <= q);
       // blocks whose last key is <= q lie entirely before the rank (the span's last key is
       // > q, so at most G-1 of them)
       return KaryStep<B, G, SMEM, STRICT>::run(nk, base + (uint32_t)__popc(by & gmask) * B, q, gl, gmask);
@@ -275,6 +287,101 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_search(c
   }
 }
 
+// ---- k-ary NTG with two queries per group (ILP 2) ----------------------------------------
+// The search is latency-bound at full occupancy (64 warps/SM): every level is a chain of
+// dependent loads.  Here each G-lane group carries two independent queries and issues the
+// loads of both before comparing, so two chains are in flight per group.  Same arithmetic,
+// same ballots, same results.
+template <int S, int G, bool SMEM>
+struct KaryStep2 {
+  static __device__ __forceinline__ void run(const uint64_t* nka, const uint64_t* nkb, uint32_t& ba, uint32_t& bb,
+                                             uint64_t qa, uint64_t qb, int gl, uint32_t gmask) {
+    if constexpr (S / 2 <= G) {
+      constexpr int L = S / 2;
+      ulonglong2 ka = make_ulonglong2(kPad, kPad), kb = make_ulonglong2(kPad, kPad);
+      if constexpr (L < G) {
+        ld_pair_if<SMEM>(ka, nka + (ba + 2 * gl), gl < L);
+        ld_pair_if<SMEM>(kb, nkb + (bb + 2 * gl), gl < L);
+      } else {
+        ka = ld_pair<SMEM>(nka + (ba + 2 * gl));
+        kb = ld_pair<SMEM>(nkb + (bb + 2 * gl));
+      }
+      ba += __popc(ballot(ka.x <= qa) & gmask) + __popc(ballot(ka.y <= qa) & gmask);
+      bb += __popc(ballot(kb.x <= qb) & gmask) + __popc(ballot(kb.y <= qb) & gmask);
+    } else {
+      constexpr int B = S / G;
+      const uint64_t ka = ld_key<SMEM>(nka + (ba + gl * B + (B - 1)));
+      const uint64_t kb = ld_key<SMEM>(nkb + (bb + gl * B + (B - 1)));
+      ba += (uint32_t)__popc(ballot(ka <= qa) & gmask) * B;
+      bb += (uint32_t)__popc(ballot(kb <= qb) & gmask) * B;
+      KaryStep2<B, G, SMEM>::run(nka, nkb, ba, bb, qa, qb, gl, gmask);
+    }
+  }
+};
+
+template <int F, int G>
+__global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_search2(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  constexpr int QPW = 32 / G;
+  const int lane = threadIdx.x & 31, grp = lane / G, gl = lane % G;
+  const uint32_t gmask = (G == 32) ? kFull : (((1u << G) - 1u) << (grp * G));
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  // a warp takes 2*QPW consecutive queries per iteration: chunk A then chunk B
+  for (uint64_t base = warp * 2 * QPW; base < a.n; base += nwarps * 2 * QPW) {
+    const uint64_t ja = base + grp, jb = base + QPW + grp;
+    const bool acta = ja < a.n, actb = jb < a.n;
+    const uint64_t qa0 = acta ? ld_stream(a.q + ja) : kPad, qb0 = actb ? ld_stream(a.q + jb) : kPad;
+    const bool la = acta && qa0 != kPad, lb = actb && qb0 != kPad;
+    const uint64_t qa = la ? qa0 : 0, qb = lb ? qb0 : 0;  // inactive groups stay inside nodes
+    uint64_t oa = ja, ob = jb;
+    if (a.idx && gl == 0) {
+      if (acta) oa = ld_stream32(a.idx + ja);
+      if (actb) ob = ld_stream32(a.idx + jb);
+    }
+    uint32_t na = 0, nb = 0;
+    for (uint32_t l = 0; l + 1 < a.h; ++l) {
+      const uint32_t fa = ps_smem ? s_ps[na] : __ldg(a.ps + na);
+      const uint32_t fb = ps_smem ? s_ps[nb] : __ldg(a.ps + nb);
+      uint32_t ra = 0, rb = 0;
+      if (l < a.smem_levels)
+        KaryStep2<F, G, true>::run(s_keys + (uint64_t)na * F, s_keys + (uint64_t)nb * F, ra, rb, qa, qb, gl, gmask);
+      else
+        KaryStep2<F, G, false>::run(a.keys + (uint64_t)na * F, a.keys + (uint64_t)nb * F, ra, rb, qa, qb, gl, gmask);
+      na = fa + (la ? ra : 0u);  // Eq 1
+      nb = fb + (lb ? rb : 0u);
+    }
+    const uint64_t* lka = a.keys + (uint64_t)na * F;
+    const uint64_t* lkb = a.keys + (uint64_t)nb * F;
+    uint32_t ra = 0, rb = 0;
+    if (leaf_smem)
+      KaryStep2<F, G, true>::run(s_keys + (uint64_t)na * F, s_keys + (uint64_t)nb * F, ra, rb, qa, qb, gl, gmask);
+    else
+      KaryStep2<F, G, false>::run(lka, lkb, ra, rb, qa, qb, gl, gmask);
+    if (gl == 0) {
+      const uint64_t* lva = a.vals + (uint64_t)(na - a.leaf_start) * F;
+      const uint64_t* lvb = a.vals + (uint64_t)(nb - a.leaf_start) * F;
+      uint64_t ka = 0, va = 0, kb = 0, vb = 0;
+      if (la && ra > 0) {
+        ka = __ldg(lka + (ra - 1));
+        va = __ldg(lva + (ra - 1));
+      }
+      if (lb && rb > 0) {
+        kb = __ldg(lkb + (rb - 1));
+        vb = __ldg(lvb + (rb - 1));
+      }
+      if (acta) a.out[oa] = (la && ra > 0 && ka == qa) ? va : kNotFound;
+      if (actb) a.out[ob] = (lb && rb > 0 && kb == qb) ? vb : kNotFound;
+    }
+  }
+}
+
 // Range scan: descend with lo, then walk leaf slots in key-region order.
 template <int F, int G, int MODE>
 __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(const RangeArgs a) {
@@ -367,11 +474,12 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(co
 
 template <int F, int G>
 harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
-  auto kern = p.kary ? k_ntg_search<F, G, 1> : k_ntg_search<F, G, 0>;
-  static int configured_smem[2] = {-1, -1};  // per instantiation and mode
-  if ((int)p.smem_bytes > configured_smem[p.kary]) {
+  const int mode = p.kary ? (p.ilp2 ? 2 : 1) : 0;
+  auto kern = mode == 2 ? k_ntg_search2<F, G> : (mode == 1 ? k_ntg_search<F, G, 1> : k_ntg_search<F, G, 0>);
+  static int configured_smem[3] = {-1, -1, -1};  // per instantiation and mode
+  if ((int)p.smem_bytes > configured_smem[mode]) {
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem[p.kary] = (int)p.smem_bytes;
+    configured_smem[mode] = (int)p.smem_bytes;
   }
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kQueryBlock, p.smem_bytes));

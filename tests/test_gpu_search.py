@@ -132,7 +132,8 @@ def test_every_fanout_and_group_size(hm, orc, F, G):
     for kw in ({}, {"psa_bits": -1}, {"window": 4096}, {"smem_levels": -1}, {"smem_levels": 2},
                {"flags": hm.QF_GATHER, "window": 8192}, {"psa_bits": 3}, {"flags": hm.QF_LINEAR},
                {"flags": hm.QF_LINEAR, "psa_bits": -1, "smem_levels": 1},
-               {"flags": hm.QF_PSA_GLOBAL}, {"flags": hm.QF_PSA_GLOBAL | hm.QF_LINEAR, "window": 3072}):
+               {"flags": hm.QF_PSA_GLOBAL}, {"flags": hm.QF_PSA_GLOBAL | hm.QF_LINEAR, "window": 3072},
+               {"flags": hm.QF_ILP1}, {"flags": hm.QF_ILP1, "psa_bits": -1, "smem_levels": -1}):
         assert np.array_equal(host(t.search(cu(q), group_size=G, **kw)), exp), kw
 
 
