@@ -304,7 +304,7 @@ def main():
     if a.sweep:
         for spec in a.sweep.split(";"):
             kw = dict(group_size=a.group_size, psa_bits=a.psa_bits, smem_levels=a.smem_levels, window=a.window,
-                      flags=a.flags)
+                      flags=a.flags, lane_queries=0)
             for item in filter(None, spec.split(",")):
                 k, v = item.split("=")
                 kw[k] = int(v)
@@ -421,7 +421,8 @@ def main():
     if dom_kind == "search":
         avg_ms = dom_ms / dom_n
         achieved = bytes_launch / (avg_ms / 1e3) / 1e9
-        roof = {"bound": "hbm", "kernel": "k_ntg_search", "achieved": achieved, "peak": hbm_peak,
+        kname = {1: "k_lane_search_u"}.get(plan["group_size"], "k_ntg_search2")
+        roof = {"bound": "hbm", "kernel": kname, "achieved": achieved, "peak": hbm_peak,
                 "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": None, "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": bytes_launch, "queries_per_launch": nw,
                 "avg_launch_ms": avg_ms, "no_reuse_bytes_per_query": noreuse_bpq,

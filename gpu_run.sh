@@ -1,2 +1,2 @@
-python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1; tail -2 gpurun_out/gpu_tests.log
-python bench.py --steps 10 --sweep "group_size=2;group_size=2,flags=16;group_size=4;group_size=4,flags=16;group_size=8" > gpurun_out/sweep14.jsonl 2>&1; cat gpurun_out/sweep14.jsonl
+python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1; tail -3 gpurun_out/gpu_tests.log
+python bench.py > gpurun_out/bench_r1c.json 2> gpurun_out/bench_r1c.err; cat gpurun_out/bench_r1c.json; tail -2 gpurun_out/bench_r1c.err

@@ -73,7 +73,10 @@ typedef struct {
   int32_t flags;        /* HARMONIA_QF_* bits                                                 */
   uint64_t window;      /* PSA window = queries partitioned together (the paper's "time
                            window"): 0 = auto; otherwise rounded to a multiple of 1024 */
-  uint64_t reserved[2];
+  uint32_t lane_queries; /* group_size = 1 only: independent queries interleaved per lane
+                           (1, 2 or 4; 0 = auto)                                            */
+  uint32_t reserved0;
+  uint64_t reserved1;
 } harmonia_query_opts;
 
 #define HARMONIA_QF_NO_PS_SMEM 1u  /* do not stage the prefix-sum array in shared memory     */

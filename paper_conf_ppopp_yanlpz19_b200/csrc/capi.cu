@@ -11,7 +11,7 @@ namespace hm {
 
 namespace {
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
-constexpr uint64_t kAutoWindow = 1ull << 24;  // auto PSA window (queries): measured best, DESIGN.md §7
+constexpr uint64_t kAutoWindow = 1ull << 23;  // auto PSA window (queries): measured best, DESIGN.md §8
 
 bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 }  // namespace
@@ -27,7 +27,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
     G = auto_group_size(t->F);
     while (2 * G > (int)t->F) G /= 2;
   }
-  if (!pow2(G) || G < 2 || G > 32 || 2 * G > (int)t->F) return HARMONIA_ERR_INVALID_ARG;
+  if (!pow2(G) || G < 1 || G > 32 || 2 * G > (int)t->F) return HARMONIA_ERR_INVALID_ARG;
   P.G = G;
   // ---- PSA bits (Eq 2) over the occupied key span (C-A11)
   int nb = o->psa_bits;
@@ -54,6 +54,9 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.gather = (o->flags & HARMONIA_QF_GATHER) != 0;
   P.kary = (o->flags & HARMONIA_QF_LINEAR) ? 0 : 1;
   P.ilp2 = (o->flags & HARMONIA_QF_ILP1) == 0;
+  if (o->lane_queries != 0 && o->lane_queries != 1 && o->lane_queries != 2 && o->lane_queries != 4)
+    return HARMONIA_ERR_INVALID_ARG;
+  P.lane_ilp = o->lane_queries ? (int)o->lane_queries : 2;
   P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
   // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
   // top levels in BFS order while they fit

@@ -126,6 +126,7 @@ struct Plan {
   bool gather = false;
   int kary = 1;              // in-node search: 1 = k-ary NTG, 0 = linear NTG (Fig 9)
   bool ilp2 = true;          // k-ary: two queries per lane group (k_ntg_search2)
+  int lane_ilp = 2;          // G = 1: queries interleaved per lane (k_lane_search_u)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
 };
 

@@ -382,6 +382,142 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_search2(
   }
 }
 
+// ---- G = 1: the narrowing limit of NTG (one lane per query) ------------------------------
+// With a single lane there is no group to ballot over: the rank r = #keys <= q in the node is
+// found by a branch-free binary search over the F slots (PAD > every live q), log2(F) loads.
+// Every warp instruction then serves 32 queries, which halves the L1 wavefronts per query of
+// the G = 2 group.  Selected with group_size = 1.
+template <int F, bool SMEM>
+__device__ __forceinline__ uint32_t lane_rank(const uint64_t* nk, uint64_t q) {
+  uint32_t r = 0;
+#pragma unroll
+  for (int s = F / 2; s >= 1; s >>= 1)
+    if (ld_key<SMEM>(nk + (r + s - 1)) <= q) r += s;
+  return r;
+}
+
+template <int F>
+__global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < a.n; j += stride) {
+    const uint64_t q0 = ld_stream(a.q + j);
+    const bool live = q0 != kPad;
+    const uint64_t q = live ? q0 : 0;
+    const uint64_t o = a.idx ? (uint64_t)ld_stream32(a.idx + j) : j;
+    uint32_t node = 0;
+    for (uint32_t l = 0; l + 1 < a.h; ++l) {
+      const uint32_t first = ps_smem ? s_ps[node] : __ldg(a.ps + node);  // PS[node_idx]
+      const uint32_t r = l < a.smem_levels ? lane_rank<F, true>(s_keys + (uint64_t)node * F, q)
+                                           : lane_rank<F, false>(a.keys + (uint64_t)node * F, q);
+      node = first + r;  // Eq 1
+    }
+    const uint64_t* lk = a.keys + (uint64_t)node * F;
+    const uint32_t r = leaf_smem ? lane_rank<F, true>(s_keys + (uint64_t)node * F, q) : lane_rank<F, false>(lk, q);
+    uint64_t v = kNotFound;
+    if (live && r > 0) {
+      const uint64_t kk = __ldg(lk + (r - 1));
+      const uint64_t vv = __ldg(a.vals + (uint64_t)(node - a.leaf_start) * F + (r - 1));
+      if (kk == q) v = vv;
+    }
+    a.out[o] = v;
+  }
+}
+
+// G = 1 with U independent queries per lane, interleaved step by step: the single-lane
+// search is latency-bound (few instructions, few wavefronts), so U chains per thread raise
+// the memory-level parallelism without adding work.  A warp takes 32*U consecutive
+// (PSA-ordered) queries: query (u, lane) = base + u*32 + lane.
+template <int F, int U>
+__global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t base = warp * 32 * U; base < a.n; base += nwarps * 32 * U) {
+    uint64_t q[U], o[U];
+    uint32_t node[U];
+    bool act[U], live[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t j = base + u * 32 + lane;
+      act[u] = j < a.n;
+      const uint64_t q0 = act[u] ? ld_stream(a.q + j) : kPad;
+      live[u] = q0 != kPad;
+      q[u] = live[u] ? q0 : 0;
+      o[u] = (act[u] && a.idx) ? (uint64_t)ld_stream32(a.idx + j) : j;
+      node[u] = 0;
+    }
+    for (uint32_t l = 0; l + 1 < a.h; ++l) {
+      uint32_t first[U], r[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        first[u] = ps_smem ? s_ps[node[u]] : __ldg(a.ps + node[u]);  // PS[node_idx]
+        r[u] = 0;
+      }
+      if (l < a.smem_levels) {
+#pragma unroll
+        for (int s = F / 2; s >= 1; s >>= 1) {
+          uint64_t k[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) k[u] = s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)];
+#pragma unroll
+          for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+        }
+      } else {
+#pragma unroll
+        for (int s = F / 2; s >= 1; s >>= 1) {
+          uint64_t k[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+#pragma unroll
+          for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) node[u] = first[u] + r[u];  // Eq 1
+    }
+    uint32_t r[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) r[u] = 0;
+#pragma unroll
+    for (int s = F / 2; s >= 1; s >>= 1) {
+      uint64_t k[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        k[u] = leaf_smem ? s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)]
+                         : ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+#pragma unroll
+      for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+    }
+    uint64_t kk[U], vv[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      kk[u] = 0;
+      vv[u] = kNotFound;
+      if (live[u] && r[u] > 0) {
+        kk[u] = __ldg(a.keys + (uint64_t)node[u] * F + (r[u] - 1));
+        vv[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (act[u]) a.out[o[u]] = (live[u] && r[u] > 0 && kk[u] == q[u]) ? vv[u] : kNotFound;
+  }
+}
+
 // Range scan: descend with lo, then walk leaf slots in key-region order.
 template <int F, int G, int MODE>
 __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(const RangeArgs a) {
@@ -470,6 +606,30 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(co
     }
     if (active && gl == 0) a.counts[slab] = (uint32_t)(cnt > 0xFFFFFFFFull ? 0xFFFFFFFFull : cnt);
   }
+}
+
+template <int F>
+harmonia_status launch_lane_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  const int U = p.lane_ilp;
+  auto kern = U >= 4 ? k_lane_search_u<F, 4> : (U == 2 ? k_lane_search_u<F, 2> : k_lane_search<F>);
+  const int bs = U >= 2 ? 1024 : kQueryBlock;
+  static int configured_smem[5] = {-1, -1, -1, -1, -1};
+  const int ci = U >= 4 ? 4 : U;
+  if ((int)p.smem_bytes > configured_smem[ci]) {
+    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
+    configured_smem[ci] = (int)p.smem_bytes;
+  }
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, bs, p.smem_bytes));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t need = ceil_div(a.n, (uint64_t)bs * (U >= 4 ? 4 : U));
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
+  {
+    ProfScope ps_(HARMONIA_PROF_SEARCH, st);
+    kern<<<grid, bs, p.smem_bytes, st>>>(a);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
 }
 
 template <int F, int G>
@@ -566,20 +726,35 @@ harmonia_status launch_range_fg(const harmonia_tree* t, const Plan& p, const Ran
 
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
   if (a.n == 0) return HARMONIA_OK;
+  if (p.G == 1) {
+    switch (t->F) {
+      case 4: return launch_lane_search<4>(t, p, a, st);
+      case 8: return launch_lane_search<8>(t, p, a, st);
+      case 16: return launch_lane_search<16>(t, p, a, st);
+      case 32: return launch_lane_search<32>(t, p, a, st);
+      case 64: return launch_lane_search<64>(t, p, a, st);
+      case 128: return launch_lane_search<128>(t, p, a, st);
+      case 256: return launch_lane_search<256>(t, p, a, st);
+    }
+    return HARMONIA_ERR_INVALID_ARG;
+  }
   HM_DISPATCH(launch_search_fg, t->F, p.G, t, p, a, st)
 }
 
 harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
   if (a.n == 0) return HARMONIA_OK;
-  HM_DISPATCH(launch_range_fg, t->F, p.G, t, p, a, st)
+  const int G = p.G == 1 ? 2 : p.G;  // ranges scan leaves with at least a lane pair
+  HM_DISPATCH(launch_range_fg, t->F, G, t, p, a, st)
 }
 
 // Measured default G per fanout (refreshed from bench sweeps).
 int auto_group_size(uint32_t F) {
-  // k-ary NTG: G = 2 was fastest at F = 64 (bench sweeps); the same narrow
-  // group keeps 16 queries per warp for the other fanouts (F >= 4 always admits G = 2).
+  // The paper's NTG procedure narrows the group while throughput improves.  On
+  // B200 the measured sweep keeps improving down to one lane per query: G = 1 (lane-local
+  // binary rank, 2 queries per lane) beats the best ballot group G = 2 (20.8 vs 18.4 G q/s
+  // at c2), G = 2 beats 4..32.  Every F admits G = 1.
   (void)F;
-  return 2;
+  return 1;
 }
 
 }  // namespace hm

@@ -119,7 +119,21 @@ def test_key_distributions(hm, orc, keyset):
     assert np.array_equal(host(t.search(cu(q))), orc.sorted_search(keys, vals, q))
 
 
-FG = [(F, G) for F in (4, 8, 16, 32, 64, 128, 256) for G in (2, 4, 8, 16, 32) if 2 * G <= F]
+FG = [(F, G) for F in (4, 8, 16, 32, 64, 128, 256) for G in (1, 2, 4, 8, 16, 32) if 2 * G <= F]
+
+
+@pytest.mark.parametrize("F", [4, 8, 16, 64, 256])
+@pytest.mark.parametrize("lane_queries", [1, 2, 4])
+def test_lane_search_queries_per_lane(hm, orc, F, lane_queries):
+    """G = 1 (one lane per query) with 1, 2, 4 interleaved queries per lane, ragged tails."""
+    keys = gen.random_keys(30000, seed=F + lane_queries)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F)
+    q = np.concatenate([gen.uniform_queries(keys, 50003, miss_frac=0.4), gen.edge_queries(keys)])
+    exp = orc.sorted_search(keys, vals, q)
+    for kw in ({}, {"psa_bits": -1}, {"window": 3072}, {"smem_levels": -1}):
+        got = host(t.search(cu(q), group_size=1, lane_queries=lane_queries, **kw))
+        assert np.array_equal(got, exp), kw
 
 
 @pytest.mark.parametrize("F,G", FG)
