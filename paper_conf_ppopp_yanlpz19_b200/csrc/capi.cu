@@ -57,6 +57,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   if (o->lane_queries != 0 && o->lane_queries != 1 && o->lane_queries != 2 && o->lane_queries != 4)
     return HARMONIA_ERR_INVALID_ARG;
   P.lane_ilp = o->lane_queries ? (int)o->lane_queries : 2;
+  P.psa_level2 = (o->flags & HARMONIA_QF_PSA_COARSE) ? 2 : ((o->flags & HARMONIA_QF_PSA_LSD) ? 1 : 0);
   P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
   // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
   // top levels in BFS order while they fit
@@ -113,7 +114,7 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
   for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
     harmonia_status s = p.psa_global ? psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
-                                     : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st);
+                                     : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.psa_level2);
     if (s != HARMONIA_OK) return s;
     a.q = w.sorted_q;
     a.n = nw;
@@ -318,7 +319,7 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
     s = p.psa_global ? psa_partition(d_lo + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
-                     : psa_partition2(d_lo + w0, nw, p.bucket, p.nb, w, t->sm_count, st);
+                     : psa_partition2(d_lo + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.psa_level2);
     if (s != HARMONIA_OK) return s;
     a.lo = w.sorted_q;
     a.hi = d_hi + w0;

@@ -127,6 +127,7 @@ struct Plan {
   int kary = 1;              // in-node search: 1 = k-ary NTG, 0 = linear NTG (Fig 9)
   bool ilp2 = true;          // k-ary: two queries per lane group (k_ntg_search2)
   int lane_ilp = 2;          // G = 1: queries interleaved per lane (k_lane_search_u)
+  int psa_level2 = 0;        // chunk sort: 0 counting, 1 ballot LSD, 2 none (coarse only)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
 };
 
@@ -168,7 +169,7 @@ struct SearchArgs {
   uint64_t* out;           // results: out[idx ? idx[j] : j]
 };
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
-                               int sm_count, cudaStream_t st, bool ballot_sort = false);
+                               int sm_count, cudaStream_t st, int level2 = 0);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
                               cudaStream_t st);
 

@@ -90,14 +90,26 @@ __global__ void __launch_bounds__(kBlock) k_psa2_hist(const uint64_t* __restrict
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (int i = threadIdx.x; i < kWarps * kCoarseBins; i += kBlock) (&wh[0][0])[i] = 0;
   __syncthreads();
-  const uint64_t stride = (uint64_t)gridDim.x * kBlock;
-  const uint64_t n_round = round_up_dev(n);
-  for (uint64_t i = blockIdx.x * (uint64_t)kBlock + threadIdx.x; i < n_round; i += stride) {
-    const bool valid = i < n;
-    const uint32_t d = valid ? f(__ldg(q + i)) >> shift1 : 0u;
-    const unsigned peers = peers_of<kCoarseBits>(d, __ballot_sync(kFull, valid));
-    if (valid && lane == (unsigned)(__ffs(peers) - 1)) wh[warp][d] += __popc(peers);
-    __syncwarp();
+  // tiles of kBatches x 32 queries per warp, all loads issued before the multisplit so that
+  // each thread keeps kBatches loads in flight
+  const uint64_t per_warp_tile = 32 * kBatches;
+  const uint64_t gw = (blockIdx.x * (uint64_t)kBlock + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * kBlock) >> 5;
+  for (uint64_t t0 = gw * per_warp_tile; t0 < n; t0 += nw * per_warp_tile) {
+    uint64_t v[kBatches];
+#pragma unroll
+    for (int k = 0; k < kBatches; ++k) {
+      const uint64_t i = t0 + k * 32 + lane;
+      v[k] = i < n ? __ldg(q + i) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < kBatches; ++k) {
+      const bool valid = t0 + k * 32 + lane < n;
+      const uint32_t d = valid ? f(v[k]) >> shift1 : 0u;
+      const unsigned peers = peers_of<kCoarseBits>(d, __ballot_sync(kFull, valid));
+      if (valid && lane == (unsigned)(__ffs(peers) - 1)) wh[warp][d] += __popc(peers);
+      __syncwarp();
+    }
   }
   __syncthreads();
   uint32_t c = 0;
@@ -124,10 +136,14 @@ __global__ void __launch_bounds__(kBlock) k_psa2_scatter(const uint64_t* __restr
     uint64_t v[kBatches];
     uint32_t d[kBatches], pos[kBatches];
 #pragma unroll
+    for (int k = 0; k < kBatches; ++k) {  // all loads first (kBatches in flight per thread)
+      const uint64_t e = t0 + warp * (32 * kBatches) + k * 32 + lane;
+      v[k] = e < n ? __ldg(q + e) : 0;
+    }
+#pragma unroll
     for (int k = 0; k < kBatches; ++k) {
       const uint64_t e = t0 + warp * (32 * kBatches) + k * 32 + lane;
       const bool valid = e < n;
-      v[k] = valid ? __ldg(q + e) : 0;
       d[k] = valid ? f(v[k]) >> shift1 : 0u;
       const unsigned peers = peers_of<kCoarseBits>(d[k], __ballot_sync(kFull, valid));
       const uint32_t run = valid ? wcnt[warp][d[k]] : 0u;
@@ -293,7 +309,7 @@ constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12;
 }  // namespace
 
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
-                               cudaStream_t st, bool ballot_sort) {
+                               cudaStream_t st, int level2) {
   const uint32_t b1 = (uint32_t)std::min(nb, kCoarseBits);
   const uint32_t shift1 = (uint32_t)nb - b1;
   HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * kCoarseBins * 4, st));
@@ -310,6 +326,7 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
                                                      ws.sorted_q, ws.idx);
   }
   HM_LAUNCHED();
+  if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation)
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);  // reported in the "scan" class: level-2 sort
     static bool configured = false;
@@ -320,7 +337,7 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
       configured = true;
     }
     const int g = (int)std::min<uint64_t>(ceil_div(n, kChunk), (uint64_t)sm * 4);
-    if (ballot_sort)  // two stable LSD passes of ballot multisplit (ablation)
+    if (level2 == 1)  // two stable LSD passes of ballot multisplit (ablation)
       k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
     else              // one counting pass with shared-memory atomics (default, measured faster)
       k_psa2_count_sort<<<std::max(g, 1), kSortThreads, kCountSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
