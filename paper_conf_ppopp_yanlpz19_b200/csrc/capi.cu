@@ -365,6 +365,8 @@ extern "C" harmonia_status harmonia_route_partition(const uint64_t* d_split, uin
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
   BucketSplit f{d_split, P - 1};
+  if (P <= 256)  // SMEM-aggregated two-level router (one atomic per tile and shard)
+    return route_partition2(d_q, n, f, P, w.counts, d_routed, d_pos, sm, (cudaStream_t)stream, h_counts);
   return psa_partition(d_q, n, f, P, w, sm, (cudaStream_t)stream, h_counts);
 }
 

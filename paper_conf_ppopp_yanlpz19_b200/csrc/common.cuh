@@ -170,6 +170,8 @@ struct SearchArgs {
 };
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
                                int sm_count, cudaStream_t st, int level2 = 0);
+harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, uint32_t* counts,
+                                 uint64_t* routed, uint32_t* pos, int sm, cudaStream_t st, uint64_t* h_counts);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
                               cudaStream_t st);
 

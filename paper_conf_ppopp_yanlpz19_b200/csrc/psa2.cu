@@ -83,9 +83,19 @@ __device__ __forceinline__ uint32_t block_scan(uint32_t v, uint32_t* tmp, uint32
   return r;
 }
 
+// coarse digit of the PSA bucket (top kCoarseBits of the Nb-bit bucket)
+struct CoarseDigit {
+  BucketBits f;
+  uint32_t shift;
+  __device__ __forceinline__ uint32_t operator()(uint64_t q) const { return f(q) >> shift; }
+};
+
 // ---- level 1: histogram of the coarse digit ------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_psa2_hist(const uint64_t* __restrict__ q, uint64_t n, BucketBits f,
-                                                      uint32_t shift1, uint32_t* __restrict__ counts) {
+// Digit: any functor mapping a query to [0, kCoarseBins) (PSA coarse digit, or the
+// destination shard of the partitioned multi-GPU mode).
+template <class Digit>
+__global__ void __launch_bounds__(kBlock) k_psa2_hist(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
+                                                      uint32_t* __restrict__ counts) {
   __shared__ uint32_t wh[kWarps][kCoarseBins];
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (int i = threadIdx.x; i < kWarps * kCoarseBins; i += kBlock) (&wh[0][0])[i] = 0;
@@ -105,7 +115,7 @@ __global__ void __launch_bounds__(kBlock) k_psa2_hist(const uint64_t* __restrict
 #pragma unroll
     for (int k = 0; k < kBatches; ++k) {
       const bool valid = t0 + k * 32 + lane < n;
-      const uint32_t d = valid ? f(v[k]) >> shift1 : 0u;
+      const uint32_t d = valid ? dg(v[k]) : 0u;
       const unsigned peers = peers_of<kCoarseBits>(d, __ballot_sync(kFull, valid));
       if (valid && lane == (unsigned)(__ffs(peers) - 1)) wh[warp][d] += __popc(peers);
       __syncwarp();
@@ -119,8 +129,9 @@ __global__ void __launch_bounds__(kBlock) k_psa2_hist(const uint64_t* __restrict
 }
 
 // ---- level 1: coarse scatter ------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_psa2_scatter(const uint64_t* __restrict__ q, uint64_t n, BucketBits f,
-                                                         uint32_t shift1, const uint32_t* __restrict__ counts,
+template <class Digit>
+__global__ void __launch_bounds__(kBlock) k_psa2_scatter(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
+                                                         const uint32_t* __restrict__ counts,
                                                          uint32_t* __restrict__ cursor, uint64_t* __restrict__ sorted_q,
                                                          uint32_t* __restrict__ idx) {
   __shared__ uint32_t wcnt[kWarps][kCoarseBins];
@@ -144,7 +155,7 @@ __global__ void __launch_bounds__(kBlock) k_psa2_scatter(const uint64_t* __restr
     for (int k = 0; k < kBatches; ++k) {
       const uint64_t e = t0 + warp * (32 * kBatches) + k * 32 + lane;
       const bool valid = e < n;
-      d[k] = valid ? f(v[k]) >> shift1 : 0u;
+      d[k] = valid ? dg(v[k]) : 0u;
       const unsigned peers = peers_of<kCoarseBits>(d[k], __ballot_sync(kFull, valid));
       const uint32_t run = valid ? wcnt[warp][d[k]] : 0u;
       __syncwarp();
@@ -306,26 +317,49 @@ constexpr int kLocalBins = 1 << kLocalBits;
 constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12;
 #include "psa2_count_sort.inc"
 
+// level-1 partition by any <= 256-bin digit: histogram, then the staged scatter.
+// h_counts (optional) receives the first `nbins` bin counts synchronously.
+template <class Digit>
+harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg, uint32_t* counts,
+                                 uint64_t* sorted_q, uint32_t* idx, int sm, cudaStream_t st, uint64_t* h_counts,
+                                 uint32_t nbins) {
+  HM_CUDA(cudaMemsetAsync(counts, 0, 2 * kCoarseBins * 4, st));
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
+    const int g = (int)std::min<uint64_t>(ceil_div(n, kBlock * 8), (uint64_t)sm * 8);
+    k_psa2_hist<Digit><<<std::max(g, 1), kBlock, 0, st>>>(q, n, dg, counts);
+  }
+  HM_LAUNCHED();
+  if (h_counts) {
+    uint32_t tmp[kCoarseBins];
+    HM_CUDA(cudaMemcpyAsync(tmp, counts, nbins * 4, cudaMemcpyDeviceToHost, st));
+    HM_CUDA(cudaStreamSynchronize(st));
+    for (uint32_t b = 0; b < nbins; ++b) h_counts[b] = tmp[b];
+  }
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
+    const int g = (int)std::min<uint64_t>(ceil_div(n, kCoarseTile), (uint64_t)sm * 4);
+    k_psa2_scatter<Digit><<<std::max(g, 1), kBlock, 0, st>>>(q, n, dg, counts, counts + kCoarseBins, sorted_q, idx);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
 }  // namespace
+
+// multi-GPU router: destination-major grouping by splitters (P <= 256 shards)
+harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, uint32_t* counts,
+                                 uint64_t* routed, uint32_t* pos, int sm, cudaStream_t st, uint64_t* h_counts) {
+  if (P > (uint32_t)kCoarseBins) return HARMONIA_ERR_INVALID_ARG;
+  return coarse_partition(q, n, f, counts, routed, pos, sm, st, h_counts, P);
+}
 
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
                                cudaStream_t st, int level2) {
   const uint32_t b1 = (uint32_t)std::min(nb, kCoarseBits);
   const uint32_t shift1 = (uint32_t)nb - b1;
-  HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * kCoarseBins * 4, st));
-  {
-    ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kBlock * 8), (uint64_t)sm * 8);
-    k_psa2_hist<<<std::max(g, 1), kBlock, 0, st>>>(q, n, f, shift1, ws.counts);
-  }
-  HM_LAUNCHED();
-  {
-    ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kCoarseTile), (uint64_t)sm * 4);
-    k_psa2_scatter<<<std::max(g, 1), kBlock, 0, st>>>(q, n, f, shift1, ws.counts, ws.counts + kCoarseBins,
-                                                     ws.sorted_q, ws.idx);
-  }
-  HM_LAUNCHED();
+  harmonia_status s = coarse_partition(q, n, CoarseDigit{f, shift1}, ws.counts, ws.sorted_q, ws.idx, sm, st, nullptr, 0);
+  if (s != HARMONIA_OK) return s;
   if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation)
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);  // reported in the "scan" class: level-2 sort
