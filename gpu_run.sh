@@ -1,1 +1,2 @@
-timeout 300 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29521 bench.py --gpus 1 --steps 10 --warmup 3 --mode partitioned --no-cpu > gpurun_out/bench_part3.log 2>&1; echo "rc=$?"; tail -30 gpurun_out/bench_part3.log | cut -c1-400
+python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1; tail -2 gpurun_out/gpu_tests.log
+python bench.py --steps 10 --sweep "group_size=1" 2>&1 | grep sweep

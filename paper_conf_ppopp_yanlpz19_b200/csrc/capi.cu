@@ -58,6 +58,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
     return HARMONIA_ERR_INVALID_ARG;
   P.lane_ilp = o->lane_queries ? (int)o->lane_queries : 2;
   P.psa_level2 = (o->flags & HARMONIA_QF_PSA_COARSE) ? 2 : ((o->flags & HARMONIA_QF_PSA_LSD) ? 1 : 0);
+  P.fuse = (o->flags & HARMONIA_QF_FUSE_SORT) != 0;  // measured slower
   P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
   // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
   // top levels in BFS order while they fit
@@ -113,11 +114,21 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
   const PsaWs w = psa_ws_carve(p, ws);
   for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
+    const bool fused = p.fuse && p.G == 1 && !p.psa_global && p.psa_level2 == 0 && !p.gather &&
+                       p.smem_bytes + (8u << 10) + (48u << 10) <= t->smem_optin;
     harmonia_status s = p.psa_global ? psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
-                                     : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.psa_level2);
+                                     : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st,
+                                                      fused ? 2 : p.psa_level2);
     if (s != HARMONIA_OK) return s;
     a.q = w.sorted_q;
     a.n = nw;
+    if (fused) {  // level-2 chunk sort inside the search kernel
+      a.idx = w.idx;
+      a.out = out + w0;
+      a.bucket = p.bucket;
+      if ((s = launch_sort_search(t, p, a, st)) != HARMONIA_OK) return s;
+      continue;
+    }
     if (p.gather) {
       a.idx = nullptr;
       a.out = w.sorted_out;

@@ -128,6 +128,7 @@ struct Plan {
   bool ilp2 = true;          // k-ary: two queries per lane group (k_ntg_search2)
   int lane_ilp = 2;          // G = 1: queries interleaved per lane (k_lane_search_u)
   int psa_level2 = 0;        // chunk sort: 0 counting, 1 ballot LSD, 2 none (coarse only)
+  bool fuse = false;         // G = 1 + counting chunk sort fused into the search (k_sort_search)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
 };
 
@@ -167,7 +168,10 @@ struct SearchArgs {
   const uint32_t* idx;     // original position within the window (nullptr = identity)
   uint64_t n;
   uint64_t* out;           // results: out[idx ? idx[j] : j]
+  BucketBits bucket;       // PSA bucket (fused level-2 sort only)
 };
+harmonia_status launch_sort_search(const harmonia_tree* t, const struct Plan& p, const SearchArgs& a,
+                                   cudaStream_t st);
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
                                int sm_count, cudaStream_t st, int level2 = 0);
 harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, uint32_t* counts,

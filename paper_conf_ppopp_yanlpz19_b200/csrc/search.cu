@@ -88,7 +88,15 @@ __device__ __forceinline__ uint32_t ld_stream32(const uint32_t* p) {
 
 __device__ __forceinline__ uint64_t ld_key_global(const uint64_t* p) {
   uint64_t v;
+#ifdef HM_KEYS_EVICT_LAST
+  asm volatile(
+      "{ .reg .b64 pol; createpolicy.fractional.L2::evict_last.b64 pol, 1.0; "
+      "ld.global.nc.L2::cache_hint.u64 %0, [%1], pol; }"
+      : "=l"(v)
+      : "l"(p));
+#else
   asm volatile("ld.global.nc.u64 %0, [%1];" : "=l"(v) : "l"(p));
+#endif
   return v;
 }
 // one key (the pivot of a k-ary coarse step): half the L1 wavefront data of a pair load
@@ -434,30 +442,19 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
 // search is latency-bound (few instructions, few wavefronts), so U chains per thread raise
 // the memory-level parallelism without adding work.  A warp takes 32*U consecutive
 // (PSA-ordered) queries: query (u, lane) = base + u*32 + lane.
+// one lane, U interleaved queries: descent (Eq 1) + leaf probe + result write
 template <int F, int U>
-__global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const SearchArgs a) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ __align__(8) uint64_t bar;
-  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
-  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
-  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
-  const bool ps_smem = a.ps_smem_bytes != 0;
-  const bool leaf_smem = a.h - 1 < a.smem_levels;
-  const unsigned lane = threadIdx.x & 31;
-  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t base = warp * 32 * U; base < a.n; base += nwarps * 32 * U) {
-    uint64_t q[U], o[U];
+__device__ __forceinline__ void lane_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
+                                          bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
+                                          const uint64_t (&o)[U], const bool (&act)[U]) {
+  {
+    uint64_t q[U];
     uint32_t node[U];
-    bool act[U], live[U];
+    bool live[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      const uint64_t j = base + u * 32 + lane;
-      act[u] = j < a.n;
-      const uint64_t q0 = act[u] ? ld_stream(a.q + j) : kPad;
-      live[u] = q0 != kPad;
-      q[u] = live[u] ? q0 : 0;
-      o[u] = (act[u] && a.idx) ? (uint64_t)ld_stream32(a.idx + j) : j;
+      live[u] = act[u] && q0[u] != kPad;  // PAD is never a key (C-A2)
+      q[u] = live[u] ? q0[u] : 0;
       node[u] = 0;
     }
     for (uint32_t l = 0; l + 1 < a.h; ++l) {
@@ -515,6 +512,153 @@ __global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const 
 #pragma unroll
     for (int u = 0; u < U; ++u)
       if (act[u]) a.out[o[u]] = (live[u] && r[u] > 0 && kk[u] == q[u]) ? vv[u] : kNotFound;
+  }
+}
+
+template <int F, int U>
+__global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t base = warp * 32 * U; base < a.n; base += nwarps * 32 * U) {
+    uint64_t q0[U], o[U];
+    bool act[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t j = base + u * 32 + lane;
+      act[u] = j < a.n;
+      q0[u] = act[u] ? ld_stream(a.q + j) : kPad;
+      o[u] = (act[u] && a.idx) ? (uint64_t)ld_stream32(a.idx + j) : j;
+    }
+    lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, o, act);
+  }
+}
+
+// ---- level-2 PSA fused with the G = 1 search (default search path) -----------------------
+// Each CTA takes chunks of kFuseChunk queries of the level-1 (coarse) PSA order, sorts the
+// chunk by its full Nb-bit bucket with a shared-memory counting sort (the same arithmetic as
+// k_psa2_count_sort) and searches the sorted chunk straight from shared memory: the chunk
+// never goes back to L2/HBM between the sort and the search.
+constexpr int kFuseThreads = 1024, kFusePer = 4, kFuseChunk = kFuseThreads * kFusePer;  // 4096
+constexpr int kFuseBins = 2048;
+constexpr uint32_t kFuseSmem = kFuseBins * 4 + kFuseChunk * 12;  // + the staged tree top
+
+template <int F>
+__global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ uint32_t tmp[kFuseThreads / 32 + 1], s_mm[2][kFuseThreads / 32];
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const uint32_t top = a.ps_smem_bytes + a.smem_nodes * F * 8;  // multiple of 16
+  uint64_t* sq = reinterpret_cast<uint64_t*>(smem + top);
+  uint32_t* si = reinterpret_cast<uint32_t*>(smem + top + kFuseChunk * 8);
+  uint32_t* hist = reinterpret_cast<uint32_t*>(smem + top + kFuseChunk * 12);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint64_t c0 = (uint64_t)blockIdx.x * kFuseChunk; c0 < a.n; c0 += (uint64_t)gridDim.x * kFuseChunk) {
+    const uint32_t m = (uint32_t)((a.n - c0) < (uint64_t)kFuseChunk ? (a.n - c0) : (uint64_t)kFuseChunk);
+    // ---- load and bucket (sort by the most significant Nb bits)
+    uint64_t v[kFusePer];
+    uint32_t ix[kFusePer], b[kFusePer], rk[kFusePer];
+    uint32_t bmin = 0xFFFFFFFFu, bmax = 0;
+#pragma unroll
+    for (int k = 0; k < kFusePer; ++k) {
+      const uint32_t e = k * kFuseThreads + threadIdx.x;
+      v[k] = 0;
+      ix[k] = 0;
+      b[k] = 0;
+      if (e < m) {
+        v[k] = ld_stream(a.q + c0 + e);
+        ix[k] = ld_stream32(a.idx + c0 + e);
+        b[k] = a.bucket(v[k]);
+        bmin = min(bmin, b[k]);
+        bmax = max(bmax, b[k]);
+      }
+    }
+    bmin = __reduce_min_sync(kFull, bmin);
+    bmax = __reduce_max_sync(kFull, bmax);
+    if (lane == 0) {
+      s_mm[0][warp] = bmin;
+      s_mm[1][warp] = bmax;
+    }
+    for (uint32_t i = threadIdx.x; i < kFuseBins; i += kFuseThreads) hist[i] = 0;
+    __syncthreads();
+#pragma unroll 4
+    for (int w = 0; w < kFuseThreads / 32; ++w) {
+      bmin = min(bmin, s_mm[0][w]);
+      bmax = max(bmax, s_mm[1][w]);
+    }
+    uint32_t sh = 0;
+    while (((bmax - bmin) >> sh) >= (uint32_t)kFuseBins) ++sh;
+#pragma unroll
+    for (int k = 0; k < kFusePer; ++k) {
+      const uint32_t e = k * kFuseThreads + threadIdx.x;
+      if (e < m) {
+        b[k] = (b[k] - bmin) >> sh;
+        rk[k] = atomicAdd(&hist[b[k]], 1u);
+      }
+    }
+    __syncthreads();
+    // ---- exclusive scan of the 2048 counters (2 per thread)
+    const uint32_t h0 = hist[2 * threadIdx.x], h1 = hist[2 * threadIdx.x + 1];
+    uint32_t inc = h0 + h1;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFull, inc, d);
+      if (lane >= (unsigned)d) inc += y;
+    }
+    if (lane == 31) tmp[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+      const uint32_t w = tmp[lane];
+      uint32_t wi = w;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, wi, d);
+        if (lane >= (unsigned)d) wi += y;
+      }
+      tmp[lane] = wi - w;
+    }
+    __syncthreads();
+    const uint32_t ex = tmp[warp] + inc - (h0 + h1);
+    hist[2 * threadIdx.x] = ex;
+    hist[2 * threadIdx.x + 1] = ex + h0;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < kFusePer; ++k) {
+      const uint32_t e = k * kFuseThreads + threadIdx.x;
+      if (e < m) {
+        const uint32_t dst = hist[b[k]] + rk[k];
+        sq[dst] = v[k];
+        si[dst] = ix[k];
+      }
+    }
+    __syncthreads();
+    // ---- search the sorted chunk: warp w takes positions [w*128, w*128+128), 2 per lane per round
+#pragma unroll
+    for (int rd = 0; rd < kFusePer / 2; ++rd) {
+      uint64_t q0[2], o[2];
+      bool act[2];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const uint32_t p = warp * (32 * kFusePer) + (rd * 2 + u) * 32 + lane;
+        act[u] = p < m;
+        q0[u] = act[u] ? sq[p] : kPad;
+        o[u] = act[u] ? si[p] : 0;
+      }
+      lane_core<F, 2>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, o, act);
+    }
+    __syncthreads();  // the chunk buffers are reused
   }
 }
 
@@ -606,6 +750,28 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(co
     }
     if (active && gl == 0) a.counts[slab] = (uint32_t)(cnt > 0xFFFFFFFFull ? 0xFFFFFFFFull : cnt);
   }
+}
+
+template <int F>
+harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  auto kern = k_sort_search<F>;
+  const uint32_t smem = p.smem_bytes + kFuseSmem;
+  static int configured_smem = -1;
+  if ((int)smem > configured_smem) {
+    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    configured_smem = (int)smem;
+  }
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFuseThreads, smem));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t need = ceil_div(a.n, kFuseChunk);
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
+  {
+    ProfScope ps_(HARMONIA_PROF_SEARCH, st);
+    kern<<<grid, kFuseThreads, smem, st>>>(a);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
 }
 
 template <int F>
@@ -745,6 +911,20 @@ harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeA
   if (a.n == 0) return HARMONIA_OK;
   const int G = p.G == 1 ? 2 : p.G;  // ranges scan leaves with at least a lane pair
   HM_DISPATCH(launch_range_fg, t->F, G, t, p, a, st)
+}
+
+harmonia_status launch_sort_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  if (a.n == 0) return HARMONIA_OK;
+  switch (t->F) {
+    case 4: return launch_sort_search_f<4>(t, p, a, st);
+    case 8: return launch_sort_search_f<8>(t, p, a, st);
+    case 16: return launch_sort_search_f<16>(t, p, a, st);
+    case 32: return launch_sort_search_f<32>(t, p, a, st);
+    case 64: return launch_sort_search_f<64>(t, p, a, st);
+    case 128: return launch_sort_search_f<128>(t, p, a, st);
+    case 256: return launch_sort_search_f<256>(t, p, a, st);
+  }
+  return HARMONIA_ERR_INVALID_ARG;
 }
 
 // Measured default G per fanout (refreshed from bench sweeps).
