@@ -25,7 +25,10 @@ constexpr int kCoarseBits = 8, kCoarseBins = 1 << kCoarseBits;
 constexpr int kWarps = kBlock / 32;                      // 8 warps per 256-thread CTA
 constexpr int kBatches = 8;                              // 32-query batches per warp per tile
 constexpr int kCoarseTile = kBlock * kBatches;           // 2048 queries per scatter tile
-constexpr int kSortThreads = 512, kSortWarps = kSortThreads / 32;
+#ifndef HM_SORT_THREADS
+#define HM_SORT_THREADS 512
+#endif
+constexpr int kSortThreads = HM_SORT_THREADS, kSortWarps = kSortThreads / 32;
 constexpr int kChunk = kSortThreads * kBatches;          // 4096 queries per local-sort chunk
 constexpr int kLocalBits = 11, kLoBits = 6, kHiBits = kLocalBits - kLoBits;
 constexpr size_t kSortSmem = (size_t)kChunk * (8 + 4 + 2);  // keys, positions, local digits
