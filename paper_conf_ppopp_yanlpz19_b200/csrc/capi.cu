@@ -29,6 +29,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   }
   if (!pow2(G) || G < 1 || G > 32 || 2 * G > (int)t->F) return HARMONIA_ERR_INVALID_ARG;
   P.G = G;
+  P.g_auto = o->group_size == 0;
   // ---- PSA bits (Eq 2) over the occupied key span (C-A11)
   int nb = o->psa_bits;
   if (nb == 0) nb = psa_bits_for(t->n_keys);
@@ -316,6 +317,12 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   a.smem_nodes = p.smem_nodes;
   a.ps_smem_bytes = p.ps_smem ? p.ps_smem_bytes : 0;
   a.cap = cap;
+  if (p.g_auto) {  // the leaf scan wants wide groups for long ranges (measured)
+    int G = 8;
+    while (G < 32 && (uint32_t)(4 * G) < cap) G *= 2;
+    while (2 * G > (int)t->F) G /= 2;
+    p.G = G;
+  }
   if (!p.psa) {
     a.lo = d_lo;
     a.hi = d_hi;

@@ -113,6 +113,7 @@ namespace hm {
 // ---- query plan (host) ----------------------------------------------------------------
 struct Plan {
   int G = 4;
+  bool g_auto = true;        // group size chosen by the library (search: G=1; range: by cap)
   bool psa = false;
   int nb = 0;                // PSA bits
   uint64_t window = 0;       // queries per PSA window

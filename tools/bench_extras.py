@@ -44,7 +44,7 @@ def update_bench(T=1 << 23, batch=1 << 22, reps=3):
     return res
 
 
-def range_bench(T=1 << 23, F=64, reps=5):
+def range_bench(T=1 << 23, F=64, reps=5, groups=(0,), flags=0):
     keys = gen.uniform_keys(T)
     vals = gen.values_for(keys)
     t = hm.Tree(torch.from_numpy(keys).cuda(), torch.from_numpy(vals).cuda(), fanout=F)
@@ -52,13 +52,14 @@ def range_bench(T=1 << 23, F=64, reps=5):
     for length, Qr in ((16, 1 << 22), (64, 1 << 21), (256, 1 << 20), (1024, 1 << 18)):
         lo, hi = gen.ranges(keys, Qr, length)
         lo, hi = torch.from_numpy(lo).cuda(), torch.from_numpy(hi).cuda()
-        ko = torch.empty((Qr, length), dtype=torch.uint64, device="cuda")
-        ms = timed(lambda: t.range(lo, hi, length), reps)
-        res.append({"what": "range_batch", "T": T, "F": F, "len": length, "Qr": Qr, "ms": ms,
-                    "Gq_per_s": Qr / ms / 1e6, "G_records_per_s": Qr * length / ms / 1e6,
-                    "GB_per_s_out": Qr * length * 16 / ms / 1e6})
-        del ko
-    return res
+        for G in groups:
+            o = hm.make_opts(group_size=G, flags=flags)
+            ms = timed(lambda: t.range(lo, hi, length, opts=o), reps)
+            res.append({"what": "range_batch", "T": T, "F": F, "G": G, "len": length, "Qr": Qr, "ms": ms,
+                        "Gq_per_s": Qr / ms / 1e6, "G_records_per_s": Qr * length / ms / 1e6,
+                        "GB_per_s_out": Qr * length * 16 / ms / 1e6})
+            print(json.dumps(res[-1]), flush=True)
+    return []
 
 
 def sweep_bench(T=1 << 26, Q=1 << 26, dist="zipf", reps=5):
@@ -92,6 +93,7 @@ if __name__ == "__main__":
     a = ap.parse_args()
     for w in a.what.split(","):
         rows = {"update": update_bench, "range": range_bench,
+                "range_sweep": lambda: range_bench(groups=(2, 4, 8, 16, 32)),
                 "sweep": lambda: sweep_bench(dist=a.sweep_dist)}[w]()
         for r in rows:
             print(json.dumps(r), flush=True)
