@@ -196,6 +196,66 @@ def random_ranges(keys: np.ndarray, Qr: int, seed: int = SEED_RANGE, max_width_k
     return np.ascontiguousarray(lo.astype(np.uint64)), np.ascontiguousarray(hi.astype(np.uint64))
 
 
+# ------------------------------------------------------------------------------ torch (device)
+# The same counter-based streams computed with torch int64 tensors (wrapping arithmetic, bit
+# patterns identical to the numpy uint64 versions) so that multi-GiB key sets and batches can
+# be generated directly in device memory.  tests/test_gen.py pins them to the numpy versions.
+def _t_lsr(x, s: int):
+    import torch
+
+    return (x >> s) & torch.tensor((1 << (64 - s)) - 1, dtype=torch.int64, device=x.device)
+
+
+def _t_const(v: int, device):
+    import torch
+
+    return torch.tensor(v - (1 << 64) if v >= (1 << 63) else v, dtype=torch.int64, device=device)
+
+
+def splitmix64_t(x):
+    """splitmix64 over an int64 tensor holding uint64 bit patterns."""
+    dev = x.device
+    x = x + _t_const(0x9E3779B97F4A7C15, dev)
+    z = (x ^ _t_lsr(x, 30)) * _t_const(0xBF58476D1CE4E5B9, dev)
+    z = (z ^ _t_lsr(z, 27)) * _t_const(0x94D049BB133111EB, dev)
+    return z ^ _t_lsr(z, 31)
+
+
+def _t_umod(h, m: int):
+    """unsigned 64-bit h mod m (m < 2^62) with int64 tensor ops."""
+    half = _t_lsr(h, 1) % m
+    return (half * 2 + (h & 1)) % m
+
+
+def _t_stream(seed: int, start: int, n: int, device):
+    import torch
+
+    idx = torch.arange(start, start + n, dtype=torch.int64, device=device)
+    return splitmix64_t(_t_const(seed & _M64, device) ^ idx)
+
+
+def uniform_keys_t(T: int, device, seed: int = SEED_KEY, start: int = 0, count: int | None = None):
+    """uniform_keys(T)[start:start+count] generated on `device` (int64 tensor of the uint64
+    keys); a slice is e.g. one key-range shard of the partitioned configuration."""
+    import torch
+
+    if count is None:
+        count = T - start
+    D = ((1 << 64) - 2) // T
+    i = torch.arange(start, start + count, dtype=torch.int64, device=device)
+    return i * _t_const(D, device) + _t_umod(_t_stream(seed, start, count, device), D)
+
+
+def values_for_t(keys, seed: int = SEED_VAL):
+    v = splitmix64_t(keys ^ _t_const(seed & _M64, keys.device))
+    return v ^ (v == -1).to(v.dtype)  # UINT64_MAX -> ^1
+
+
+def uniform_queries_t(keys, Q: int, seed: int = SEED_QUERY, start: int = 0):
+    T = keys.shape[0]
+    return keys[_t_umod(_t_stream(seed, start, Q, keys.device), T)]
+
+
 # ------------------------------------------------------------------------------ updates
 def update_ops(keys: np.ndarray, n: int, insert_frac: float = 0.05, delete_frac: float = 0.0,
                seed: int = SEED_OPS):

@@ -49,6 +49,21 @@ def test_queries_and_values():
     assert np.all(np.diff(s.reshape(4, 1024).astype(np.float64), axis=1) > 0)
 
 
+def test_torch_generators_equal_numpy():
+    import torch
+
+    for T in (4, 1000, 123457):
+        kn = gen.uniform_keys(T)
+        kt = gen.uniform_keys_t(T, "cpu").numpy().view(np.uint64)
+        assert np.array_equal(kn, kt)
+        assert np.array_equal(gen.values_for(kn), gen.values_for_t(torch.from_numpy(kn.view(np.int64))).numpy().view(np.uint64))
+        qn = gen.uniform_queries(kn, 5000, start=77)
+        qt = gen.uniform_queries_t(torch.from_numpy(kn.view(np.int64)), 5000, start=77).numpy().view(np.uint64)
+        assert np.array_equal(qn, qt)
+    x = np.array([0, 1, (1 << 64) - 1, 0x9E3779B97F4A7C15], dtype=np.uint64)
+    assert np.array_equal(gen.splitmix64(x), gen.splitmix64_t(torch.from_numpy(x.view(np.int64))).numpy().view(np.uint64))
+
+
 def test_ranges_count_len():
     k = gen.uniform_keys(1 << 12)
     lo, hi = gen.ranges(k, 100, 16)
