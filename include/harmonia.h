@@ -85,6 +85,9 @@ typedef struct {
 #define HARMONIA_QF_ILP1       16u /* k-ary search with one query per lane group instead of two */
 #define HARMONIA_QF_FUSE_SORT 128u /* G = 1: PSA chunk sort fused into the search kernel
                                       (ablation; measured slower than two kernels)          */
+#define HARMONIA_QF_SCATTER_RETURN 256u /* G = 1 PSA path: the search scatters results to
+                                      out[original position] instead of the default staged
+                                      return (chunk-local smem permutation + k_psa2_unmove) */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic

@@ -80,6 +80,12 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.smem_levels = lv;
   P.smem_nodes = (uint32_t)t->level_start[lv];
   P.smem_bytes = used + P.smem_nodes * t->F * 8;
+  // staged return (default for the G = 1 PSA path): results leave the search in level-1
+  // order through a kPsaChunk x 8-byte shared-memory stage, k_psa2_unmove restores the
+  // caller's order; two 1024-thread CTAs per SM must still fit
+  P.ret = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather && !P.fuse &&
+          !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
+          2 * (round_up(P.smem_bytes, 16) + kPsaChunk * 8 + 1024) <= t->smem_per_sm;
   *p = P;
   return HARMONIA_OK;
 }
@@ -117,10 +123,12 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
     const bool fused = p.fuse && p.G == 1 && !p.psa_global && p.psa_level2 == 0 && !p.gather &&
                        p.smem_bytes + (8u << 10) + (48u << 10) <= t->smem_optin;
-    harmonia_status s = p.psa_global ? psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
-                                     : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st,
-                                                      fused ? 2 : p.psa_level2);
-    if (s != HARMONIA_OK) return s;
+    harmonia_status s = HARMONIA_OK;
+    if (!p.ret) {
+      s = p.psa_global ? psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
+                       : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : p.psa_level2);
+      if (s != HARMONIA_OK) return s;
+    }
     a.q = w.sorted_q;
     a.n = nw;
     if (fused) {  // level-2 chunk sort inside the search kernel
@@ -128,6 +136,17 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       a.out = out + w0;
       a.bucket = p.bucket;
       if ((s = launch_sort_search(t, p, a, st)) != HARMONIA_OK) return s;
+      continue;
+    }
+    if (p.ret) {  // staged return: level-1-order results, then the inverse move
+      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, 0, true);
+      if (s != HARMONIA_OK) return s;
+      a.idx = w.idx;
+      a.out = w.sorted_out;
+      a.staged = 1;
+      a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
+      if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+      if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, st)) != HARMONIA_OK) return s;
       continue;
     }
     if (p.gather) {
@@ -384,7 +403,7 @@ extern "C" harmonia_status harmonia_route_partition(const uint64_t* d_split, uin
   cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
   BucketSplit f{d_split, P - 1};
   if (P <= 256)  // SMEM-aggregated two-level router (one atomic per tile and shard)
-    return route_partition2(d_q, n, f, P, w.counts, d_routed, d_pos, sm, (cudaStream_t)stream, h_counts);
+    return route_partition2(d_q, n, f, P, w, sm, (cudaStream_t)stream, h_counts);
   return psa_partition(d_q, n, f, P, w, sm, (cudaStream_t)stream, h_counts);
 }
 

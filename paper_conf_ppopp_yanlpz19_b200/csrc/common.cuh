@@ -102,6 +102,7 @@ struct harmonia_tree {
   float fill = 1.0f;
   int sm_count = 148;
   size_t smem_optin = 0;
+  size_t smem_per_sm = 0;
   size_t l2_bytes = 0;
   // host-pipeline streams/events (harmonia_search_batch_host)
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
@@ -131,6 +132,7 @@ struct Plan {
   int psa_level2 = 0;        // chunk sort: 0 counting, 1 ballot LSD, 2 none (coarse only)
   bool fuse = false;         // G = 1 + counting chunk sort fused into the search (k_sort_search)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
+  bool ret = false;          // staged inverse return (chunk-local result staging + unmove)
 };
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
@@ -145,7 +147,12 @@ struct PsaWs {
   uint64_t* sorted_q;   // window
   uint32_t* idx;        // window
   uint64_t* sorted_out; // window (gather mode only)
+  uint32_t* packed;     // window: coarse digit | rank-in-tile << 8 (two-level PSA / router)
+  uint32_t* tile_counts;// ceil(window / 2048) x 256 per-tile coarse bin counts
+  uint32_t* tile_base;  // ceil(window / 2048) x 256 level-1 start of each (tile, bin) run
 };
+constexpr uint32_t kPsaTile = 2048;   // level-1 tile (queries)
+constexpr uint32_t kPsaChunk = 4096;  // level-2 chunk (queries)
 constexpr uint32_t kScanTile = 4096;
 size_t psa_ws_bytes(const Plan& p);
 PsaWs psa_ws_carve(const Plan& p, void* base);
@@ -170,13 +177,19 @@ struct SearchArgs {
   uint64_t n;
   uint64_t* out;           // results: out[idx ? idx[j] : j]
   BucketBits bucket;       // PSA bucket (fused level-2 sort only)
+  uint32_t staged;         // staged return: idx holds chunk-local level-1 offsets and results
+                           // go through shared memory (at dynamic-smem offset res_smem_off)
+                           // to out[] in level-1 order, chunk by chunk (kPsaChunk)
+  uint32_t res_smem_off;
 };
 harmonia_status launch_sort_search(const harmonia_tree* t, const struct Plan& p, const SearchArgs& a,
                                    cudaStream_t st);
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
-                               int sm_count, cudaStream_t st, int level2 = 0);
-harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, uint32_t* counts,
-                                 uint64_t* routed, uint32_t* pos, int sm, cudaStream_t st, uint64_t* h_counts);
+                               int sm_count, cudaStream_t st, int level2 = 0, bool local = false);
+// inverse of the level-1 move for the staged return: out[e] = res1[level-1 position of e]
+harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, cudaStream_t st);
+harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
+                                 int sm, cudaStream_t st, uint64_t* h_counts);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
                               cudaStream_t st);
 

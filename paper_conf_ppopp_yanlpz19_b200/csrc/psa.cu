@@ -164,7 +164,9 @@ size_t psa_ws_bytes(const Plan& p) {
   b += round_up(ceil_div(p.nbins, kScanTile) * 4, 256);
   b += round_up(p.window * 8, 256);
   b += round_up(p.window * 4, 256);
-  if (p.gather) b += round_up(p.window * 8, 256);
+  if (p.gather || p.ret) b += round_up(p.window * 8, 256);
+  b += round_up(p.window * 4, 256);                        // packed digit/rank
+  b += 2 * round_up(ceil_div(p.window, kPsaTile) * 1024, 256);  // per-tile counts, run starts
   return b;
 }
 
@@ -179,7 +181,13 @@ PsaWs psa_ws_carve(const Plan& p, void* base) {
   c += round_up(p.window * 8, 256);
   w.idx = (uint32_t*)c;
   c += round_up(p.window * 4, 256);
-  w.sorted_out = p.gather ? (uint64_t*)c : nullptr;
+  w.sorted_out = (p.gather || p.ret) ? (uint64_t*)c : nullptr;
+  if (p.gather || p.ret) c += round_up(p.window * 8, 256);
+  w.packed = (uint32_t*)c;
+  c += round_up(p.window * 4, 256);
+  w.tile_counts = (uint32_t*)c;
+  c += round_up(ceil_div(p.window, kPsaTile) * 1024, 256);
+  w.tile_base = (uint32_t*)c;
   return w;
 }
 

@@ -446,7 +446,7 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
 template <int F, int U>
 __device__ __forceinline__ void lane_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                           bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
-                                          const uint64_t (&o)[U], const bool (&act)[U]) {
+                                          const bool (&act)[U], uint64_t (&res)[U]) {
   {
     uint64_t q[U];
     uint32_t node[U];
@@ -486,9 +486,15 @@ __device__ __forceinline__ void lane_core(const SearchArgs& a, const uint64_t* s
 #pragma unroll
       for (int u = 0; u < U; ++u) node[u] = first[u] + r[u];  // Eq 1
     }
+    // leaf: r = #keys <= q; the last key that compared <= q is key[r-1] (the successful
+    // steps of the power-of-two search visit increasing slots), so the probe needs no reload
     uint32_t r[U];
+    uint64_t best[U];
 #pragma unroll
-    for (int u = 0; u < U; ++u) r[u] = 0;
+    for (int u = 0; u < U; ++u) {
+      r[u] = 0;
+      best[u] = 0;
+    }
 #pragma unroll
     for (int s = F / 2; s >= 1; s >>= 1) {
       uint64_t k[U];
@@ -497,21 +503,18 @@ __device__ __forceinline__ void lane_core(const SearchArgs& a, const uint64_t* s
         k[u] = leaf_smem ? s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)]
                          : ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
 #pragma unroll
-      for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
-    }
-    uint64_t kk[U], vv[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      kk[u] = 0;
-      vv[u] = kNotFound;
-      if (live[u] && r[u] > 0) {
-        kk[u] = __ldg(a.keys + (uint64_t)node[u] * F + (r[u] - 1));
-        vv[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+      for (int u = 0; u < U; ++u) {
+        const bool le = k[u] <= q[u];
+        r[u] += le ? s : 0;
+        best[u] = le ? k[u] : best[u];
       }
     }
 #pragma unroll
-    for (int u = 0; u < U; ++u)
-      if (act[u]) a.out[o[u]] = (live[u] && r[u] > 0 && kk[u] == q[u]) ? vv[u] : kNotFound;
+    for (int u = 0; u < U; ++u) {
+      res[u] = kNotFound;
+      if (live[u] && r[u] > 0 && best[u] == q[u])
+        res[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+    }
   }
 }
 
@@ -537,7 +540,52 @@ __global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const 
       q0[u] = act[u] ? ld_stream(a.q + j) : kPad;
       o[u] = (act[u] && a.idx) ? (uint64_t)ld_stream32(a.idx + j) : j;
     }
-    lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, o, act);
+    uint64_t res[U];
+    lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (act[u]) a.out[o[u]] = res[u];
+  }
+}
+
+// G = 1 search with the staged return (default PSA path). A CTA takes whole level-2 chunks;
+// idx holds each query's chunk-local level-1 offset, so the chunk's results are permuted
+// back to level-1 order in shared memory and written contiguously -- the scattered 8-byte
+// stores to out[original position] (measured: a third of the kernel) are replaced by
+// k_psa2_unmove's run-wise copy.
+template <int F, int U>
+__global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  uint64_t* s_res = reinterpret_cast<uint64_t*>(smem + a.res_smem_off);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint64_t c0 = (uint64_t)blockIdx.x * kPsaChunk; c0 < a.n; c0 += (uint64_t)gridDim.x * kPsaChunk) {
+    const uint32_t m = (uint32_t)(a.n - c0 < kPsaChunk ? a.n - c0 : kPsaChunk);
+    for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
+      uint64_t q0[U];
+      uint32_t o[U];
+      bool act[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const uint32_t j = b0 + u * 32 + lane;
+        act[u] = j < m;
+        q0[u] = act[u] ? ld_stream(a.q + c0 + j) : kPad;
+        o[u] = act[u] ? ld_stream32(a.idx + c0 + j) : 0u;
+      }
+      uint64_t res[U];
+      lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (act[u]) s_res[o[u]] = res[u];
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) a.out[c0 + i] = s_res[i];
+    __syncthreads();
   }
 }
 
@@ -656,7 +704,11 @@ __global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArg
         q0[u] = act[u] ? sq[p] : kPad;
         o[u] = act[u] ? si[p] : 0;
       }
-      lane_core<F, 2>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, o, act);
+      uint64_t res[2];
+      lane_core<F, 2>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+#pragma unroll
+      for (int u = 0; u < 2; ++u)
+        if (act[u]) a.out[o[u]] = res[u];
     }
     __syncthreads();  // the chunk buffers are reused
   }
@@ -775,7 +827,32 @@ harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, cons
 }
 
 template <int F>
+harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  const int U = p.lane_ilp;
+  auto kern = U >= 4 ? k_lane_search_c<F, 4> : (U == 2 ? k_lane_search_c<F, 2> : k_lane_search_c<F, 1>);
+  const uint32_t smem = a.res_smem_off + kPsaChunk * 8;
+  static int configured_smem[5] = {-1, -1, -1, -1, -1};
+  const int ci = U >= 4 ? 4 : U;
+  if ((int)smem > configured_smem[ci]) {
+    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    configured_smem[ci] = (int)smem;
+  }
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, smem));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t need = ceil_div(a.n, kPsaChunk);
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
+  {
+    ProfScope ps_(HARMONIA_PROF_SEARCH, st);
+    kern<<<grid, 1024, smem, st>>>(a);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+template <int F>
 harmonia_status launch_lane_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
+  if (a.staged) return launch_lane_search_c<F>(t, p, a, st);
   const int U = p.lane_ilp;
   auto kern = U >= 4 ? k_lane_search_u<F, 4> : (U == 2 ? k_lane_search_u<F, 2> : k_lane_search<F>);
   const int bs = U >= 2 ? 1024 : kQueryBlock;

@@ -239,6 +239,7 @@ extern "C" harmonia_status harmonia_build(const uint64_t* keys, const uint64_t* 
   }
   t->sm_count = prop.multiProcessorCount;
   t->smem_optin = prop.sharedMemPerBlockOptin;
+  t->smem_per_sm = prop.sharedMemPerMultiprocessor;
   t->l2_bytes = prop.l2CacheSize;
 
   if (on_dev && n > 0) {
