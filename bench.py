@@ -421,7 +421,8 @@ def main():
     if dom_kind == "search":
         avg_ms = dom_ms / dom_n
         achieved = bytes_launch / (avg_ms / 1e3) / 1e9
-        kname = {1: "k_lane_search_u"}.get(plan["group_size"], "k_ntg_search2")
+        kname = ("k_lane_search_c" if plan.get("staged_return") else "k_lane_search_u") \
+            if plan["group_size"] == 1 else "k_ntg_search2"
         roof = {"bound": "hbm", "kernel": kname, "achieved": achieved, "peak": hbm_peak,
                 "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": None, "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": bytes_launch, "queries_per_launch": nw,
@@ -429,7 +430,10 @@ def main():
                 "no_reuse_frac": (nw * noreuse_bpq) / (avg_ms / 1e3) / 1e9 / hbm_peak}
     else:
         # PSA kernels are streaming passes over the window: 8 B read (+12 B written by scatter)
-        per_q = {"psa_hist": 8, "psa_scatter": 8 + 8 + 4, "psa_scan": 0, "return": 8 + 4 + 8}.get(dom_kind, 8)
+        # rank: 8 B query in, 4 B packed digit/rank out; move: query + packed in, query out;
+        # chunk sort: query in, query + 4 B offset out; unmove: packed + result in, result out
+        per_q = {"psa_hist": 8 + 4, "psa_scatter": 8 + 4 + 8, "psa_scan": 8 + 8 + 4,
+                 "return": 4 + 8 + 8}.get(dom_kind, 8)
         avg_ms = dom_ms / dom_n
         achieved = nw * per_q / (avg_ms / 1e3) / 1e9
         roof = {"bound": "hbm", "kernel": dom_kind, "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
@@ -442,6 +446,9 @@ def main():
         if ent:
             roof["traffic"] = ent["dram_bytes_per_launch"]
             roof["traffic_source"] = ent.get("source")
+            if "l1_wavefront_pct" in ent:  # the on-chip limiter of the search
+                roof["limiter"] = {"resource": "L1 data-pipe (LSU) wavefronts", "frac": ent["l1_wavefront_pct"] / 100,
+                                   "source": ent.get("source")}
     except Exception:
         pass
 

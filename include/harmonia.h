@@ -136,10 +136,13 @@ harmonia_status harmonia_export_layout(const harmonia_tree* tree, uint64_t* h_ke
 /* ---------------------------------------------------------------------------------------
  * harmonia_search_batch — n point queries (§3.2.1; PSA §4.1; NTG §4.2).
  *   d_queries[n] -> d_values_out[n]: the value of each query's key, or HARMONIA_NOT_FOUND.
- *   Pipeline per PSA window: bucket histogram on the top Nb key bits, scan, stable-per-warp
- *   bucket scatter (PSA, Eq 2), NTG descent with Eq 1 (child = PS[node] + i - 1) and leaf
- *   probe, results written back in the caller's order.  d_queries and d_values_out may not
- *   overlap.  d_workspace must hold harmonia_search_workspace_bytes(tree, n, opts) bytes,
+ *   Pipeline per PSA window (default: the whole batch up to 2^27 queries): PSA (Eq 2) as a
+ *   two-level partition on the top Nb key bits -- 8-bit coarse rank + move passes, then a
+ *   4096-query chunk counting sort on all Nb bits -- the descent with Eq 1 (child =
+ *   PS[node] + i - 1) and leaf probe, then the results go back to the caller's order through
+ *   a chunk-local shared-memory permutation and the inverse of the coarse move.  d_queries
+ *   and d_values_out may not overlap.  d_workspace must hold
+ *   harmonia_search_workspace_bytes(tree, n, opts) bytes (about 36 bytes per window query),
  *   16-byte aligned.   Errors: INVALID_ARG, DEVICE_MISMATCH, CUDA.
  * ------------------------------------------------------------------------------------- */
 size_t harmonia_search_workspace_bytes(const harmonia_tree* tree, uint64_t n,
@@ -218,7 +221,9 @@ typedef struct {
   int32_t group_size, psa_bits, smem_levels, ps_in_smem;
   uint64_t window;
   uint32_t smem_bytes, smem_nodes;
-  uint64_t reserved[2];
+  uint32_t staged_return;  /* 1: results return through the chunk-local stage + inverse move */
+  uint32_t lane_queries;   /* G = 1: queries interleaved per lane */
+  uint64_t reserved;
 } harmonia_plan;
 harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
                                     const harmonia_query_opts* opts, harmonia_plan* out);

@@ -55,7 +55,8 @@ class QueryOpts(C.Structure):
 class PlanInfo(C.Structure):
     _fields_ = [("group_size", C.c_int32), ("psa_bits", C.c_int32), ("smem_levels", C.c_int32),
                 ("ps_in_smem", C.c_int32), ("window", C.c_uint64), ("smem_bytes", C.c_uint32),
-                ("smem_nodes", C.c_uint32), ("reserved", C.c_uint64 * 2)]
+                ("smem_nodes", C.c_uint32), ("staged_return", C.c_uint32), ("lane_queries", C.c_uint32),
+                ("reserved", C.c_uint64)]
 
 
 class Info(C.Structure):

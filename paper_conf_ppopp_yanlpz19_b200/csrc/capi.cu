@@ -11,7 +11,7 @@ namespace hm {
 
 namespace {
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
-constexpr uint64_t kAutoWindow = 1ull << 23;  // auto PSA window (queries): measured best, DESIGN.md §8
+constexpr uint64_t kAutoWindow = 1ull << 27;  // auto PSA window (queries): measured best, DESIGN.md §8
 
 bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 }  // namespace
@@ -83,7 +83,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   // staged return (default for the G = 1 PSA path): results leave the search in level-1
   // order through a kPsaChunk x 8-byte shared-memory stage, k_psa2_unmove restores the
   // caller's order; two 1024-thread CTAs per SM must still fit
-  P.ret = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather && !P.fuse &&
+  P.ret = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather &&
           !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
           2 * (round_up(P.smem_bytes, 16) + kPsaChunk * 8 + 1024) <= t->smem_per_sm;
   *p = P;
@@ -131,7 +131,7 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
     }
     a.q = w.sorted_q;
     a.n = nw;
-    if (fused) {  // level-2 chunk sort inside the search kernel
+    if (fused && !p.ret) {  // level-2 chunk sort inside the search kernel
       a.idx = w.idx;
       a.out = out + w0;
       a.bucket = p.bucket;
@@ -139,13 +139,14 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       continue;
     }
     if (p.ret) {  // staged return: level-1-order results, then the inverse move
-      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, 0, true);
+      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : 0, true);
       if (s != HARMONIA_OK) return s;
       a.idx = w.idx;
       a.out = w.sorted_out;
       a.staged = 1;
       a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
-      if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+      a.bucket = p.bucket;
+      if ((s = fused ? launch_sort_search(t, p, a, st) : launch_search(t, p, a, st)) != HARMONIA_OK) return s;
       if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, st)) != HARMONIA_OK) return s;
       continue;
     }
@@ -219,6 +220,8 @@ extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t 
   out->window = p.psa ? p.window : 0;
   out->smem_bytes = p.smem_bytes;
   out->smem_nodes = p.smem_nodes;
+  out->staged_return = p.ret ? 1u : 0u;
+  out->lane_queries = p.G == 1 ? (uint32_t)p.lane_ilp : 0u;
   return HARMONIA_OK;
 }
 

@@ -598,7 +598,10 @@ constexpr int kFuseThreads = 1024, kFusePer = 4, kFuseChunk = kFuseThreads * kFu
 constexpr int kFuseBins = 2048;
 constexpr uint32_t kFuseSmem = kFuseBins * 4 + kFuseChunk * 12;  // + the staged tree top
 
-template <int F>
+// kStaged (staged return): the chunk's own positions are the level-1 offsets, so idx is not
+// read; results are permuted back to chunk order in shared memory (over the sorted queries,
+// after every lane has read its queries) and written contiguously.
+template <int F, bool kStaged>
 __global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
@@ -627,7 +630,7 @@ __global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArg
       b[k] = 0;
       if (e < m) {
         v[k] = ld_stream(a.q + c0 + e);
-        ix[k] = ld_stream32(a.idx + c0 + e);
+        ix[k] = kStaged ? e : ld_stream32(a.idx + c0 + e);
         b[k] = a.bucket(v[k]);
         bmin = min(bmin, b[k]);
         bmax = max(bmax, b[k]);
@@ -693,6 +696,9 @@ __global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArg
     }
     __syncthreads();
     // ---- search the sorted chunk: warp w takes positions [w*128, w*128+128), 2 per lane per round
+    uint64_t rr[kFusePer];
+    uint32_t ro[kFusePer];
+    bool ra[kFusePer];
 #pragma unroll
     for (int rd = 0; rd < kFusePer / 2; ++rd) {
       uint64_t q0[2], o[2];
@@ -707,8 +713,23 @@ __global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArg
       uint64_t res[2];
       lane_core<F, 2>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
 #pragma unroll
-      for (int u = 0; u < 2; ++u)
-        if (act[u]) a.out[o[u]] = res[u];
+      for (int u = 0; u < 2; ++u) {
+        if constexpr (kStaged) {
+          rr[rd * 2 + u] = res[u];
+          ro[rd * 2 + u] = (uint32_t)o[u];
+          ra[rd * 2 + u] = act[u];
+        } else if (act[u]) {
+          a.out[o[u]] = res[u];
+        }
+      }
+    }
+    if constexpr (kStaged) {
+      __syncthreads();  // every lane has read its queries: sq becomes the result stage
+#pragma unroll
+      for (int k = 0; k < kFusePer; ++k)
+        if (ra[k]) sq[ro[k]] = rr[k];
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < m; i += kFuseThreads) a.out[c0 + i] = sq[i];
     }
     __syncthreads();  // the chunk buffers are reused
   }
@@ -806,12 +827,12 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(co
 
 template <int F>
 harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
-  auto kern = k_sort_search<F>;
+  auto kern = a.staged ? k_sort_search<F, true> : k_sort_search<F, false>;
   const uint32_t smem = p.smem_bytes + kFuseSmem;
-  static int configured_smem = -1;
-  if ((int)smem > configured_smem) {
+  static int configured_smem[2] = {-1, -1};
+  if ((int)smem > configured_smem[a.staged ? 1 : 0]) {
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured_smem = (int)smem;
+    configured_smem[a.staged ? 1 : 0] = (int)smem;
   }
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFuseThreads, smem));

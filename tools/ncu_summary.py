@@ -10,6 +10,7 @@ import csv
 import io
 import json
 import os
+import re
 import subprocess
 
 METRICS = [
@@ -22,13 +23,15 @@ METRICS = [
     "smsp__sass_average_branch_targets_threads_uniform.pct",
     "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
     "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
+    "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
 ]
 
 
 def short(name):
-    n = name.split("(")[0]
-    for p in ("void ", "hm::", "<unnamed>::", "unnamed>::", "(anonymous namespace)::"):
-        n = n.replace(p, "")
+    n = name.replace("(anonymous namespace)::", "").replace("::<unnamed>::", "::")
+    n = re.sub(r"^(void )?<unnamed>::", "", n).replace("unnamed>::", "")
+    n = n.replace("void ", "").replace("hm::", "").split("(")[0]
     return n.strip()
 
 
@@ -103,8 +106,12 @@ if __name__ == "__main__":
         k = d["kernel"].split("<")[0]
         rd = to_bytes(d.get("dram__bytes_read.sum", 0), d.get("dram__bytes_read.sum.unit", "byte"))
         wr = to_bytes(d.get("dram__bytes_write.sum", 0), d.get("dram__bytes_write.sum.unit", "byte"))
-        tr.setdefault(a.workload, {}).setdefault(k, {"dram_bytes_per_launch": rd + wr,
-                                                     "source": os.path.basename(a.out) + ".json (ncu --set full, cold L2)"})
+        ent = {"dram_bytes_per_launch": rd + wr,
+               "source": os.path.basename(a.out) + ".json (ncu --set full, cold L2)"}
+        l1 = d.get("l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed")
+        if isinstance(l1, float):
+            ent["l1_wavefront_pct"] = l1
+        tr.setdefault(a.workload, {})[k] = ent  # the newest capture supersedes
     json.dump(tr, open(tr_path, "w"), indent=1)
     with open(a.out + ".md", "w") as f:
         f.write(f"# ncu summary {os.path.basename(a.out)} — {a.workload}\n\n")
