@@ -88,6 +88,9 @@ typedef struct {
 #define HARMONIA_QF_SCATTER_RETURN 256u /* G = 1 PSA path: the search scatters results to
                                       out[original position] instead of the default staged
                                       return (chunk-local smem permutation + k_psa2_unmove) */
+#define HARMONIA_QF_PSA_WIDE 512u /* staged return with an 11-bit (2048-bin) level-1 partition
+                                      instead of the default 8-bit one (ablation: denser
+                                      chunks for the search, but 2-query runs in the moves)  */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic

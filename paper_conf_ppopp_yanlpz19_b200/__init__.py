@@ -28,6 +28,7 @@ QF_PSA_COARSE = 32
 QF_PSA_LSD = 64
 QF_FUSE_SORT = 128
 QF_SCATTER_RETURN = 256
+QF_PSA_WIDE = 512
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
            6: "DEVICE_MISMATCH", 7: "TOO_LARGE"}
 

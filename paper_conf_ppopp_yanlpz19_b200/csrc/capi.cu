@@ -86,6 +86,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.ret = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather &&
           !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
           2 * (round_up(P.smem_bytes, 16) + kPsaChunk * 8 + 1024) <= t->smem_per_sm;
+  P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
   *p = P;
   return HARMONIA_OK;
 }
@@ -139,7 +140,7 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       continue;
     }
     if (p.ret) {  // staged return: level-1-order results, then the inverse move
-      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : 0, true);
+      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : 0, true, p.wide);
       if (s != HARMONIA_OK) return s;
       a.idx = w.idx;
       a.out = w.sorted_out;
@@ -147,7 +148,7 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
       a.bucket = p.bucket;
       if ((s = fused ? launch_sort_search(t, p, a, st) : launch_search(t, p, a, st)) != HARMONIA_OK) return s;
-      if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, st)) != HARMONIA_OK) return s;
+      if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, t->sm_count, st, p.wide)) != HARMONIA_OK) return s;
       continue;
     }
     if (p.gather) {

@@ -133,6 +133,7 @@ struct Plan {
   bool fuse = false;         // G = 1 + counting chunk sort fused into the search (k_sort_search)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
   bool ret = false;          // staged inverse return (chunk-local result staging + unmove)
+  bool wide = false;         // staged return with the 11-bit level-1 partition
 };
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
@@ -149,9 +150,18 @@ struct PsaWs {
   uint64_t* sorted_out; // window (gather mode only)
   uint32_t* packed;     // window: coarse digit | rank-in-tile << 8 (two-level PSA / router)
   uint32_t* tile_counts;// ceil(window / 2048) x 256 per-tile coarse bin counts
-  uint32_t* tile_base;  // ceil(window / 2048) x 256 level-1 start of each (tile, bin) run
+  uint32_t* cta_counts; // kL1CtaRows: per level-1 CTA bin totals
+  uint32_t* cta_base;   // kL1CtaRows: per level-1 CTA first global slot of each bin
 };
-constexpr uint32_t kPsaTile = 2048;   // level-1 tile (queries)
+constexpr uint64_t kL1CtaRows = 2048 * 2048;  // >= (level-1 CTAs) x (bins) for every tiling
+constexpr uint32_t kPsaTile = 2048;   // level-1 tile (queries), 256-bin configuration
+// bytes of one per-(tile, bin) array: max over the level-1 tilings (256 bins / 2048-query
+// tiles; 2048 bins / 4096- or 8192-query tiles), 4 bytes per (tile, bin)
+inline uint64_t l1_rows_bytes(uint64_t window) {
+  const uint64_t a = (window + 2047) / 2048 * 256 * 4, b = (window + 4095) / 4096 * 2048 * 4,
+                 c = (window + 8191) / 8192 * 2048 * 4;
+  return a > b ? (a > c ? a : c) : (b > c ? b : c);
+}
 constexpr uint32_t kPsaChunk = 4096;  // level-2 chunk (queries)
 constexpr uint32_t kScanTile = 4096;
 size_t psa_ws_bytes(const Plan& p);
@@ -185,9 +195,11 @@ struct SearchArgs {
 harmonia_status launch_sort_search(const harmonia_tree* t, const struct Plan& p, const SearchArgs& a,
                                    cudaStream_t st);
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
-                               int sm_count, cudaStream_t st, int level2 = 0, bool local = false);
+                               int sm_count, cudaStream_t st, int level2 = 0, bool local = false,
+                               bool wide = false);
 // inverse of the level-1 move for the staged return: out[e] = res1[level-1 position of e]
-harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, cudaStream_t st);
+harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
+                                 cudaStream_t st, bool wide);
 harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
                                  int sm, cudaStream_t st, uint64_t* h_counts);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,

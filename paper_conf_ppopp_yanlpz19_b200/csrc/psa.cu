@@ -166,7 +166,8 @@ size_t psa_ws_bytes(const Plan& p) {
   b += round_up(p.window * 4, 256);
   if (p.gather || p.ret) b += round_up(p.window * 8, 256);
   b += round_up(p.window * 4, 256);                        // packed digit/rank
-  b += 2 * round_up(ceil_div(p.window, kPsaTile) * 1024, 256);  // per-tile counts, run starts
+  b += round_up(l1_rows_bytes(p.window), 256);        // per-tile counts
+  b += 2 * kL1CtaRows * 4;                             // per-CTA counts and bases
   return b;
 }
 
@@ -186,8 +187,10 @@ PsaWs psa_ws_carve(const Plan& p, void* base) {
   w.packed = (uint32_t*)c;
   c += round_up(p.window * 4, 256);
   w.tile_counts = (uint32_t*)c;
-  c += round_up(ceil_div(p.window, kPsaTile) * 1024, 256);
-  w.tile_base = (uint32_t*)c;
+  c += round_up(l1_rows_bytes(p.window), 256);
+  w.cta_counts = (uint32_t*)c;
+  c += kL1CtaRows * 4;
+  w.cta_base = (uint32_t*)c;
   return w;
 }
 

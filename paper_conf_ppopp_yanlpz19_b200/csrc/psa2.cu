@@ -23,8 +23,6 @@ namespace hm {
 
 namespace {
 
-constexpr int kCoarseBits = 8, kCoarseBins = 1 << kCoarseBits;
-constexpr int kWarps = kBlock / 32;                      // 8 warps per 256-thread CTA
 constexpr int kBatches = 8;                              // 32-query batches per warp per tile
 constexpr int kCoarseTile = kBlock * kBatches;           // 2048 queries per scatter tile
 #ifndef HM_SORT_THREADS
@@ -96,211 +94,276 @@ struct CoarseDigit {
   __device__ __forceinline__ uint32_t operator()(uint64_t q) const { return f(q) >> shift; }
 };
 
-// ---- level 1, pass 1: per-tile digit ranks ---------------------------------------------
-// Tiles of kCoarseTile consecutive queries. Each query's coarse digit d and its rank among the
-// tile's queries with digit d are taken once, with a shared-memory atomic, and stored packed
-// (d | rank << 8) so that the move pass below needs no multisplit. Per-tile bin counts go to
-// tile_counts[tile][256]; bin totals to counts[256] (one global atomic per tile and bin).
-// Digit: any functor mapping a query to [0, kCoarseBins) (the PSA coarse digit, or the
-// destination shard of the partitioned multi-GPU mode).
-template <class Digit>
-__global__ void __launch_bounds__(kBlock) k_psa2_rank(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
-                                                      uint32_t* __restrict__ counts,
-                                                      uint32_t* __restrict__ tile_counts,
-                                                      uint32_t* __restrict__ packed) {
-#ifndef HARMONIA_RANK_BALLOT
-  __shared__ uint32_t cnt[kCoarseBins];
-  uint64_t v[kBatches];
+// ---- level-1 configurations -------------------------------------------------------------
+// BITS-bit coarse digit, TILE queries per tile, NT threads per CTA (PER = TILE / NT queries
+// per thread).  Narrow: 256 bins -- the multi-GPU router and the non-staged PSA modes.  Wide:
+// 2048 bins -- the default staged-return PSA: a 4096-query level-2 chunk then spans ~2
+// coarse bins instead of 1/8 of one, so the search sees ~8x denser key ranges per warp.
+template <int BITS_, int TILE_, int NT_>
+struct L1Cfg {
+  static constexpr int BITS = BITS_, BINS = 1 << BITS_, TILE = TILE_, NT = NT_, PER = TILE_ / NT_;
+  static constexpr int BPT = BINS / NT_;  // bins per thread in scans
+  static constexpr int MINB = 1024 / NT_;  // >= 1024 resident threads per SM (<= 64 registers)
+  static constexpr int TILE_SHIFT = (TILE_ == 2048 ? 11 : TILE_ == 4096 ? 12 : 13);
+  static_assert(BINS % NT_ == 0 && TILE_ % NT_ == 0 && (1 << TILE_SHIFT) == TILE_, "L1Cfg");
+  static_assert(BITS_ + TILE_SHIFT <= 32 && BITS_ + TILE_SHIFT + 0 <= 32, "packed digit|rank");
+};
+using Narrow = L1Cfg<8, 2048, 256>;
+#ifndef HM_WIDE_TILE
+#define HM_WIDE_TILE 4096
+#endif
+using Wide = L1Cfg<11, HM_WIDE_TILE, 512>;
+
+// exclusive scan over C::BINS values held BPT per thread (thread t owns [t*BPT, t*BPT+BPT))
+template <class C>
+__device__ __forceinline__ void scan_bins(const uint32_t (&v)[C::BPT], uint32_t (&ex)[C::BPT], uint32_t* tmp) {
+  uint32_t s = 0;
 #pragma unroll
-  for (int k = 0; k < kBatches; ++k) {  // all loads first (kBatches in flight per thread)
-    const uint64_t e = (uint64_t)blockIdx.x * kCoarseTile + k * kBlock + threadIdx.x;
-    v[k] = e < n ? __ldg(q + e) : 0;
+  for (int k = 0; k < C::BPT; ++k) {
+    ex[k] = s;
+    s += v[k];
   }
-  for (uint64_t tile = blockIdx.x; tile * kCoarseTile < n; tile += gridDim.x) {
-    const uint64_t t0 = tile * kCoarseTile;
-    cnt[threadIdx.x] = 0;
+  const uint32_t base = block_scan<C::NT>(s, tmp, nullptr);
+#pragma unroll
+  for (int k = 0; k < C::BPT; ++k) ex[k] += base;
+}
+
+// Level-1 CTAs are persistent: CTA c owns the contiguous tile range [c*T/G, (c+1)*T/G) in all
+// three passes (rank, move, unmove), so bin space is reserved once per (CTA, bin) -- one
+// global atomic each -- instead of once per (tile, bin), and the inverse move recomputes
+// every tile's run starts from the CTA base and the tile counts.
+__device__ __forceinline__ void l1_tile_range(uint64_t n, uint32_t tile, uint64_t* tb, uint64_t* te) {
+  const uint64_t T = (n + tile - 1) / tile;
+  *tb = (uint64_t)blockIdx.x * T / gridDim.x;
+  *te = (uint64_t)(blockIdx.x + 1) * T / gridDim.x;
+}
+
+// ---- level 1, pass 1: per-tile digit ranks ---------------------------------------------
+// Each query's coarse digit d and its rank among the tile's queries with digit d are taken
+// once, with a shared-memory atomic, and stored packed (d | rank << BITS) so that the move
+// pass needs no multisplit (the ballot multisplit was measured slower: DESIGN.md §8).
+// Per-tile bin counts go to tile_counts[tile][BINS], the CTA's totals to cta_counts[c][BINS]
+// and the bin totals to counts[BINS].  Digit: any functor mapping a query to [0, BINS) (the
+// PSA coarse digit, or the destination shard of the partitioned multi-GPU mode).
+template <class Digit, class C>
+__global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_rank(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
+                                                              uint32_t* __restrict__ counts,
+                                                              uint32_t* __restrict__ tile_counts,
+                                                              uint32_t* __restrict__ packed,
+                                                              uint32_t* __restrict__ cta_counts) {
+  __shared__ uint32_t cnt[C::BINS];
+  uint64_t tb, te;
+  l1_tile_range(n, C::TILE, &tb, &te);
+  uint32_t acc[C::BPT];
+#pragma unroll
+  for (int k = 0; k < C::BPT; ++k) acc[k] = 0;
+  for (uint64_t tile = tb; tile < te; ++tile) {
+    const uint64_t t0 = tile * C::TILE;
+    uint64_t v[C::PER];
+#pragma unroll
+    for (int k = 0; k < C::PER; ++k) {  // all loads first (PER in flight per thread)
+      const uint64_t e = t0 + k * C::NT + threadIdx.x;
+      v[k] = e < n ? __ldg(q + e) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < C::BPT; ++k) cnt[k * C::NT + threadIdx.x] = 0;
     __syncthreads();
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + k * kBlock + threadIdx.x;
+    for (int k = 0; k < C::PER; ++k) {
+      const uint64_t e = t0 + k * C::NT + threadIdx.x;
       if (e < n) {
         const uint32_t d = dg(v[k]);
-        packed[e] = d | (atomicAdd(&cnt[d], 1u) << kCoarseBits);
+        packed[e] = d | (atomicAdd(&cnt[d], 1u) << C::BITS);
       }
     }
     __syncthreads();
-    const uint32_t c = cnt[threadIdx.x];
-    tile_counts[tile * kCoarseBins + threadIdx.x] = c;
-    if (c) atomicAdd(counts + threadIdx.x, c);
-    __syncthreads();
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + (uint64_t)gridDim.x * kCoarseTile + k * kBlock + threadIdx.x;
-      v[k] = e < n ? __ldg(q + e) : 0;
-    }
-  }
-#else  // ballot multisplit ranks (per-warp runs, then warp offsets per bin)
-  __shared__ uint32_t wcnt[kWarps][kCoarseBins];
-  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t tile = blockIdx.x; tile * kCoarseTile < n; tile += gridDim.x) {
-    const uint64_t t0 = tile * kCoarseTile;
-    for (int i = threadIdx.x; i < kWarps * kCoarseBins; i += kBlock) (&wcnt[0][0])[i] = 0;
-    __syncthreads();
-    uint64_t v[kBatches];
-    uint32_t d[kBatches], pos[kBatches];
-#pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + warp * (32 * kBatches) + k * 32 + lane;
-      v[k] = e < n ? __ldg(q + e) : 0;
-    }
-#pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + warp * (32 * kBatches) + k * 32 + lane;
-      const bool valid = e < n;
-      d[k] = valid ? dg(v[k]) : 0u;
-      const unsigned peers = peers_of<kCoarseBits>(d[k], __ballot_sync(kFull, valid));
-      const uint32_t run = valid ? wcnt[warp][d[k]] : 0u;
-      __syncwarp();
-      if (valid && lane == (unsigned)(__ffs(peers) - 1)) wcnt[warp][d[k]] = run + __popc(peers);
-      __syncwarp();
-      pos[k] = run + __popc(peers & lane_lt());
-    }
-    __syncthreads();
-    uint32_t acc = 0;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) {
-      const uint32_t c = wcnt[w][threadIdx.x];
-      wcnt[w][threadIdx.x] = acc;
-      acc += c;
-    }
-    tile_counts[tile * kCoarseBins + threadIdx.x] = acc;
-    if (acc) atomicAdd(counts + threadIdx.x, acc);
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + warp * (32 * kBatches) + k * 32 + lane;
-      if (e < n) packed[e] = d[k] | ((wcnt[warp][d[k]] + pos[k]) << kCoarseBits);
+    for (int k = 0; k < C::BPT; ++k) {
+      const uint32_t c = cnt[k * C::NT + threadIdx.x];
+      tile_counts[tile * C::BINS + k * C::NT + threadIdx.x] = c;
+      acc[k] += c;
     }
     __syncthreads();
   }
-#endif
+#pragma unroll
+  for (int k = 0; k < C::BPT; ++k) {
+    const uint32_t b = k * C::NT + threadIdx.x;
+    cta_counts[(uint64_t)blockIdx.x * C::BINS + b] = acc[k];
+    if (acc[k]) atomicAdd(counts + b, acc[k]);
+  }
 }
 
 // ---- level 1, pass 2: move ----------------------------------------------------------------
-// Global position of query e = exclusive-prefix(counts)[d] + this tile's reservation in bin d
-// (one atomic per tile and bin on cursor[d]) + rank. Staged through shared memory in bin order
-// so that each bin's run is written by consecutive lanes. The scattered shared-memory stores
-// are the kernel's limiter (ncu: shared-store wavefronts), so only the query is staged when the
-// digit is cheap to recompute (the PSA coarse digit) and the position only when idx is wanted.
-template <class Digit>
-__global__ void __launch_bounds__(kBlock) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
-                                                      const uint32_t* __restrict__ counts,
-                                                      uint32_t* __restrict__ cursor,
-                                                      const uint32_t* __restrict__ tile_counts,
-                                                      const uint32_t* __restrict__ packed,
-                                                      uint64_t* __restrict__ sorted_q, uint32_t* __restrict__ idx,
-                                                      uint32_t* __restrict__ tile_base) {
+// Global position of query e = exclusive-prefix(counts)[d] + the CTA's reservation in bin d
+// (one atomic per CTA and non-empty bin on cursor[d]) + the earlier tiles of the CTA + rank.
+// Staged through shared memory in bin order so that each bin's run is written by consecutive
+// lanes.  The scattered shared-memory stores are the limiter (ncu: shared-store wavefronts),
+// so only the query is staged when the digit is cheap to recompute (the PSA coarse digit) and
+// the position only when idx is wanted (kIdx).
+template <class Digit, class C, bool kIdx>
+__global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
+                                                              const uint32_t* __restrict__ counts,
+                                                              uint32_t* __restrict__ cursor,
+                                                              const uint32_t* __restrict__ tile_counts,
+                                                              const uint32_t* __restrict__ packed,
+                                                              const uint32_t* __restrict__ cta_counts,
+                                                              uint32_t* __restrict__ cta_base,
+                                                              uint64_t* __restrict__ sorted_q,
+                                                              uint32_t* __restrict__ idx) {
   constexpr bool kRecompute = std::is_same<Digit, CoarseDigit>::value;
-  __shared__ uint32_t prefix[kCoarseBins], bin_start[kCoarseBins], gbase[kCoarseBins], tmp[kWarps + 1];
-  __shared__ uint64_t st_q[kCoarseTile];
-  __shared__ uint32_t st_i[kCoarseTile];
-  __shared__ uint8_t st_d[kRecompute ? 1 : kCoarseTile];
-  prefix[threadIdx.x] = block_scan<kBlock>(counts[threadIdx.x], tmp, nullptr);
-  for (uint64_t tile = blockIdx.x; tile * kCoarseTile < n; tile += gridDim.x) {
-    const uint64_t t0 = tile * kCoarseTile;
-    uint64_t v[kBatches];
-    uint32_t pk[kBatches];
+  extern __shared__ __align__(16) unsigned char l1_smem[];
+  uint64_t* st_q = reinterpret_cast<uint64_t*>(l1_smem);
+  uint32_t* bin_start = reinterpret_cast<uint32_t*>(l1_smem + C::TILE * 8);
+  uint32_t* gbase = bin_start + C::BINS;
+  uint32_t* st_i = gbase + C::BINS;                                       // kIdx
+  uint8_t* st_d = reinterpret_cast<uint8_t*>(st_i + (kIdx ? C::TILE : 0));  // !kRecompute
+  __shared__ uint32_t tmp[C::NT / 32 + 1];
+  uint64_t tb, te;
+  l1_tile_range(n, C::TILE, &tb, &te);
+  uint32_t run[C::BPT];  // next free global slot of bins threadIdx.x * BPT + k for this CTA
+  {
+    uint32_t cv[C::BPT];
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + k * kBlock + threadIdx.x;
+    for (int k = 0; k < C::BPT; ++k) cv[k] = counts[threadIdx.x * C::BPT + k];
+    scan_bins<C>(cv, run, tmp);
+#pragma unroll
+    for (int k = 0; k < C::BPT; ++k) {
+      const uint64_t b = threadIdx.x * C::BPT + k;
+      const uint32_t cc = cta_counts[(uint64_t)blockIdx.x * C::BINS + b];
+      run[k] = cc ? run[k] + atomicAdd(cursor + b, cc) : 0u;
+      cta_base[(uint64_t)blockIdx.x * C::BINS + b] = run[k];  // for the staged return
+    }
+  }
+  for (uint64_t tile = tb; tile < te; ++tile) {
+    const uint64_t t0 = tile * C::TILE;
+    uint64_t v[C::PER];
+    uint32_t pk[C::PER];
+#pragma unroll
+    for (int k = 0; k < C::PER; ++k) {
+      const uint64_t e = t0 + k * C::NT + threadIdx.x;
       v[k] = e < n ? __ldg(q + e) : 0;
       pk[k] = e < n ? __ldg(packed + e) : 0;
     }
-    const uint32_t c = tile_counts[tile * kCoarseBins + threadIdx.x];
-    bin_start[threadIdx.x] = block_scan<kBlock>(c, tmp, nullptr);
-    const uint32_t gb = c ? prefix[threadIdx.x] + atomicAdd(cursor + threadIdx.x, c) : 0u;
-    gbase[threadIdx.x] = gb;
-    if (tile_base) tile_base[tile * kCoarseBins + threadIdx.x] = gb;  // for the staged return
+    {
+      uint32_t cv[C::BPT], ex[C::BPT];
+#pragma unroll
+      for (int k = 0; k < C::BPT; ++k) cv[k] = tile_counts[tile * C::BINS + threadIdx.x * C::BPT + k];
+      scan_bins<C>(cv, ex, tmp);
+#pragma unroll
+      for (int k = 0; k < C::BPT; ++k) {
+        bin_start[threadIdx.x * C::BPT + k] = ex[k];
+        gbase[threadIdx.x * C::BPT + k] = run[k];
+        run[k] += cv[k];
+      }
+    }
     __syncthreads();
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + k * kBlock + threadIdx.x;
+    for (int k = 0; k < C::PER; ++k) {
+      const uint64_t e = t0 + k * C::NT + threadIdx.x;
       if (e < n) {
-        const uint32_t d = pk[k] & (kCoarseBins - 1);
-        const uint32_t lp = bin_start[d] + (pk[k] >> kCoarseBits);
+        const uint32_t d = pk[k] & (C::BINS - 1);
+        const uint32_t lp = bin_start[d] + (pk[k] >> C::BITS);
         st_q[lp] = v[k];
-        if (idx) st_i[lp] = (uint32_t)e;
+        if constexpr (kIdx) st_i[lp] = (uint32_t)e;
         if constexpr (!kRecompute) st_d[lp] = (uint8_t)d;
       }
     }
     __syncthreads();
-    const uint32_t tile_n = (uint32_t)std::min<uint64_t>(kCoarseTile, n - t0);
-    for (uint32_t i = threadIdx.x; i < tile_n; i += kBlock) {  // runs written by consecutive lanes
+    const uint32_t tile_n = (uint32_t)std::min<uint64_t>(C::TILE, n - t0);
+    for (uint32_t i = threadIdx.x; i < tile_n; i += C::NT) {  // runs written by consecutive lanes
       const uint64_t x = st_q[i];
       uint32_t dd;
       if constexpr (kRecompute) dd = dg(x);
       else dd = st_d[i];
       const uint32_t dst = gbase[dd] + (i - bin_start[dd]);
       sorted_q[dst] = x;
-      if (idx) idx[dst] = st_i[i];
+      if constexpr (kIdx) idx[dst] = st_i[i];
     }
     __syncthreads();
   }
 }
+template <class C, bool kIdx, bool kRecompute>
+constexpr size_t move_smem() {
+  return (size_t)C::TILE * 8 + 2 * C::BINS * 4 + (kIdx ? C::TILE * 4 : 0) + (kRecompute ? 0 : C::TILE);
+}
 
 // ---- staged return: inverse of the move -------------------------------------------------
-// res1 holds the results in level-1 order. For the tile of original positions [t0, t0+2048)
-// the slots of its (bin, rank) pairs are restaged exactly as in k_psa2_move; slot i of the
-// tile's bin order sits at level-1 position tile_base[d] + (i - bin_start[d]), so res1 is read
-// in runs and out[] written contiguously -- no scattered global access on either side.
-__global__ void __launch_bounds__(kBlock) k_psa2_unmove(const uint32_t* __restrict__ tile_counts,
-                                                        const uint32_t* __restrict__ tile_base,
-                                                        const uint32_t* __restrict__ packed,
-                                                        const uint64_t* __restrict__ res1, uint64_t n,
-                                                        uint64_t* __restrict__ out) {
-  __shared__ uint32_t bin_start[kCoarseBins], gbase[kCoarseBins], tmp[kWarps + 1];
-  __shared__ uint64_t st_r[kCoarseTile];
-  __shared__ uint32_t st_od[kCoarseTile];  // tile offset | bin << 16
-  for (uint64_t tile = blockIdx.x; tile * kCoarseTile < n; tile += gridDim.x) {
-    const uint64_t t0 = tile * kCoarseTile;
-    uint32_t pk[kBatches];
+// res1 holds the results in level-1 order.  For the tile of original positions
+// [t0, t0 + TILE) the slots of its (bin, rank) pairs are restaged exactly as in k_psa2_move;
+// slot i of the tile's bin order sits at level-1 position gbase[d] + (i - bin_start[d]) with
+// gbase rebuilt from the CTA base, so res1 is read in runs and out[] written contiguously --
+// no scattered global access on either side.
+template <class C>
+__global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* __restrict__ tile_counts,
+                                                                const uint32_t* __restrict__ cta_base,
+                                                                const uint32_t* __restrict__ packed,
+                                                                const uint64_t* __restrict__ res1, uint64_t n,
+                                                                uint64_t* __restrict__ out) {
+  extern __shared__ __align__(16) unsigned char l1_smem[];
+  uint64_t* st_r = reinterpret_cast<uint64_t*>(l1_smem);
+  uint32_t* st_od = reinterpret_cast<uint32_t*>(l1_smem + C::TILE * 8);  // offset | bin << TILE_SHIFT
+  uint32_t* bin_start = st_od + C::TILE;
+  uint32_t* gbase = bin_start + C::BINS;
+  __shared__ uint32_t tmp[C::NT / 32 + 1];
+  uint64_t tb, te;
+  l1_tile_range(n, C::TILE, &tb, &te);
+  uint32_t run[C::BPT];
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + k * kBlock + threadIdx.x;
+  for (int k = 0; k < C::BPT; ++k) run[k] = cta_base[(uint64_t)blockIdx.x * C::BINS + threadIdx.x * C::BPT + k];
+  for (uint64_t tile = tb; tile < te; ++tile) {
+    const uint64_t t0 = tile * C::TILE;
+    uint32_t pk[C::PER];
+#pragma unroll
+    for (int k = 0; k < C::PER; ++k) {
+      const uint64_t e = t0 + k * C::NT + threadIdx.x;
       pk[k] = e < n ? __ldg(packed + e) : 0;
     }
-    bin_start[threadIdx.x] = block_scan<kBlock>(tile_counts[tile * kCoarseBins + threadIdx.x], tmp, nullptr);
-    gbase[threadIdx.x] = tile_base[tile * kCoarseBins + threadIdx.x];
-    __syncthreads();
+    {
+      uint32_t cv[C::BPT], ex[C::BPT];
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint64_t e = t0 + k * kBlock + threadIdx.x;
-      if (e < n) {
-        const uint32_t d = pk[k] & (kCoarseBins - 1);
-        const uint32_t lp = bin_start[d] + (pk[k] >> kCoarseBits);
-        st_od[lp] = (uint32_t)(k * kBlock + threadIdx.x) | (d << 16);
+      for (int k = 0; k < C::BPT; ++k) cv[k] = tile_counts[tile * C::BINS + threadIdx.x * C::BPT + k];
+      scan_bins<C>(cv, ex, tmp);
+#pragma unroll
+      for (int k = 0; k < C::BPT; ++k) {
+        bin_start[threadIdx.x * C::BPT + k] = ex[k];
+        gbase[threadIdx.x * C::BPT + k] = run[k];
+        run[k] += cv[k];
       }
     }
     __syncthreads();
-    const uint32_t tile_n = (uint32_t)std::min<uint64_t>(kCoarseTile, n - t0);
-    uint64_t rv[kBatches];
-    uint32_t oo[kBatches];
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {  // all kBatches loads in flight before the stores
-      const uint32_t i = k * kBlock + threadIdx.x;
+    for (int k = 0; k < C::PER; ++k) {
+      const uint64_t e = t0 + k * C::NT + threadIdx.x;
+      if (e < n) {
+        const uint32_t d = pk[k] & (C::BINS - 1);
+        const uint32_t lp = bin_start[d] + (pk[k] >> C::BITS);
+        st_od[lp] = (uint32_t)(k * C::NT + threadIdx.x) | (d << C::TILE_SHIFT);
+      }
+    }
+    __syncthreads();
+    const uint32_t tile_n = (uint32_t)std::min<uint64_t>(C::TILE, n - t0);
+    uint64_t rv[C::PER];
+    uint32_t oo[C::PER];
+#pragma unroll
+    for (int k = 0; k < C::PER; ++k) {  // all loads in flight before the stores
+      const uint32_t i = k * C::NT + threadIdx.x;
       if (i < tile_n) {
-        const uint32_t od = st_od[i], dd = od >> 16;
-        oo[k] = od & 0xFFFFu;
+        const uint32_t od = st_od[i], dd = od >> C::TILE_SHIFT;
+        oo[k] = od & (C::TILE - 1);
         rv[k] = __ldg(res1 + gbase[dd] + (i - bin_start[dd]));
       }
     }
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k)
-      if (k * kBlock + threadIdx.x < tile_n) st_r[oo[k]] = rv[k];
+    for (int k = 0; k < C::PER; ++k)
+      if (k * C::NT + threadIdx.x < tile_n) st_r[oo[k]] = rv[k];
     __syncthreads();
-    for (uint32_t i = threadIdx.x; i < tile_n; i += kBlock) out[t0 + i] = st_r[i];
+    for (uint32_t i = threadIdx.x; i < tile_n; i += C::NT) out[t0 + i] = st_r[i];
     __syncthreads();
   }
+}
+template <class C>
+constexpr size_t unmove_smem() {
+  return (size_t)C::TILE * 12 + 2 * C::BINS * 4;
 }
 
 // ---- level 2: chunk-local sort by the N-bit bucket (two stable LSD passes) ---------------
@@ -423,32 +486,73 @@ constexpr int kLocalBins = 1 << kLocalBits;
 constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12;
 #include "psa2_count_sort.inc"
 
-// level-1 partition by any <= 256-bin digit: rank pass, then the staged move.
+// level-1 grid: persistent CTAs, ~2048 resident threads per SM, at most one CTA per tile
+template <class C>
+int l1_grid(uint64_t n, int sm) {
+#ifndef HM_L1_WAVES
+#define HM_L1_WAVES 8
+#endif
+  const uint64_t g = std::min<uint64_t>((uint64_t)sm * (2048 / C::NT) * HM_L1_WAVES, kL1CtaRows / C::BINS);
+  return (int)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(n, C::TILE), g));
+}
+
+// level-1 partition by a C::BITS-bit digit: rank pass, then the staged move.
 // h_counts (optional) receives the first `nbins` bin counts synchronously.
-template <class Digit>
+template <class C, class Digit>
 harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg, const PsaWs& ws,
                                  uint64_t* sorted_q, uint32_t* idx, int sm, cudaStream_t st, uint64_t* h_counts,
-                                 uint32_t nbins, uint32_t* tile_base = nullptr) {
-  HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * kCoarseBins * 4, st));
-  // one tile per CTA (measured faster than persistent grid-stride CTAs: the phases of
-  // different CTAs overlap)
-  const int g = (int)std::min<uint64_t>(ceil_div(n, kCoarseTile), 1u << 30);
+                                 uint32_t nbins) {
+  constexpr bool kRecompute = std::is_same<Digit, CoarseDigit>::value;
+  HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * C::BINS * 4, st));
+  const int g = l1_grid<C>(n, sm);
   {
     ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
-    k_psa2_rank<Digit><<<std::max(g, 1), kBlock, 0, st>>>(q, n, dg, ws.counts, ws.tile_counts, ws.packed);
+    k_psa2_rank<Digit, C><<<g, C::NT, 0, st>>>(q, n, dg, ws.counts, ws.tile_counts, ws.packed, ws.cta_counts);
   }
   HM_LAUNCHED();
   if (h_counts) {
-    uint32_t tmp[kCoarseBins];
+    uint32_t tmp[C::BINS];
     HM_CUDA(cudaMemcpyAsync(tmp, ws.counts, nbins * 4, cudaMemcpyDeviceToHost, st));
     HM_CUDA(cudaStreamSynchronize(st));
     for (uint32_t b = 0; b < nbins; ++b) h_counts[b] = tmp[b];
   }
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
-        k_psa2_move<Digit><<<std::max(g, 1), kBlock, 0, st>>>(q, n, dg, ws.counts, ws.counts + kCoarseBins, ws.tile_counts,
-                                                   ws.packed, sorted_q, idx, tile_base);
+    if (idx) {
+      constexpr size_t smb = move_smem<C, true, kRecompute>();
+      static bool cfg = false;
+      if (!cfg) {
+        HM_CUDA(cudaFuncSetAttribute(k_psa2_move<Digit, C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
+        cfg = true;
+      }
+      k_psa2_move<Digit, C, true><<<g, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
+                                                         ws.packed, ws.cta_counts, ws.cta_base, sorted_q, idx);
+    } else {
+      constexpr size_t smb = move_smem<C, false, kRecompute>();
+      static bool cfg = false;
+      if (!cfg) {
+        HM_CUDA(cudaFuncSetAttribute(k_psa2_move<Digit, C, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
+        cfg = true;
+      }
+      k_psa2_move<Digit, C, false><<<g, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
+                                                          ws.packed, ws.cta_counts, ws.cta_base, sorted_q, nullptr);
+    }
   }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+template <class C>
+harmonia_status unpartition(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
+                            cudaStream_t st) {
+  constexpr size_t smb = unmove_smem<C>();
+  static bool cfg = false;
+  if (!cfg) {
+    HM_CUDA(cudaFuncSetAttribute(k_psa2_unmove<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
+    cfg = true;
+  }
+  ProfScope ps_(HARMONIA_PROF_RETURN, st);
+  k_psa2_unmove<C><<<l1_grid<C>(n, sm), C::NT, smb, st>>>(ws.tile_counts, ws.cta_base, ws.packed, res1, n, out);
   HM_LAUNCHED();
   return HARMONIA_OK;
 }
@@ -458,18 +562,24 @@ harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg,
 // multi-GPU router: destination-major grouping by splitters (P <= 256 shards)
 harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
                                  int sm, cudaStream_t st, uint64_t* h_counts) {
-  if (P > (uint32_t)kCoarseBins) return HARMONIA_ERR_INVALID_ARG;
-  return coarse_partition(q, n, f, ws, ws.sorted_q, ws.idx, sm, st, h_counts, P);
+  if (P > (uint32_t)Narrow::BINS) return HARMONIA_ERR_INVALID_ARG;
+  return coarse_partition<Narrow>(q, n, f, ws, ws.sorted_q, ws.idx, sm, st, h_counts, P);
 }
 
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
-                               cudaStream_t st, int level2, bool local) {
-  const uint32_t b1 = (uint32_t)std::min(nb, kCoarseBits);
-  const uint32_t shift1 = (uint32_t)nb - b1;
-  harmonia_status s = coarse_partition(q, n, CoarseDigit{f, shift1}, ws, ws.sorted_q, local ? nullptr : ws.idx, sm,
-                                       st, nullptr, 0, local ? ws.tile_base : nullptr);
+                               cudaStream_t st, int level2, bool local, bool wide) {
+  harmonia_status s;
+  if (wide) {  // staged-return mode only (no idx)
+    const uint32_t b1 = (uint32_t)std::min(nb, Wide::BITS);
+    s = coarse_partition<Wide>(q, n, CoarseDigit{f, (uint32_t)nb - b1}, ws, ws.sorted_q, nullptr, sm, st, nullptr,
+                               0);
+  } else {
+    const uint32_t b1 = (uint32_t)std::min(nb, Narrow::BITS);
+    s = coarse_partition<Narrow>(q, n, CoarseDigit{f, (uint32_t)nb - b1}, ws, ws.sorted_q, local ? nullptr : ws.idx,
+                                 sm, st, nullptr, 0);
+  }
   if (s != HARMONIA_OK) return s;
-  if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation)
+  if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation / fused chunk sort)
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);  // reported in the "scan" class: level-2 sort
     static bool configured = false;
@@ -493,15 +603,10 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
   return HARMONIA_OK;
 }
 
-harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, cudaStream_t st) {
+harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
+                                 cudaStream_t st, bool wide) {
   if (n == 0) return HARMONIA_OK;
-  {
-    ProfScope ps_(HARMONIA_PROF_RETURN, st);
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kCoarseTile), 1u << 30);
-    k_psa2_unmove<<<g, kBlock, 0, st>>>(ws.tile_counts, ws.tile_base, ws.packed, res1, n, out);
-  }
-  HM_LAUNCHED();
-  return HARMONIA_OK;
+  return wide ? unpartition<Wide>(ws, res1, n, out, sm, st) : unpartition<Narrow>(ws, res1, n, out, sm, st);
 }
 
 }  // namespace hm

@@ -133,7 +133,8 @@ def test_lane_search_queries_per_lane(hm, orc, F, lane_queries):
     exp = orc.sorted_search(keys, vals, q)
     for kw in ({}, {"psa_bits": -1}, {"window": 3072}, {"smem_levels": -1}, {"flags": hm.QF_FUSE_SORT},
                {"flags": hm.QF_FUSE_SORT, "window": 5120, "smem_levels": 1}, {"flags": hm.QF_SCATTER_RETURN},
-               {"flags": hm.QF_SCATTER_RETURN, "window": 7168}, {"window": 7168, "smem_levels": -1}):
+               {"flags": hm.QF_SCATTER_RETURN, "window": 7168}, {"window": 7168, "smem_levels": -1},
+               {"flags": hm.QF_PSA_WIDE}, {"flags": hm.QF_PSA_WIDE, "window": 13312}):
         got = host(t.search(cu(q), group_size=1, lane_queries=lane_queries, **kw))
         assert np.array_equal(got, exp), kw
 

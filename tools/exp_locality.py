@@ -14,7 +14,6 @@ keys = gen.uniform_keys_t(T, "cuda")
 t = hm.Tree(keys.view(torch.uint64), gen.values_for_t(keys).view(torch.uint64), fanout=64)
 q = gen.uniform_queries_t(keys, Q)
 qs = torch.sort(q)[0]  # int64 view: keys < 2^63 here, so signed order = unsigned order
-qsw = qs.view(8, -1).t().contiguous().view(-1)  # 8 interleaved sorted runs per window... (see below)
 cases = {"random": (q, {}), "sorted": (qs, {}), "coarse_only": (q, {"flags": hm.QF_PSA_COARSE}),
          "scatter_return": (q, {"flags": hm.QF_SCATTER_RETURN})}
 for name, (qq, kw) in cases.items():
