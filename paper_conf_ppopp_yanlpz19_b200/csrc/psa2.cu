@@ -591,7 +591,10 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
                                    (int)kCountSortSmem));
       configured = true;
     }
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kChunk), (uint64_t)sm * 4);
+#ifndef HM_SORT_CTAS_PER_SM
+#define HM_SORT_CTAS_PER_SM 4
+#endif
+    const int g = (int)std::min<uint64_t>(ceil_div(n, kChunk), (uint64_t)sm * HM_SORT_CTAS_PER_SM);
     if (level2 == 1)  // two stable LSD passes of ballot multisplit (ablation)
       k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
     else if (local)   // one counting pass with shared-memory atomics (default, measured faster)
