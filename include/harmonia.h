@@ -91,6 +91,10 @@ typedef struct {
 #define HARMONIA_QF_PSA_WIDE 512u /* staged return with an 11-bit (2048-bin) level-1 partition
                                       instead of the default 8-bit one (ablation: denser
                                       chunks for the search, but 2-query runs in the moves)  */
+#define HARMONIA_QF_PER_LANE 1024u /* G = 1 PSA path: every lane descends on its own instead of
+                                      the default warp-shared descent (the warp's PSA-ordered
+                                      queries share the path down to the level where their
+                                      key interval splits)                           */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic
@@ -226,7 +230,8 @@ typedef struct {
   uint32_t smem_bytes, smem_nodes;
   uint32_t staged_return;  /* 1: results return through the chunk-local stage + inverse move */
   uint32_t lane_queries;   /* G = 1: queries interleaved per lane */
-  uint64_t reserved;
+  uint32_t warp_shared;    /* 1: G = 1 warp-shared descent (see HARMONIA_QF_PER_LANE) */
+  uint32_t reserved;
 } harmonia_plan;
 harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
                                     const harmonia_query_opts* opts, harmonia_plan* out);

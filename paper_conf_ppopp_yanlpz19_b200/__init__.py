@@ -29,6 +29,7 @@ QF_PSA_LSD = 64
 QF_FUSE_SORT = 128
 QF_SCATTER_RETURN = 256
 QF_PSA_WIDE = 512
+QF_PER_LANE = 1024
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
            6: "DEVICE_MISMATCH", 7: "TOO_LARGE"}
 
@@ -57,7 +58,7 @@ class PlanInfo(C.Structure):
     _fields_ = [("group_size", C.c_int32), ("psa_bits", C.c_int32), ("smem_levels", C.c_int32),
                 ("ps_in_smem", C.c_int32), ("window", C.c_uint64), ("smem_bytes", C.c_uint32),
                 ("smem_nodes", C.c_uint32), ("staged_return", C.c_uint32), ("lane_queries", C.c_uint32),
-                ("reserved", C.c_uint64)]
+                ("warp_shared", C.c_uint32), ("reserved", C.c_uint32)]
 
 
 class Info(C.Structure):

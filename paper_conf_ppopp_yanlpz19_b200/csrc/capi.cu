@@ -87,6 +87,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
           !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
           2 * (round_up(P.smem_bytes, 16) + kPsaChunk * 8 + 1024) <= t->smem_per_sm;
   P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
+  P.coop = P.ret && !(o->flags & HARMONIA_QF_PER_LANE);
   *p = P;
   return HARMONIA_OK;
 }
@@ -101,6 +102,11 @@ static SearchArgs search_args(const harmonia_tree* t, const Plan& p) {
   a.smem_levels = (uint32_t)p.smem_levels;
   a.smem_nodes = p.smem_nodes;
   a.ps_smem_bytes = p.ps_smem ? p.ps_smem_bytes : 0;
+  a.coop = p.coop ? 1u : 0u;
+  a.kmin = t->min_key;
+  a.kmax = t->max_key;
+  const uint32_t span = t->min_key < t->max_key ? 64 - __builtin_clzll(t->min_key ^ t->max_key) : 0;
+  a.cshift = span > 32 ? span - 32 : 0;
   return a;
 }
 
@@ -223,6 +229,7 @@ extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t 
   out->smem_nodes = p.smem_nodes;
   out->staged_return = p.ret ? 1u : 0u;
   out->lane_queries = p.G == 1 ? (uint32_t)p.lane_ilp : 0u;
+  out->warp_shared = p.coop ? 1u : 0u;
   return HARMONIA_OK;
 }
 

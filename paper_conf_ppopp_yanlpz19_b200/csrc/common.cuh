@@ -134,6 +134,7 @@ struct Plan {
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
   bool ret = false;          // staged inverse return (chunk-local result staging + unmove)
   bool wide = false;         // staged return with the 11-bit level-1 partition
+  bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
 };
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
@@ -191,6 +192,11 @@ struct SearchArgs {
                            // go through shared memory (at dynamic-smem offset res_smem_off)
                            // to out[] in level-1 order, chunk by chunk (kPsaChunk)
   uint32_t res_smem_off;
+  // warp-shared descent (G = 1 PSA path): clamp(q) -> (clamp(q) - kmin) >> cshift is a
+  // monotone 32-bit image of the key, so two 32-bit warp reductions bound the warp's queries
+  uint32_t coop;
+  uint32_t cshift;
+  uint64_t kmin, kmax;
 };
 harmonia_status launch_sort_search(const harmonia_tree* t, const struct Plan& p, const SearchArgs& a,
                                    cudaStream_t st);

@@ -442,79 +442,210 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
 // search is latency-bound (few instructions, few wavefronts), so U chains per thread raise
 // the memory-level parallelism without adding work.  A warp takes 32*U consecutive
 // (PSA-ordered) queries: query (u, lane) = base + u*32 + lane.
-// one lane, U interleaved queries: descent (Eq 1) + leaf probe + result write
+// one lane, U interleaved queries, from level l0 at nodes node[]: descent (Eq 1) + leaf probe
+template <int F, int U>
+__device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
+                                             bool ps_smem, bool leaf_smem, uint32_t l0, uint32_t (&node)[U],
+                                             const uint64_t (&q)[U], const bool (&live)[U], uint64_t (&res)[U]) {
+  for (uint32_t l = l0; l + 1 < a.h; ++l) {
+    uint32_t first[U], r[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      first[u] = ps_smem ? s_ps[node[u]] : __ldg(a.ps + node[u]);  // PS[node_idx]
+      r[u] = 0;
+    }
+    if (l < a.smem_levels) {
+#pragma unroll
+      for (int s = F / 2; s >= 1; s >>= 1) {
+        uint64_t k[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) k[u] = s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)];
+#pragma unroll
+        for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+      }
+    } else {
+#pragma unroll
+      for (int s = F / 2; s >= 1; s >>= 1) {
+        uint64_t k[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+#pragma unroll
+        for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) node[u] = first[u] + r[u];  // Eq 1
+  }
+  // leaf: r = #keys <= q; the last key that compared <= q is key[r-1] (the successful
+  // steps of the power-of-two search visit increasing slots), so the probe needs no reload
+  uint32_t r[U];
+  uint64_t best[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    r[u] = 0;
+    best[u] = 0;
+  }
+#pragma unroll
+  for (int s = F / 2; s >= 1; s >>= 1) {
+    uint64_t k[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      k[u] = leaf_smem ? s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)]
+                       : ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool le = k[u] <= q[u];
+      r[u] += le ? s : 0;
+      best[u] = le ? k[u] : best[u];
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    res[u] = kNotFound;
+    if (live[u] && r[u] > 0 && best[u] == q[u])
+      res[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+  }
+}
+
 template <int F, int U>
 __device__ __forceinline__ void lane_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                           bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
                                           const bool (&act)[U], uint64_t (&res)[U]) {
-  {
-    uint64_t q[U];
-    uint32_t node[U];
-    bool live[U];
+  uint64_t q[U];
+  uint32_t node[U];
+  bool live[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    live[u] = act[u] && q0[u] != kPad;  // PAD is never a key (C-A2)
+    q[u] = live[u] ? q0[u] : 0;
+    node[u] = 0;
+  }
+  lane_descend<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, 0, node, q, live, res);
+}
+
+// ---- warp-shared descent (G = 1, PSA-ordered queries) -------------------------------------
+// After PSA a warp's 32*U queries lie in a narrow key interval [qlo, qhi] (sorted
+// neighbours walk the same path).  The warp bounds it with two 32-bit reductions of the
+// monotone image (clamp(q) - kmin) >> cshift, then ranks qlo and qhi in each node with one
+// cooperative 128-bit load per lane and four ballots: while both ranks agree, every query of
+// the warp takes the same child (clamp preserves the path: every separator lies in
+// (kmin, kmax]), so the level costs one load instruction for the whole warp instead of
+// log2(F) per query.  Where they differ, each lane's rank lies in [rank(qlo), rank(qhi)], so
+// the lane searches only that window, then goes on alone.  At the leaf the window is
+// [#keys < qlo, #keys <= qhi]: a key equal to q can only lie inside it.
+
+// ranks of qlo and qhi in node nk: #keys (< or <=) qlo and #keys <= qhi, warp-cooperatively
+template <int F, bool SMEM, bool STRICT_LO>
+__device__ __forceinline__ void coop_rank(const uint64_t* nk, uint64_t qlo, uint64_t qhi, uint32_t& rlo,
+                                          uint32_t& rhi) {
+  const unsigned lane = threadIdx.x & 31;
+  constexpr int NP = F >= 64 ? F / 64 : 1;  // 128-bit loads per lane
+  rlo = 0;
+  rhi = 0;
+#pragma unroll
+  for (int p = 0; p < NP; ++p) {
+    const uint32_t slot = p * 64 + 2 * lane;
+    ulonglong2 k = make_ulonglong2(kPad, kPad);  // PAD > every bound
+    if (F >= 64 || slot < F) k = ld_pair<SMEM>(nk + slot);
+    const bool lx = STRICT_LO ? k.x < qlo : k.x <= qlo, ly = STRICT_LO ? k.y < qlo : k.y <= qlo;
+    rlo += __popc(ballot(lx)) + __popc(ballot(ly));
+    rhi += __popc(ballot(k.x <= qhi)) + __popc(ballot(k.y <= qhi));
+  }
+}
+
+// per-lane rank inside the warp-uniform window [rlo, rhi]: keys below rlo are <= q, keys from
+// rhi on are > q; binary lifting over the rhi - rlo undecided slots (warp-uniform trip count).
+// best = the last key that compared <= q (valid when r > rlo).
+template <int F, int U, bool SMEM>
+__device__ __forceinline__ void window_rank(const uint64_t* base, const uint64_t (&nodeoff)[U], const uint64_t (&q)[U],
+                                            uint32_t rlo, uint32_t rhi, uint32_t (&r)[U], uint64_t (&best)[U]) {
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    r[u] = rlo;
+    best[u] = 0;
+  }
+  const uint32_t w = rhi - rlo;
+  if (w == 0) return;
+  for (uint32_t s = 1u << (31 - __clz(w)); s >= 1; s >>= 1) {
+    uint64_t k[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      live[u] = act[u] && q0[u] != kPad;  // PAD is never a key (C-A2)
-      q[u] = live[u] ? q0[u] : 0;
-      node[u] = 0;
-    }
-    for (uint32_t l = 0; l + 1 < a.h; ++l) {
-      uint32_t first[U], r[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        first[u] = ps_smem ? s_ps[node[u]] : __ldg(a.ps + node[u]);  // PS[node_idx]
-        r[u] = 0;
-      }
-      if (l < a.smem_levels) {
-#pragma unroll
-        for (int s = F / 2; s >= 1; s >>= 1) {
-          uint64_t k[U];
-#pragma unroll
-          for (int u = 0; u < U; ++u) k[u] = s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)];
-#pragma unroll
-          for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
-        }
-      } else {
-#pragma unroll
-        for (int s = F / 2; s >= 1; s >>= 1) {
-          uint64_t k[U];
-#pragma unroll
-          for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
-#pragma unroll
-          for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u) node[u] = first[u] + r[u];  // Eq 1
-    }
-    // leaf: r = #keys <= q; the last key that compared <= q is key[r-1] (the successful
-    // steps of the power-of-two search visit increasing slots), so the probe needs no reload
-    uint32_t r[U];
-    uint64_t best[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      r[u] = 0;
-      best[u] = 0;
-    }
-#pragma unroll
-    for (int s = F / 2; s >= 1; s >>= 1) {
-      uint64_t k[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-        k[u] = leaf_smem ? s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)]
-                         : ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const bool le = k[u] <= q[u];
-        r[u] += le ? s : 0;
-        best[u] = le ? k[u] : best[u];
-      }
+      const bool in = r[u] + s <= rhi;
+      const uint64_t* p = base + nodeoff[u] + (in ? r[u] + s - 1 : 0);
+      k[u] = in ? ld_key<SMEM>(p) : kPad;
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      res[u] = kNotFound;
-      if (live[u] && r[u] > 0 && best[u] == q[u])
-        res[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+      const bool le = k[u] <= q[u];
+      r[u] += le ? s : 0;
+      best[u] = le ? k[u] : best[u];
     }
+  }
+}
+
+template <int F, int U>
+__device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
+                                          bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
+                                          const bool (&act)[U], uint64_t (&res)[U]) {
+  uint64_t q[U];
+  bool live[U];
+  uint32_t tmin = 0xFFFFFFFFu, tmax = 0;
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    live[u] = act[u] && q0[u] != kPad;  // PAD is never a key (C-A2)
+    q[u] = live[u] ? q0[u] : 0;
+    const uint64_t c = q0[u] < a.kmin ? a.kmin : (q0[u] > a.kmax ? a.kmax : q0[u]);
+    const uint32_t t = (uint32_t)((c - a.kmin) >> a.cshift);
+    tmin = live[u] ? min(tmin, t) : tmin;
+    tmax = live[u] ? max(tmax, t) : tmax;
+  }
+  tmin = __reduce_min_sync(kFull, tmin);
+  tmax = __reduce_max_sync(kFull, tmax);
+  if (tmin > tmax) {  // no live query in this warp
+#pragma unroll
+    for (int u = 0; u < U; ++u) res[u] = kNotFound;
+    return;
+  }
+  const uint64_t qlo = a.kmin + ((uint64_t)tmin << a.cshift);
+  const uint64_t d = (uint64_t)tmax << a.cshift, m = (1ull << a.cshift) - 1;
+  const uint64_t qhi = (a.kmax - a.kmin - d <= m) ? a.kmax : a.kmin + d + m;
+  uint32_t node = 0, l = 0;
+  for (; l + 1 < a.h; ++l) {
+    const uint32_t first = ps_smem ? s_ps[node] : __ldg(a.ps + node);  // PS[node_idx]
+    uint32_t rlo, rhi;
+    if (l < a.smem_levels) coop_rank<F, true, false>(s_keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
+    else coop_rank<F, false, false>(a.keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
+    if (rlo == rhi) {
+      node = first + rlo;  // Eq 1, the same child for the whole warp
+      continue;
+    }
+    // the warp's interval splits here: per-lane window search, then per-lane descent
+    uint32_t r[U], nd[U];
+    uint64_t off[U], best[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) off[u] = (uint64_t)node * F;
+    if (l < a.smem_levels) window_rank<F, U, true>(s_keys, off, q, rlo, rhi, r, best);
+    else window_rank<F, U, false>(a.keys, off, q, rlo, rhi, r, best);
+#pragma unroll
+    for (int u = 0; u < U; ++u) nd[u] = first + r[u];
+    lane_descend<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, l + 1, nd, q, live, res);
+    return;
+  }
+  // the whole warp reached the same leaf
+  uint32_t rlo, rhi;
+  if (leaf_smem) coop_rank<F, true, true>(s_keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
+  else coop_rank<F, false, true>(a.keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
+  uint32_t r[U];
+  uint64_t off[U], best[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) off[u] = (uint64_t)node * F;
+  if (leaf_smem) window_rank<F, U, true>(s_keys, off, q, rlo, rhi, r, best);
+  else window_rank<F, U, false>(a.keys, off, q, rlo, rhi, r, best);
+  const uint64_t* vrow = a.vals + (uint64_t)(node - a.leaf_start) * F;
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    res[u] = kNotFound;
+    if (live[u] && r[u] > rlo && best[u] == q[u]) res[u] = __ldg(vrow + (r[u] - 1));
   }
 }
 
@@ -553,7 +684,7 @@ __global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const 
 // back to level-1 order in shared memory and written contiguously -- the scattered 8-byte
 // stores to out[original position] (measured: a third of the kernel) are replaced by
 // k_psa2_unmove's run-wise copy.
-template <int F, int U>
+template <int F, int U, bool COOP>
 __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
@@ -578,7 +709,8 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
         o[u] = act[u] ? ld_stream32(a.idx + c0 + j) : 0u;
       }
       uint64_t res[U];
-      lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      else lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (act[u]) s_res[o[u]] = res[u];
@@ -850,10 +982,11 @@ harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, cons
 template <int F>
 harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
   const int U = p.lane_ilp;
-  auto kern = U >= 4 ? k_lane_search_c<F, 4> : (U == 2 ? k_lane_search_c<F, 2> : k_lane_search_c<F, 1>);
+  auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
+                     : (U >= 4 ? k_lane_search_c<F, 4, false> : (U == 2 ? k_lane_search_c<F, 2, false> : k_lane_search_c<F, 1, false>));
   const uint32_t smem = a.res_smem_off + kPsaChunk * 8;
-  static int configured_smem[5] = {-1, -1, -1, -1, -1};
-  const int ci = U >= 4 ? 4 : U;
+  static int configured_smem[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
+  const int ci = (U >= 4 ? 4 : U) + (a.coop ? 5 : 0);
   if ((int)smem > configured_smem[ci]) {
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     configured_smem[ci] = (int)smem;

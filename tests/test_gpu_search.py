@@ -134,9 +134,40 @@ def test_lane_search_queries_per_lane(hm, orc, F, lane_queries):
     for kw in ({}, {"psa_bits": -1}, {"window": 3072}, {"smem_levels": -1}, {"flags": hm.QF_FUSE_SORT},
                {"flags": hm.QF_FUSE_SORT, "window": 5120, "smem_levels": 1}, {"flags": hm.QF_SCATTER_RETURN},
                {"flags": hm.QF_SCATTER_RETURN, "window": 7168}, {"window": 7168, "smem_levels": -1},
-               {"flags": hm.QF_PSA_WIDE}, {"flags": hm.QF_PSA_WIDE, "window": 13312}):
+               {"flags": hm.QF_PSA_WIDE}, {"flags": hm.QF_PSA_WIDE, "window": 13312},
+               {"flags": hm.QF_PER_LANE}, {"flags": hm.QF_PER_LANE, "window": 7168, "smem_levels": -1}):
         got = host(t.search(cu(q), group_size=1, lane_queries=lane_queries, **kw))
         assert np.array_equal(got, exp), kw
+
+
+@pytest.mark.parametrize("F", [4, 16, 64, 128])
+@pytest.mark.parametrize("keyset", ["dense", "top", "clustered", "wide"])
+def test_warp_shared_descent(hm, orc, F, keyset):
+    """The default G = 1 PSA path descends warp by warp while the warp's query interval stays
+    inside one child (search.cu warp_core).  Cases aimed at its bounds: every query in one
+    leaf, intervals straddling leaf and parent boundaries, queries below min / above max key
+    in the same warp as hits, keys at the top of the 64-bit space (qhi saturation), a dense
+    key set (cshift = 0) and a 64-bit-wide span (cshift = 32)."""
+    n = 20000
+    keys = {"dense": np.arange(n, dtype=np.uint64) + np.uint64(5),
+            "top": np.uint64(MAX - 1) - np.arange(n, dtype=np.uint64)[::-1] * np.uint64(3),
+            "clustered": gen.clustered_keys(n), "wide": gen.uniform_keys(n)}[keyset]
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F)
+    rng = np.random.default_rng(F)
+    parts = [np.full(5000, keys[n // 2]),                          # one key, every lane
+             keys[rng.integers(100, 140, 30000)],                   # a few neighbouring leaves
+             np.repeat(keys[::F - 1], 3),                           # leaf boundaries
+             np.concatenate([keys[:200], np.zeros(50, np.uint64), keys[-200:],
+                             np.full(50, MAX - 1, np.uint64), np.full(50, MAX, np.uint64)]),
+             keys[:3000] + np.uint64(1), keys[-3000:] - np.uint64(1),
+             gen.uniform_queries(keys, 40000, miss_frac=0.3)]
+    q = np.concatenate(parts)
+    exp = orc.sorted_search(keys, vals, q)
+    for kw in ({}, {"window": 5120}, {"smem_levels": -1}, {"smem_levels": 1}, {"lane_queries": 1},
+               {"lane_queries": 4}, {"flags": hm.QF_PER_LANE}):
+        assert np.array_equal(host(t.search(cu(q), group_size=1, **kw)), exp), kw
+    assert t.plan(len(q))["warp_shared"] == 1 and t.plan(len(q), flags=hm.QF_PER_LANE)["warp_shared"] == 0
 
 
 @pytest.mark.parametrize("F,G", FG)
