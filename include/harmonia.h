@@ -236,6 +236,35 @@ typedef struct {
 harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
                                     const harmonia_query_opts* opts, harmonia_plan* out);
 
+/* ---------------------------------------------------------------------------------------
+ * NTG static profiling (§4.2): the paper's model for the thread-group size.
+ *
+ * harmonia_ntg_choose — host-only arithmetic (no GPU needed).
+ *   prof[n][h][2]: per sample query j and level l, prof[j][l][0] = r = keys of the node on
+ *     j's path before the target (<= q in internal nodes, < q at the leaf) and
+ *     prof[j][l][1] = cnt = valid keys in that node.  bucket[n] (may be NULL = identity):
+ *     PSA bucket per sample; the samples are taken in stable bucket order.
+ *   Fig 9 steps (C-A13): min(r/(GS*kpl)+1, ceil(cnt/(GS*kpl))).  Eq 3: S(GS) = mean over
+ *   warps of 32/GS consecutive samples of the per-level max steps summed over levels
+ *   [lev0, h).  Eq 4 (C-A22): starting at gs0, halve GS while 2*S(GS)/S(GS/2) > 1, GS >= 2
+ *   (C-A14).  *gs_out = the chosen GS; steps_out[6] (may be NULL) = S(1), S(2), ..., S(32)
+ *   (0 for GS > gs0).  INVALID_ARG on null prof/gs_out, n == 0, h == 0, kpl == 0 or gs0 not a
+ *   power of two in [1, 32].
+ *
+ * harmonia_tune_group_size — the same model on a device sample: one profiling kernel (a plain
+ *   Eq-1 descent per sample on the legacy default stream), a synchronous copy of the n*h*2
+ *   counters, then harmonia_ntg_choose with gs0 = min(32, F/2), kpl = 2 (128-bit loads),
+ *   lev0 = the shared-memory-staged levels of the plan `opts` selects and the plan's PSA
+ *   bucket.  d_samples: n <= 2^20 device queries.  Offline (allocates a temporary device
+ *   buffer); the result is advice for harmonia_query_opts.group_size, which stays 0 = the
+ *   measured auto choice unless the caller passes it.
+ * --------------------------------------------------------------------------------------- */
+harmonia_status harmonia_ntg_choose(const uint32_t* prof, const uint32_t* bucket, uint32_t n, uint32_t h,
+                                    uint32_t lev0, uint32_t gs0, uint32_t kpl, int32_t* gs_out,
+                                    double* steps_out);
+harmonia_status harmonia_tune_group_size(const harmonia_tree* tree, const uint64_t* d_samples, uint32_t n,
+                                         const harmonia_query_opts* opts, int32_t* gs_out, double* steps_out);
+
 /* Eq 2 as used by psa_bits = 0: ceil(log2(T/K)) clamped to [0, 28], K = 16. */
 int32_t harmonia_psa_bits_auto(uint64_t n_keys);
 

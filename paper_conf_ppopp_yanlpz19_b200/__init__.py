@@ -102,6 +102,10 @@ def lib():
             "harmonia_route_partition": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _vp, _vp, _sz, _vp]),
             "harmonia_scatter_results": (C.c_int, [_vp, _vp, _u64, _vp, _vp]),
             "harmonia_psa_bits_auto": (C.c_int32, [_u64]),
+            "harmonia_ntg_choose": (C.c_int, [_vp, _vp, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
+                                              C.c_uint32, C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
+            "harmonia_tune_group_size": (C.c_int, [_vp, _vp, C.c_uint32, C.POINTER(QueryOpts),
+                                                   C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
             "harmonia_query_plan": (C.c_int, [_vp, _u64, C.POINTER(QueryOpts), C.POINTER(PlanInfo)]),
             "harmonia_profile_enable": (None, [C.c_int]),
             "harmonia_profile_read": (C.c_int, [C.POINTER(C.c_double), C.POINTER(_u64)]),
@@ -116,6 +120,18 @@ def lib():
             f.argtypes = args
         _lib = L
     return _lib
+
+
+def ntg_choose(prof, bucket, h: int, lev0: int, gs0: int, kpl: int = 2):
+    """NTG model (Eq 3/4) over host profile counters: prof uint32[n, h, 2] of
+    (r, cnt) per sample and level, bucket uint32[n] or None.  Returns (GS, [S(1), ..., S(32)])."""
+    prof = np.ascontiguousarray(prof, dtype=np.uint32)
+    n = prof.shape[0]
+    b = None if bucket is None else np.ascontiguousarray(bucket, dtype=np.uint32)
+    gs, st = C.c_int32(0), (C.c_double * 6)()
+    _check(lib().harmonia_ntg_choose(prof.ctypes.data, None if b is None else b.ctypes.data, n, h, lev0, gs0, kpl,
+                                     C.byref(gs), st), "harmonia_ntg_choose")
+    return int(gs.value), [float(x) for x in st]
 
 
 def _check(status: int, what: str):
@@ -226,6 +242,16 @@ class Tree:
         d = {f: getattr(inf, f) for f, _ in Info._fields_ if f not in ("level_start", "reserved")}
         d["level_start"] = [int(inf.level_start[i]) for i in range(inf.height + 1)]
         return d
+
+    def tune_group_size(self, samples, opts: QueryOpts | None = None, **kw):
+        """NTG static profiling on a device sample of queries (~1000): the paper's
+        Eq 3/4 group size and the per-size warp step counts S(1..32).  Offline, synchronous."""
+        o = opts if opts is not None else make_opts(**kw)
+        gs, st = C.c_int32(0), (C.c_double * 6)()
+        samples = samples.contiguous()
+        _check(lib().harmonia_tune_group_size(self._h, samples.data_ptr(), samples.numel(), C.byref(o), C.byref(gs), st),
+               "harmonia_tune_group_size")
+        return int(gs.value), [float(x) for x in st]
 
     def plan(self, n: int, opts: QueryOpts | None = None, **kw) -> dict:
         o = opts if opts is not None else make_opts(**kw)
