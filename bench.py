@@ -60,7 +60,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
-    ap.add_argument("--mode", default="replicated", choices=["replicated", "partitioned"])
+    ap.add_argument("--mode", default="replicated", choices=["replicated", "partitioned", "peer"])
     ap.add_argument("--sweep", default="", help="comma list of k=v option sets separated by ';' (diagnostics)")
     return ap.parse_args()
 
@@ -259,7 +259,7 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     pg = None
-    if world > 1 or a.mode == "partitioned":
+    if world > 1 or a.mode in ("partitioned", "peer"):
         import torch.distributed as dist
 
         dist.init_process_group("nccl", device_id=dev)
@@ -277,14 +277,15 @@ def main():
     vals = gen.values_for(keys)
     opts = hm.make_opts(a.group_size, a.psa_bits, a.smem_levels, a.window, a.flags)
     pt = None
-    if a.mode == "partitioned":
-        from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree, key_splitters
+    if a.mode in ("partitioned", "peer"):
+        from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree, PeerPartitionedTree, key_splitters
 
         sp = key_splitters(keys, world)
         bnd = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [c["T"]]
         lk, lv = keys[bnd[rank]:bnd[rank + 1]], vals[bnd[rank]:bnd[rank + 1]]
-        pt = PartitionedTree(torch.from_numpy(lk).to(dev), torch.from_numpy(lv).to(dev), sp, fanout=c["F"],
-                             fill=a.fill, device=dev)
+        cls = PeerPartitionedTree if a.mode == "peer" else PartitionedTree
+        pt = cls(torch.from_numpy(lk).to(dev), torch.from_numpy(lv).to(dev), sp, fanout=c["F"], fill=a.fill,
+                 device=dev)
         t = pt.ops.tree
     else:
         t = hm.Tree(torch.from_numpy(keys).to(dev), torch.from_numpy(vals).to(dev), fanout=c["F"], fill=a.fill)
@@ -395,7 +396,7 @@ def main():
         e2e = {"value": c["Q"] * world * k2 / (hms / 1e3) / 1e9, "unit": UNIT,
                "h2d_bytes_per_step": int(c["Q"] * 8), "d2h_bytes_per_step": int(c["Q"] * 8),
                "steps": k2, "ms_per_step": hms / k2,
-               "api": "PartitionedTree.search + pinned copies" if pt is not None else
+               "api": type(pt).__name__ + ".search + pinned copies" if pt is not None else
                "harmonia_search_batch_host (pinned)"}
 
     if rank != 0:
@@ -464,7 +465,7 @@ def main():
         "warmup": max(3, a.warmup), "ms_per_step": ms_max / a.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": c["name"], "T": c["T"], "fanout": c["F"], "fill": a.fill, "Q_per_gpu": c["Q"],
-                   "queries": c["dist"], "mode": a.mode if (world > 1 or a.mode == "partitioned") else "single",
+                   "queries": c["dist"], "mode": a.mode if (world > 1 or a.mode in ("partitioned", "peer")) else "single",
                    "l2_flush": "inputs_larger_than_L2 (queries+results %d MiB/GPU > L2 %d MiB)" % (
                        c["Q"] * 16 >> 20, l2_bytes >> 20),
                    "plan": plan, "height": info["height"]},

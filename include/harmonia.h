@@ -223,6 +223,48 @@ harmonia_status harmonia_route_partition(const uint64_t* d_splitters, uint32_t P
 harmonia_status harmonia_scatter_results(const uint64_t* d_routed_values, const uint32_t* d_pos,
                                          uint64_t n, uint64_t* d_out, void* stream);
 
+/* ---------------------------------------------------------------------------------------
+ * Fused routing over peer memory (partitioned mode without NCCL data collectives; the
+ * north_star's "queries routed ... and results returned" step).  Per batch,
+ * all calls on one rank use the same workspace (harmonia_route_workspace_bytes(P, n)):
+ *   1. harmonia_route_count: dest(q) as in harmonia_route_partition; the per-query rank
+ *      inside its destination run is kept in the workspace; h_counts[P] (host, synchronous).
+ *   2. (caller) exchange the P x P count matrix; rank p's run for destination d starts at
+ *      sum_{p' < p} counts[p'][d] in d's receive buffer.
+ *   3. harmonia_route_push: the destination-major partition writes the run of destination d
+ *      straight to h_dst[d] (a device address: this rank's own buffer or a peer buffer mapped
+ *      with harmonia_peer_open; NVLink stores); the order inside a run is unspecified.
+ *      No local copy of the routed batch exists.  Asynchronous on `stream`.
+ *   4. (caller) barrier; each rank searches its receive buffer (harmonia_search_batch) and
+ *      returns the results of source p's segment with harmonia_segments_push to p's "back"
+ *      buffer at the offset of this rank's run in p's routed order; barrier.
+ *   5. harmonia_route_return: d_out[i] = d_back[routed position of query i] (the inverse of
+ *      step 3's partition; reads back in runs, writes d_out contiguously).
+ * harmonia_segments_push: for s < nseg, copy d_src[h_src_off[s] .. + h_len[s]) to the device
+ *   address h_dst[s] (16-byte stores when aligned).  nseg <= 1024.  Workspace: any buffer of
+ *   harmonia_route_workspace_bytes(1, 1) bytes not in use by a pending route call.
+ * P <= 256, n < 2^32; INVALID_ARG on violations or a short workspace.
+ * harmonia_peer_alloc: cudaMalloc(bytes) + its CUDA IPC handle (64 bytes written to
+ *   handle_out) for the other ranks; harmonia_peer_open maps a peer's handle into this
+ *   process (cudaIpcOpenMemHandle, lazy peer access); harmonia_peer_close unmaps it;
+ *   harmonia_peer_free releases an own buffer.  Setup-time calls, never on a query path.
+ * ------------------------------------------------------------------------------------- */
+harmonia_status harmonia_route_count(const uint64_t* d_splitters, uint32_t P, const uint64_t* d_queries,
+                                     uint64_t n, uint64_t* h_counts, void* d_workspace,
+                                     size_t workspace_bytes, void* stream);
+harmonia_status harmonia_route_push(const uint64_t* d_splitters, uint32_t P, const uint64_t* d_queries,
+                                    uint64_t n, const uint64_t* h_dst, void* d_workspace,
+                                    size_t workspace_bytes, void* stream);
+harmonia_status harmonia_route_return(uint32_t P, const uint64_t* d_back, uint64_t n, uint64_t* d_out,
+                                      void* d_workspace, size_t workspace_bytes, void* stream);
+harmonia_status harmonia_segments_push(const uint64_t* d_src, uint32_t nseg, const uint64_t* h_src_off,
+                                       const uint64_t* h_len, const uint64_t* h_dst, void* d_workspace,
+                                       size_t workspace_bytes, void* stream);
+harmonia_status harmonia_peer_alloc(size_t bytes, void** d_ptr, void* handle_out);
+harmonia_status harmonia_peer_open(const void* handle, void** d_ptr);
+harmonia_status harmonia_peer_close(void* d_ptr);
+harmonia_status harmonia_peer_free(void* d_ptr);
+
 /* The plan a search/range call with these options would use (for reporting). */
 typedef struct {
   int32_t group_size, psa_bits, smem_levels, ps_in_smem;

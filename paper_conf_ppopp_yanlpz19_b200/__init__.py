@@ -101,6 +101,14 @@ def lib():
             "harmonia_route_workspace_bytes": (_sz, [C.c_uint32, _u64]),
             "harmonia_route_partition": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _vp, _vp, _sz, _vp]),
             "harmonia_scatter_results": (C.c_int, [_vp, _vp, _u64, _vp, _vp]),
+            "harmonia_route_count": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _sz, _vp]),
+            "harmonia_route_push": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _sz, _vp]),
+            "harmonia_route_return": (C.c_int, [C.c_uint32, _vp, _u64, _vp, _vp, _sz, _vp]),
+            "harmonia_segments_push": (C.c_int, [_vp, C.c_uint32, _vp, _vp, _vp, _vp, _sz, _vp]),
+            "harmonia_peer_alloc": (C.c_int, [_sz, C.POINTER(_vp), _vp]),
+            "harmonia_peer_open": (C.c_int, [_vp, C.POINTER(_vp)]),
+            "harmonia_peer_close": (C.c_int, [_vp]),
+            "harmonia_peer_free": (C.c_int, [_vp]),
             "harmonia_psa_bits_auto": (C.c_int32, [_u64]),
             "harmonia_ntg_choose": (C.c_int, [_vp, _vp, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
                                               C.c_uint32, C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
@@ -296,6 +304,16 @@ class Tree:
                "harmonia_search_batch")
         return out
 
+    def search_addr(self, q_addr: int, n: int, out, *, opts: QueryOpts | None = None, stream=None, **kw):
+        """Point queries read from a raw device address (e.g. a peer-mapped receive buffer)."""
+        o = opts if opts is not None else make_opts(**kw)
+        ws_b = lib().harmonia_search_workspace_bytes(self._h, n, C.byref(o))
+        ws = self._workspace(ws_b)
+        _check(lib().harmonia_search_batch(self._h, q_addr, n, out.data_ptr(),
+                                           ws.data_ptr() if ws is not None else None, ws_b, C.byref(o),
+                                           _stream_ptr(stream, self.device)), "harmonia_search_batch")
+        return out
+
     def search_host(self, q_host, out_host=None, *, opts: QueryOpts | None = None, stream=None, **kw):
         """End-to-end point queries from host memory (pinned CPU tensors for overlap)."""
         torch = _torch()
@@ -371,3 +389,80 @@ def scatter_results(vals, pos, out=None, stream=None):
     _check(lib().harmonia_scatter_results(vals.data_ptr(), pos.data_ptr(), n, out.data_ptr(),
                                           _stream_ptr(stream, vals.device)), "harmonia_scatter_results")
     return out
+
+
+# ----------------------------------------------------------------------------- fused routing
+def _u64_array(vals):
+    a = (C.c_uint64 * max(len(vals), 1))()
+    for i, v in enumerate(vals):
+        a[i] = int(v) & ((1 << 64) - 1)
+    return a
+
+
+def route_workspace(P: int, n: int, device):
+    """Workspace for one batch of the fused-routing calls (kept for the whole batch)."""
+    torch = _torch()
+    b = lib().harmonia_route_workspace_bytes(P, n)
+    return torch.empty(b, dtype=torch.uint8, device=device)
+
+
+def route_count(splitters, P: int, q, ws, stream=None) -> list:
+    """Destination counts of the batch (harmonia_route_count; ranks kept in ws)."""
+    counts = (C.c_uint64 * P)()
+    sp = splitters.data_ptr() if P > 1 else None
+    _check(lib().harmonia_route_count(sp, P, q.data_ptr(), q.numel(), counts, ws.data_ptr(), ws.numel(),
+                                      _stream_ptr(stream, q.device)), "harmonia_route_count")
+    return [int(c) for c in counts]
+
+
+def route_push(splitters, P: int, q, dst_addrs, ws, stream=None):
+    """Write destination d's run of the batch to device address dst_addrs[d] (harmonia_route_push)."""
+    sp = splitters.data_ptr() if P > 1 else None
+    _check(lib().harmonia_route_push(sp, P, q.data_ptr(), q.numel(), _u64_array(dst_addrs), ws.data_ptr(),
+                                     ws.numel(), _stream_ptr(stream, q.device)), "harmonia_route_push")
+
+
+def route_return(P: int, back_addr: int, n: int, out, ws, stream=None):
+    """out[i] = back[routed position of query i] (harmonia_route_return)."""
+    _check(lib().harmonia_route_return(P, back_addr, n, out.data_ptr(), ws.data_ptr(), ws.numel(),
+                                       _stream_ptr(stream, out.device)), "harmonia_route_return")
+    return out
+
+
+def segments_push(src, src_off, lens, dst_addrs, ws, stream=None):
+    """Copy src[src_off[s] : +lens[s]] to device address dst_addrs[s] for every segment."""
+    _check(lib().harmonia_segments_push(src.data_ptr(), len(lens), _u64_array(src_off), _u64_array(lens),
+                                        _u64_array(dst_addrs), ws.data_ptr(), ws.numel(),
+                                        _stream_ptr(stream, src.device)), "harmonia_segments_push")
+
+
+class PeerBuffer:
+    """A device buffer other processes can map (CUDA IPC, harmonia_peer_alloc/open)."""
+
+    def __init__(self, nbytes: int):
+        self.ptr, self.nbytes = C.c_void_p(), nbytes
+        self.handle = (C.c_char * 64)()
+        _check(lib().harmonia_peer_alloc(nbytes, C.byref(self.ptr), self.handle), "harmonia_peer_alloc")
+
+    @property
+    def addr(self) -> int:
+        return int(self.ptr.value)
+
+    def handle_bytes(self) -> bytes:
+        return bytes(self.handle)
+
+    @staticmethod
+    def open(handle: bytes) -> int:
+        p = C.c_void_p()
+        h = (C.c_char * 64).from_buffer_copy(handle)
+        _check(lib().harmonia_peer_open(h, C.byref(p)), "harmonia_peer_open")
+        return int(p.value)
+
+    @staticmethod
+    def close_mapping(addr: int):
+        _check(lib().harmonia_peer_close(C.c_void_p(addr)), "harmonia_peer_close")
+
+    def free(self):
+        if self.ptr.value:
+            _check(lib().harmonia_peer_free(self.ptr), "harmonia_peer_free")
+            self.ptr = C.c_void_p()

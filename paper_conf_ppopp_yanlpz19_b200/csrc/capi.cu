@@ -382,12 +382,143 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
 }
 
 // ---- multi-GPU routing helpers ---------------------------------------------------------
+// the fused-routing calls keep their small host-built tables (push destinations, segment
+// descriptors) in the first kRouteTables bytes of the workspace; the PSA arrays follow
+constexpr size_t kRouteTables = 32 * 1024;
+constexpr uint32_t kMaxSegments = 1024;
+
 extern "C" size_t harmonia_route_workspace_bytes(uint32_t P, uint64_t n) {
   Plan p;
   p.psa = true;
   p.nbins = std::max<uint32_t>(P, 1);
   p.window = round_up(std::max<uint64_t>(n, 1), 1024);
-  return psa_ws_bytes(p) + 256;
+  return psa_ws_bytes(p) + 256 + kRouteTables;
+}
+
+namespace {
+// carve the routing workspace: tables first, then the PSA arrays of an n-query window
+harmonia_status route_carve(uint32_t P, uint64_t n, void* ws, size_t ws_bytes, PsaWs* w, uint64_t** tables) {
+  if (!ws) return HARMONIA_ERR_INVALID_ARG;
+  Plan p;
+  p.psa = true;
+  p.nbins = std::max<uint32_t>(P, 1);
+  p.window = round_up(std::max<uint64_t>(n, 1), 1024);
+  if (ws_bytes < psa_ws_bytes(p) + 256 + kRouteTables) return HARMONIA_ERR_INVALID_ARG;
+  if ((uintptr_t)ws & 255) ws = (char*)ws + (256 - ((uintptr_t)ws & 255));
+  *tables = reinterpret_cast<uint64_t*>(ws);
+  *w = psa_ws_carve(p, (char*)ws + kRouteTables);
+  return HARMONIA_OK;
+}
+int device_sms() {
+  int dev = 0, sm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
+  return sm;
+}
+}  // namespace
+
+extern "C" harmonia_status harmonia_route_count(const uint64_t* d_split, uint32_t P, const uint64_t* d_q, uint64_t n,
+                                                uint64_t* h_counts, void* ws, size_t ws_bytes, void* stream) {
+  if (P == 0 || P > 256 || !h_counts || (P > 1 && !d_split) || n >= (1ull << 32)) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) {
+    for (uint32_t i = 0; i < P; ++i) h_counts[i] = 0;
+    return HARMONIA_OK;
+  }
+  if (!d_q) return HARMONIA_ERR_INVALID_ARG;
+  PsaWs w;
+  uint64_t* tab;
+  harmonia_status s = route_carve(P, n, ws, ws_bytes, &w, &tab);
+  if (s != HARMONIA_OK) return s;
+  return route_count2(d_q, n, BucketSplit{d_split, P - 1}, P, w, device_sms(), (cudaStream_t)stream, h_counts);
+}
+
+extern "C" harmonia_status harmonia_route_push(const uint64_t* d_split, uint32_t P, const uint64_t* d_q, uint64_t n,
+                                               const uint64_t* h_dst, void* ws, size_t ws_bytes, void* stream) {
+  if (P == 0 || P > 256 || !h_dst || (P > 1 && !d_split) || n >= (1ull << 32)) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!d_q) return HARMONIA_ERR_INVALID_ARG;
+  PsaWs w;
+  uint64_t* tab;
+  harmonia_status s = route_carve(P, n, ws, ws_bytes, &w, &tab);
+  if (s != HARMONIA_OK) return s;
+  uint64_t table[256] = {};
+  for (uint32_t d = 0; d < P; ++d) table[d] = h_dst[d];
+  HM_CUDA(cudaMemcpyAsync(tab, table, sizeof(table), cudaMemcpyHostToDevice, (cudaStream_t)stream));
+  return route_push2(d_q, n, BucketSplit{d_split, P - 1}, P, w, tab, device_sms(), (cudaStream_t)stream);
+}
+
+extern "C" harmonia_status harmonia_route_return(uint32_t P, const uint64_t* d_back, uint64_t n, uint64_t* d_out,
+                                                 void* ws, size_t ws_bytes, void* stream) {
+  if (P == 0 || P > 256 || n >= (1ull << 32)) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!d_back || !d_out) return HARMONIA_ERR_INVALID_ARG;
+  PsaWs w;
+  uint64_t* tab;
+  harmonia_status s = route_carve(P, n, ws, ws_bytes, &w, &tab);
+  if (s != HARMONIA_OK) return s;
+  return route_return2(w, d_back, n, d_out, device_sms(), (cudaStream_t)stream);
+}
+
+extern "C" harmonia_status harmonia_segments_push(const uint64_t* d_src, uint32_t nseg, const uint64_t* h_src_off,
+                                                  const uint64_t* h_len, const uint64_t* h_dst, void* ws,
+                                                  size_t ws_bytes, void* stream) {
+  if (nseg == 0) return HARMONIA_OK;
+  if (nseg > kMaxSegments || !d_src || !h_src_off || !h_len || !h_dst || !ws || ws_bytes < kRouteTables + 256)
+    return HARMONIA_ERR_INVALID_ARG;
+  if ((uintptr_t)ws & 255) ws = (char*)ws + (256 - ((uintptr_t)ws & 255));
+  uint64_t* tab = reinterpret_cast<uint64_t*>(ws) + 256;  // after the push-destination table
+  uint64_t desc[3 * kMaxSegments];
+  uint64_t max_len = 0;
+  for (uint32_t s = 0; s < nseg; ++s) {
+    desc[3 * s] = h_src_off[s];
+    desc[3 * s + 1] = h_len[s];
+    desc[3 * s + 2] = h_dst[s];
+    if (h_len[s] && !h_dst[s]) return HARMONIA_ERR_INVALID_ARG;
+    max_len = std::max(max_len, h_len[s]);
+  }
+  HM_CUDA(cudaMemcpyAsync(tab, desc, nseg * 24, cudaMemcpyHostToDevice, (cudaStream_t)stream));
+  return segments_push(d_src, nseg, tab, max_len, device_sms(), (cudaStream_t)stream);
+}
+
+// ---- peer memory (CUDA IPC) for the fused routing ------------------------------------------
+extern "C" harmonia_status harmonia_peer_alloc(size_t bytes, void** d_ptr, void* handle_out) {
+  if (!d_ptr || !handle_out || bytes == 0) return HARMONIA_ERR_INVALID_ARG;
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    return HARMONIA_ERR_OUT_OF_MEMORY;
+  }
+  HM_CUDA(e);
+  cudaIpcMemHandle_t h;
+  e = cudaIpcGetMemHandle(&h, p);
+  if (e != cudaSuccess) {
+    cudaFree(p);
+    return cuda_fail(e);
+  }
+  std::memcpy(handle_out, &h, sizeof(h));
+  *d_ptr = p;
+  return HARMONIA_OK;
+}
+
+extern "C" harmonia_status harmonia_peer_open(const void* handle, void** d_ptr) {
+  if (!handle || !d_ptr) return HARMONIA_ERR_INVALID_ARG;
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  HM_CUDA(cudaIpcOpenMemHandle(d_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+  return HARMONIA_OK;
+}
+
+extern "C" harmonia_status harmonia_peer_close(void* d_ptr) {
+  if (!d_ptr) return HARMONIA_ERR_INVALID_ARG;
+  HM_CUDA(cudaIpcCloseMemHandle(d_ptr));
+  return HARMONIA_OK;
+}
+
+extern "C" harmonia_status harmonia_peer_free(void* d_ptr) {
+  if (!d_ptr) return HARMONIA_ERR_INVALID_ARG;
+  HM_CUDA(cudaFree(d_ptr));
+  return HARMONIA_OK;
 }
 
 extern "C" harmonia_status harmonia_route_partition(const uint64_t* d_split, uint32_t P, const uint64_t* d_q,

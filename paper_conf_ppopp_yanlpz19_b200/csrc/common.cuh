@@ -208,6 +208,15 @@ harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t
                                  cudaStream_t st, bool wide);
 harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
                                  int sm, cudaStream_t st, uint64_t* h_counts);
+// fused routing over peer memory (partitioned multi-GPU mode)
+harmonia_status route_count2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws, int sm,
+                             cudaStream_t st, uint64_t* h_counts);
+harmonia_status route_push2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
+                            const uint64_t* d_push, int sm, cudaStream_t st);
+harmonia_status route_return2(const PsaWs& ws, const uint64_t* back, uint64_t n, uint64_t* out, int sm,
+                              cudaStream_t st);
+harmonia_status segments_push(const uint64_t* src, uint32_t nseg, const uint64_t* d_desc, uint64_t max_len, int sm,
+                              cudaStream_t st);
 harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a,
                               cudaStream_t st);
 

@@ -200,7 +200,11 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_rank(const uint64_t* __
 // lanes.  The scattered shared-memory stores are the limiter (ncu: shared-store wavefronts),
 // so only the query is staged when the digit is cheap to recompute (the PSA coarse digit) and
 // the position only when idx is wanted (kIdx).
-template <class Digit, class C, bool kIdx>
+//
+// kPush (partitioned multi-GPU mode, fused routing): the run of destination d is written
+// straight into the receive buffer of rank d (a peer-mapped device pointer, NVLink stores),
+// push_dst[d] = address of this rank's segment there; nothing is written locally.
+template <class Digit, class C, bool kIdx, bool kPush = false>
 __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
                                                               const uint32_t* __restrict__ counts,
                                                               uint32_t* __restrict__ cursor,
@@ -209,8 +213,10 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
                                                               const uint32_t* __restrict__ cta_counts,
                                                               uint32_t* __restrict__ cta_base,
                                                               uint64_t* __restrict__ sorted_q,
-                                                              uint32_t* __restrict__ idx) {
+                                                              uint32_t* __restrict__ idx,
+                                                              const uint64_t* __restrict__ push_dst = nullptr) {
   constexpr bool kRecompute = std::is_same<Digit, CoarseDigit>::value;
+  __shared__ uint64_t s_push[kPush ? C::BINS : 1];  // push_dst[d] - 8 * (first global slot of bin d)
   extern __shared__ __align__(16) unsigned char l1_smem[];
   uint64_t* st_q = reinterpret_cast<uint64_t*>(l1_smem);
   uint32_t* bin_start = reinterpret_cast<uint32_t*>(l1_smem + C::TILE * 8);
@@ -229,6 +235,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
 #pragma unroll
     for (int k = 0; k < C::BPT; ++k) {
       const uint64_t b = threadIdx.x * C::BPT + k;
+      if constexpr (kPush) s_push[b] = push_dst[b] - 8ull * run[k];  // run[k] = bin start here
       const uint32_t cc = cta_counts[(uint64_t)blockIdx.x * C::BINS + b];
       run[k] = cc ? run[k] + atomicAdd(cursor + b, cc) : 0u;
       cta_base[(uint64_t)blockIdx.x * C::BINS + b] = run[k];  // for the staged return
@@ -276,7 +283,11 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
       if constexpr (kRecompute) dd = dg(x);
       else dd = st_d[i];
       const uint32_t dst = gbase[dd] + (i - bin_start[dd]);
-      sorted_q[dst] = x;
+      if constexpr (kPush) {
+        *reinterpret_cast<uint64_t*>(s_push[dd] + 8ull * dst) = x;
+      } else {
+        sorted_q[dst] = x;
+      }
       if constexpr (kIdx) idx[dst] = st_i[i];
     }
     __syncthreads();
@@ -557,7 +568,86 @@ harmonia_status unpartition(const PsaWs& ws, const uint64_t* res1, uint64_t n, u
   return HARMONIA_OK;
 }
 
+// copy nseg segments: dst_addr[s] <- src[src_off[s] .. + len[s]) (peer-mapped destinations);
+// grid.y = segment, 16-byte vector stores when both ends are aligned
+__global__ void __launch_bounds__(256) k_segments_push(const uint64_t* __restrict__ src,
+                                                       const uint64_t* __restrict__ desc) {
+  const uint64_t off = desc[blockIdx.y * 3], len = desc[blockIdx.y * 3 + 1];
+  uint64_t* dst = reinterpret_cast<uint64_t*>(desc[blockIdx.y * 3 + 2]);
+  const uint64_t* s = src + off;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if ((((uintptr_t)s | (uintptr_t)dst) & 15) == 0) {
+    const uint64_t pairs = len / 2;
+    for (uint64_t i = t0; i < pairs; i += stride)
+      reinterpret_cast<ulonglong2*>(dst)[i] = __ldg(reinterpret_cast<const ulonglong2*>(s) + i);
+    if (t0 == 0 && (len & 1)) dst[len - 1] = s[len - 1];
+  } else {
+    for (uint64_t i = t0; i < len; i += stride) dst[i] = s[i];
+  }
+}
+
 }  // namespace
+
+// fused routing (partitioned mode, peer memory): pass 1 = destination ranks and counts
+harmonia_status route_count2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws, int sm,
+                             cudaStream_t st, uint64_t* h_counts) {
+  using C = Narrow;
+  if (P > (uint32_t)C::BINS) return HARMONIA_ERR_INVALID_ARG;
+  HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * C::BINS * 4, st));
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
+    k_psa2_rank<BucketSplit, C><<<l1_grid<C>(n, sm), C::NT, 0, st>>>(q, n, f, ws.counts, ws.tile_counts, ws.packed,
+                                                                    ws.cta_counts);
+  }
+  HM_LAUNCHED();
+  uint32_t tmp[C::BINS];
+  HM_CUDA(cudaMemcpyAsync(tmp, ws.counts, P * 4, cudaMemcpyDeviceToHost, st));
+  HM_CUDA(cudaStreamSynchronize(st));
+  for (uint32_t b = 0; b < P; ++b) h_counts[b] = tmp[b];
+  return HARMONIA_OK;
+}
+
+// pass 2: every destination's run stored straight into its receive buffer (d_push[d])
+harmonia_status route_push2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
+                            const uint64_t* d_push, int sm, cudaStream_t st) {
+  using C = Narrow;
+  if (P > (uint32_t)C::BINS) return HARMONIA_ERR_INVALID_ARG;
+  constexpr size_t smb = move_smem<C, false, false>();
+  static bool cfg = false;
+  if (!cfg) {
+    HM_CUDA(cudaFuncSetAttribute(k_psa2_move<BucketSplit, C, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smb));
+    cfg = true;
+  }
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
+    k_psa2_move<BucketSplit, C, false, true><<<l1_grid<C>(n, sm), C::NT, smb, st>>>(
+        q, n, f, ws.counts, ws.counts + C::BINS, ws.tile_counts, ws.packed, ws.cta_counts, ws.cta_base, nullptr,
+        nullptr, d_push);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+// results in routed (destination-major) order -> caller order: the inverse move
+harmonia_status route_return2(const PsaWs& ws, const uint64_t* back, uint64_t n, uint64_t* out, int sm,
+                              cudaStream_t st) {
+  if (n == 0) return HARMONIA_OK;
+  return unpartition<Narrow>(ws, back, n, out, sm, st);
+}
+
+harmonia_status segments_push(const uint64_t* src, uint32_t nseg, const uint64_t* d_desc, uint64_t max_len, int sm,
+                              cudaStream_t st) {
+  if (nseg == 0 || max_len == 0) return HARMONIA_OK;
+  const uint64_t blocks = std::min<uint64_t>(ceil_div(max_len, 2 * 256), (uint64_t)sm * 8);
+  {
+    ProfScope ps_(HARMONIA_PROF_RETURN, st);
+    k_segments_push<<<dim3((unsigned)std::max<uint64_t>(blocks, 1), nseg), 256, 0, st>>>(src, d_desc);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
 
 // multi-GPU router: destination-major grouping by splitters (P <= 256 shards)
 harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,

@@ -10,6 +10,13 @@ PartitionedTree  rank p owns the keys in [splitter[p-1], splitter[p]) (key quant
                  reverse splits) -> harmonia_scatter_results back to the caller's order.
                  Ranges are cut at every splitter they cross; pieces are answered by their
                  shards and concatenated in shard order (= key order).
+PeerPartitionedTree  the same shards with the exchange fused into the kernels over peer memory
+                 (no NCCL data collective): harmonia_route_count -> all_gather of the P x P count
+                 matrix -> harmonia_route_push writes every destination's run straight into
+                 that rank's receive buffer (CUDA IPC mapping, NVLink stores) -> barrier ->
+                 local search of the receive buffer -> harmonia_segments_push returns every
+                 source's results into its "back" buffer -> barrier -> harmonia_route_return
+                 (inverse partition) restores the caller's order.
 
 The per-device steps go through a small `ops` object so that the exchange logic can be
 tested on CPU with a gloo group (tests/test_dist.py injects CPU stand-ins); the default ops
@@ -22,7 +29,8 @@ import torch.distributed as dist
 
 from . import Tree, route_partition, scatter_results
 
-__all__ = ["ReplicatedTree", "PartitionedTree", "CudaOps", "key_splitters"]
+__all__ = ["ReplicatedTree", "PartitionedTree", "PeerPartitionedTree", "CudaOps", "CudaPeerOps", "key_splitters",
+           "peer_offsets"]
 
 
 def _i64(t: torch.Tensor) -> torch.Tensor:
@@ -181,3 +189,156 @@ class PartitionedTree:
             out_k[rows, slot[valid]] = res[:, :cap][valid]
             out_v[rows, slot[valid]] = res[:, cap:2 * cap][valid]
         return _u64(out_k), _u64(out_v), total
+
+
+# ------------------------------------------------------------------ fused routing (peer memory)
+def peer_offsets(M, me: int):
+    """Offsets of the peer exchange from the P x P count matrix M[p][d] (queries rank p routes
+    to shard d), for rank `me`:
+      push_off[d]  element offset of me's run in d's receive buffer   = sum_{p<me} M[p][d]
+      recv_off[p]  where source p's segment starts in me's receive buffer = sum_{p'<p} M[p'][me]
+      recv_n       queries me receives                               = sum_p M[p][me]
+      back_off[p]  offset of me's run in p's routed order (= in p's back buffer) = sum_{d<me} M[p][d]
+    """
+    P = len(M)
+    push_off = [sum(M[p][d] for p in range(me)) for d in range(P)]
+    recv_off = [sum(M[q][me] for q in range(p)) for p in range(P)]
+    recv_n = sum(M[p][me] for p in range(P))
+    back_off = [sum(M[p][d] for d in range(me)) for p in range(P)]
+    return push_off, recv_off, recv_n, back_off
+
+
+class CudaPeerOps:
+    """Device steps and peer buffers of PeerPartitionedTree (libharmonia.so kernels, CUDA IPC)."""
+
+    def __init__(self, tree: Tree, splitters: torch.Tensor, P: int, group=None):
+        self.tree, self.split, self.P, self.group = tree, splitters, P, group
+        self.dev = tree.device
+        self.recv = self.back = None
+        self.recv_addr, self.back_addr = [], []
+        self.cap_recv = self.cap_back = 0
+        self.ws, self.ws_n = None, -1
+
+    # buffers --------------------------------------------------------------------------
+    def ensure_capacity(self, cap_recv: int, cap_back: int):
+        """Collective: every rank calls it with the same (cap_recv, cap_back)."""
+        from . import PeerBuffer
+
+        if cap_recv <= self.cap_recv and cap_back <= self.cap_back:
+            return
+        self.close()
+        cap_recv, cap_back = max(cap_recv, 1), max(cap_back, 1)
+        self.recv, self.back = PeerBuffer(cap_recv * 8), PeerBuffer(cap_back * 8)
+        mine = (self.recv.handle_bytes(), self.back.handle_bytes())
+        allh = [None] * self.P
+        dist.all_gather_object(allh, mine, group=self.group)
+        me = dist.get_rank(self.group)
+        self.recv_addr = [self.recv.addr if p == me else PeerBuffer.open(allh[p][0]) for p in range(self.P)]
+        self.back_addr = [self.back.addr if p == me else PeerBuffer.open(allh[p][1]) for p in range(self.P)]
+        self.cap_recv, self.cap_back = cap_recv, cap_back
+
+    def close(self):
+        from . import PeerBuffer
+
+        if self.recv is None:
+            return
+        torch.cuda.synchronize(self.dev)
+        dist.barrier(group=self.group)  # no peer still writes into the buffers being released
+        me = dist.get_rank(self.group)
+        for p in range(self.P):
+            if p != me:
+                PeerBuffer.close_mapping(self.recv_addr[p])
+                PeerBuffer.close_mapping(self.back_addr[p])
+        dist.barrier(group=self.group)  # every mapping closed before the owners free
+        self.recv.free()
+        self.back.free()
+        self.recv = self.back = None
+        self.cap_recv = self.cap_back = 0
+
+    # steps ----------------------------------------------------------------------------
+    def route_count(self, q):
+        from . import route_count, route_workspace
+
+        n = q.numel()
+        if self.ws is None or n > self.ws_n:
+            self.ws, self.ws_n = route_workspace(self.P, max(n, 1), self.dev), n
+        return route_count(self.split, self.P, q, self.ws)
+
+    def route_push(self, q, targets):
+        from . import route_push
+
+        route_push(self.split, self.P, q, [self.recv_addr[d] + 8 * off for d, off in targets], self.ws)
+
+    def search_recv(self, n: int):
+        out = torch.empty(n, dtype=torch.uint64, device=self.dev)
+        if n:
+            self.tree.search_addr(self.recv.addr, n, out)
+        return out
+
+    def segments_push(self, vals, segs):
+        from . import segments_push
+
+        segs = [s for s in segs if s[1] > 0]
+        if segs:
+            segments_push(vals, [s[0] for s in segs], [s[1] for s in segs],
+                          [self.back_addr[s[2]] + 8 * s[3] for s in segs], self.ws)
+
+    def route_return(self, n: int):
+        from . import route_return
+
+        out = torch.empty(n, dtype=torch.uint64, device=self.dev)
+        if n:
+            route_return(self.P, self.back.addr, n, out, self.ws)
+        return out
+
+    def fence(self):
+        torch.cuda.current_stream(self.dev).synchronize()  # the pushes of this rank are complete
+
+
+class PeerPartitionedTree:
+    """Key-range partitioned layout whose query exchange runs over peer memory (no NCCL data
+    collective): the route kernel stores every query straight into its shard's receive
+    buffer and the results come back the same way."""
+
+    def __init__(self, local_keys, local_values, splitters, fanout: int = 64, fill: float = 1.0, group=None,
+                 ops=None, device=None):
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        assert len(splitters) == self.world - 1, "P-1 splitters for P ranks"
+        if ops is None:
+            dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+            tree = Tree(local_keys, local_values, fanout=fanout, fill=fill, device=dev)
+            ops = CudaPeerOps(tree, _u64_words(splitters, dev).view(torch.uint64), self.world, group)
+        self.ops = ops
+        self.splitters = list(splitters)
+
+    def _count_matrix(self, counts):
+        nccl = dist.get_backend(self.group) == "nccl"
+        dev = torch.device("cuda", torch.cuda.current_device()) if nccl else torch.device("cpu")
+        mine = torch.tensor(counts, dtype=torch.int64, device=dev)
+        allc = torch.empty(self.world * self.world, dtype=torch.int64, device=dev)
+        dist.all_gather_into_tensor(allc, mine, group=self.group)
+        a = allc.view(self.world, self.world).tolist()
+        return a
+
+    def search(self, q: torch.Tensor) -> torch.Tensor:
+        P, me, n = self.world, self.rank, q.numel()
+        counts = self.ops.route_count(q)                       # kernel: destination ranks
+        M = self._count_matrix(counts)                         # P x P ints
+        push_off, recv_off, recv_n, back_off = peer_offsets(M, me)
+        need_recv = max(sum(M[p][d] for p in range(P)) for d in range(P))
+        need_back = max(sum(row) for row in M)
+        self.ops.ensure_capacity(need_recv, need_back)         # collective, same numbers everywhere
+        self.ops.route_push(q, [(d, push_off[d]) for d in range(P)])  # kernel: NVLink stores
+        self.ops.fence()
+        dist.barrier(group=self.group)                         # every run has arrived
+        vals = self.ops.search_recv(recv_n)                    # local Harmonia search
+        self.ops.segments_push(vals, [(recv_off[p], M[p][me], p, back_off[p]) for p in range(P)])
+        self.ops.fence()
+        dist.barrier(group=self.group)                         # every result has arrived
+        return self.ops.route_return(n)                        # kernel: caller's order
+
+    def close(self):
+        if hasattr(self.ops, "close"):
+            self.ops.close()

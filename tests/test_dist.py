@@ -135,3 +135,105 @@ def test_splitters_and_slices():
     sp = key_splitters(keys, 4)
     assert sp == [int(keys[250]), int(keys[500]), int(keys[750])]
     assert key_splitters(keys, 1) == []
+
+
+# ----------------------------------------------------------------------------- peer exchange
+class CpuPeerOps:
+    """Shared-memory stand-ins for CudaPeerOps (test only): recv[p] / back[p] are CPU tensors in
+    shared memory playing the peer-mapped device buffers, the oracle plays the local search."""
+
+    def __init__(self, keys, vals, splitters, P, me, recv, back):
+        import oracle
+
+        self.orc, self.keys, self.vals = oracle, keys, vals
+        self.split = np.asarray(splitters, dtype=np.uint64)
+        self.P, self.me, self.recv, self.back = P, me, recv, back
+
+    def ensure_capacity(self, cap_recv, cap_back):
+        assert cap_recv <= self.recv[0].numel() and cap_back <= self.back[0].numel()
+
+    def route_count(self, q):
+        self.q = q.view(torch.int64).numpy().view(np.uint64)
+        dest = np.searchsorted(self.split, self.q, side="right")
+        self.order = np.argsort(dest, kind="stable")  # routed (destination-major) order
+        self.dest = dest
+        return np.bincount(dest, minlength=self.P).tolist()
+
+    def route_push(self, q, targets):
+        qs = self.q[self.order].view(np.int64)
+        start = 0
+        for d, off in targets:
+            c = int(np.sum(self.dest == d))
+            self.recv[d][off:off + c] = torch.from_numpy(qs[start:start + c].copy())
+            start += c
+
+    def search_recv(self, n):
+        qn = self.recv[self.me][:n].numpy().view(np.uint64)
+        out = self.orc.sorted_search(self.keys, self.vals, qn, 1)
+        return torch.from_numpy(out.view(np.int64).copy())
+
+    def segments_push(self, vals, segs):
+        for off, ln, p, doff in segs:
+            self.back[p][doff:doff + ln] = vals[off:off + ln]
+
+    def route_return(self, n):
+        out = np.empty(n, dtype=np.int64)
+        out[self.order] = self.back[self.me][:n].numpy()
+        return torch.from_numpy(out).view(torch.uint64)
+
+    def fence(self):
+        pass
+
+
+def _peer_worker(rank, world, port, T, recv, back, result_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_ppopp_yanlpz19_b200.dist import PeerPartitionedTree, key_splitters
+
+        keys = gen.uniform_keys(T)
+        vals = gen.values_for(keys)
+        sp = key_splitters(keys, world)
+        bounds = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
+        lk, lv = keys[bounds[rank]:bounds[rank + 1]], vals[bounds[rank]:bounds[rank + 1]]
+        pt = PeerPartitionedTree(lk, lv, sp, ops=CpuPeerOps(lk, lv, sp, world, rank, recv, back))
+        ok = True
+        for b in range(3):  # several batches through the same buffers, uneven sizes per rank
+            nq = 0 if (b == 1 and rank == 0) else 2000 + 300 * rank + 50 * b
+            q = np.concatenate([gen.uniform_queries(keys, nq, seed=gen.SEED_QUERY + 10 * b + rank, miss_frac=0.3),
+                                np.asarray(sp, dtype=np.uint64)[:nq]])
+            got = pt.search(torch.from_numpy(q.view(np.int64).copy()).view(torch.uint64))
+            ok = ok and bool(np.array_equal(got.view(torch.int64).numpy().view(np.uint64),
+                                            oracle.sorted_search(keys, vals, q)))
+        result_q.put((rank, ok))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_peer_exchange_gloo(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    recv = [torch.zeros(20000, dtype=torch.int64).share_memory_() for _ in range(world)]
+    back = [torch.zeros(20000, dtype=torch.int64).share_memory_() for _ in range(world)]
+    procs = [ctx.Process(target=_peer_worker, args=(r, world, port, 20000, recv, back, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, ok in res:
+        assert ok, f"rank {rank}: peer-exchange results differ from the oracle"
+
+
+def test_peer_offsets():
+    from paper_conf_ppopp_yanlpz19_b200.dist import peer_offsets
+
+    M = [[1, 2, 3], [4, 5, 6], [7, 8, 9]]  # M[p][d]: queries rank p sends to shard d
+    push, roff, rn, boff = peer_offsets(M, 1)
+    assert push == [1, 2, 3]          # rank 0's runs precede rank 1's in every receive buffer
+    assert roff == [0, 2, 7] and rn == 15  # segments from ranks 0, 1, 2 of shard 1's buffer
+    assert boff == [1, 4, 7]          # shard 1's run in each source's routed order

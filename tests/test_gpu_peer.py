@@ -1,0 +1,125 @@
+"""Fused routing over peer memory (harmonia_route_count / route_push / segments_push /
+route_return, CUDA IPC buffers) on the GPU, bit-exact against the oracle.
+
+* single process: P virtual shards whose receive and back buffers are slices of local
+  tensors, so every kernel of the exchange runs without IPC;
+* two processes on the same GPU (gloo for the small control collectives): the full
+  PeerPartitionedTree path with real CUDA IPC mappings of the peer buffers (the box has one
+  GPU; across GPUs the same stores go over NVLink)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+
+import harmonia_gen as gen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def hm():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_ppopp_yanlpz19_b200 as m
+
+    m.lib()
+    return m
+
+
+def _u64(a):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint64).view(np.int64)).view(torch.uint64).cuda()
+
+
+def _np(t):
+    return t.view(torch.int64).cpu().numpy().view(np.uint64)
+
+
+@pytest.mark.parametrize("P,n", [(1, 1000), (3, 50001), (7, 4096), (64, 100000), (256, 30000)])
+def test_route_push_return_single_process(hm, orc, P, n):
+    keys = gen.uniform_keys(1 << 16)
+    vals = gen.values_for(keys)
+    sp = [int(keys[(p * len(keys)) // P]) for p in range(1, P)]
+    q = np.concatenate([gen.uniform_queries(keys, n, miss_frac=0.2), np.asarray(sp, dtype=np.uint64)])
+    qd = _u64(q)
+    spd = _u64(np.asarray(sp if sp else [0], dtype=np.uint64))
+    ws = hm.route_workspace(P, qd.numel(), qd.device)
+    counts = hm.route_count(spd, P, qd, ws)
+    dest = np.searchsorted(np.asarray(sp, dtype=np.uint64), q, side="right")
+    assert counts == np.bincount(dest, minlength=P).tolist()
+    # every shard's receive buffer is a slice of `recv`, with a gap so stray writes show up
+    gap = 5
+    starts = np.concatenate([[0], np.cumsum(np.asarray(counts) + gap)])[:P]
+    recv = torch.full((int(starts[-1]) + counts[-1] + gap,), -7, dtype=torch.int64, device="cuda")
+    hm.route_push(spd, P, qd, [recv.data_ptr() + 8 * int(s) for s in starts], ws)
+    torch.cuda.synchronize()
+    r = recv.cpu().numpy().view(np.uint64)
+    for d in range(P):
+        run = r[starts[d]:starts[d] + counts[d]]
+        assert np.array_equal(np.sort(run), np.sort(q[dest == d]))  # order inside a run: unspecified
+        assert np.all(recv.cpu().numpy()[starts[d] + counts[d]:starts[d] + counts[d] + gap] == -7)
+    # answer each run, push the answers back into one routed-order buffer, invert the partition
+    res = torch.from_numpy(orc.sorted_search(keys, vals, r).view(np.int64)).cuda()
+    back = torch.full((qd.numel(),), -1, dtype=torch.int64, device="cuda")
+    excl = np.concatenate([[0], np.cumsum(counts)])[:P]
+    ws2 = hm.route_workspace(1, 1, qd.device)
+    hm.segments_push(res, [int(s) for s in starts], counts, [back.data_ptr() + 8 * int(e) for e in excl], ws2)
+    out = torch.empty_like(qd)
+    hm.route_return(P, back.data_ptr(), qd.numel(), out, ws)
+    assert np.array_equal(_np(out), orc.sorted_search(keys, vals, q))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _ipc_worker(rank, world, port, T, result_q):
+    import torch.distributed as dist
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        import oracle
+        from paper_conf_ppopp_yanlpz19_b200.dist import PeerPartitionedTree, key_splitters
+
+        keys = gen.uniform_keys(T)
+        vals = gen.values_for(keys)
+        sp = key_splitters(keys, world)
+        bnd = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
+        lk, lv = keys[bnd[rank]:bnd[rank + 1]], vals[bnd[rank]:bnd[rank + 1]]
+        pt = PeerPartitionedTree(_u64(lk), _u64(lv), sp, fanout=16, device=torch.device("cuda", 0))
+        ok = True
+        for b, nq in enumerate((3000, 0, 70000, 5000)):  # growth of the buffers, an empty batch
+            nq = nq + 111 * rank if nq else (0 if rank == 0 else 900)
+            q = np.concatenate([gen.uniform_queries(keys, nq, seed=gen.SEED_QUERY + 10 * b + rank, miss_frac=0.3),
+                                gen.edge_queries(keys) if nq else np.zeros(0, np.uint64)])
+            got = _np(pt.search(_u64(q)))
+            ok = ok and bool(np.array_equal(got, oracle.sorted_search(keys, vals, q)))
+        pt.close()
+        result_q.put((rank, ok, ""))
+    except Exception as e:  # report instead of hanging the parent
+        result_q.put((rank, False, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_peer_partitioned_two_processes_ipc(world):
+    import torch.multiprocessing as mp
+
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ipc_worker, args=(r, world, port, 60000, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=120)
+    for rank, ok, err in res:
+        assert ok, f"rank {rank}: {err or 'peer-routed results differ from the oracle'}"
