@@ -206,6 +206,20 @@ harmonia_status harmonia_update_batch(harmonia_tree* tree, const uint8_t* d_ops,
                                       const uint64_t* d_keys, const uint64_t* d_values,
                                       uint64_t n, void* d_workspace, size_t workspace_bytes,
                                       void* stream);
+/* harmonia_update_batch_seq: the same with the batch order given explicitly: op i counts as
+ * issued at d_seq[i] (uint64, distinct), so the last op per key is the one with the largest
+ * seq (C-A18).  d_seq = NULL is harmonia_update_batch.  Used by the partitioned mode, where a
+ * shard receives the ops of several ranks in routed order.  Same workspace size.
+ * harmonia_route_update_payload: after harmonia_route_partition of the update keys (d_pos =
+ * its positions), d_ops_out[i] = d_ops[d_pos[i]], d_values_out[i] = d_values[d_pos[i]] and
+ * d_seq_out[i] = rank << 32 | d_pos[i] (global batch order = rank-major, then batch order). */
+harmonia_status harmonia_update_batch_seq(harmonia_tree* tree, const uint8_t* d_ops, const uint64_t* d_keys,
+                                          const uint64_t* d_values, const uint64_t* d_seq, uint64_t n,
+                                          void* d_workspace, size_t workspace_bytes, void* stream);
+harmonia_status harmonia_route_update_payload(const uint8_t* d_ops, const uint64_t* d_values,
+                                              const uint32_t* d_pos, uint64_t n, uint32_t rank,
+                                              uint8_t* d_ops_out, uint64_t* d_values_out,
+                                              uint64_t* d_seq_out, void* stream);
 
 /* ---------------------------------------------------------------------------------------
  * Key-range partitioning across P devices (multi-GPU mode).

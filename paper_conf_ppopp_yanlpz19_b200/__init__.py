@@ -98,6 +98,8 @@ def lib():
                                                C.POINTER(QueryOpts), _vp]),
             "harmonia_update_workspace_bytes": (_sz, [_vp, _u64]),
             "harmonia_update_batch": (C.c_int, [_vp, _vp, _vp, _vp, _u64, _vp, _sz, _vp]),
+            "harmonia_update_batch_seq": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _u64, _vp, _sz, _vp]),
+            "harmonia_route_update_payload": (C.c_int, [_vp, _vp, _vp, _u64, C.c_uint32, _vp, _vp, _vp, _vp]),
             "harmonia_route_workspace_bytes": (_sz, [C.c_uint32, _u64]),
             "harmonia_route_partition": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _vp, _vp, _sz, _vp]),
             "harmonia_scatter_results": (C.c_int, [_vp, _vp, _u64, _vp, _vp]),
@@ -350,8 +352,9 @@ class Tree:
                "harmonia_range_batch")
         return ko, vo, cnt
 
-    def update(self, ops, keys, values, stream=None):
-        """Batched upsert (op 0) / delete (op 1), sequential semantics in batch order."""
+    def update(self, ops, keys, values, seq=None, stream=None):
+        """Batched upsert (op 0) / delete (op 1), sequential semantics in batch order (or in
+        ascending `seq`, uint64 per op, when given: harmonia_update_batch_seq)."""
         torch = _torch()
         if isinstance(ops, np.ndarray):
             ops = torch.from_numpy(np.ascontiguousarray(ops.astype(np.uint8)))
@@ -361,8 +364,14 @@ class Tree:
         ws_b = lib().harmonia_update_workspace_bytes(self._h, n)
         ws = torch.empty(max(ws_b, 1), dtype=torch.uint8, device=self.device)
         st = _stream_ptr(stream, self.device)
-        _check(lib().harmonia_update_batch(self._h, ops.data_ptr(), keys.data_ptr(), values.data_ptr(), n,
-                                           ws.data_ptr(), ws_b, st), "harmonia_update_batch")
+        if seq is None:
+            _check(lib().harmonia_update_batch(self._h, ops.data_ptr(), keys.data_ptr(), values.data_ptr(), n,
+                                               ws.data_ptr(), ws_b, st), "harmonia_update_batch")
+        else:
+            seq = _as_u64_dev(seq, self.device)
+            _check(lib().harmonia_update_batch_seq(self._h, ops.data_ptr(), keys.data_ptr(), values.data_ptr(),
+                                                   seq.data_ptr(), n, ws.data_ptr(), ws_b, st),
+                   "harmonia_update_batch_seq")
 
 
 def route_partition(splitters, P: int, q, stream=None):
@@ -379,6 +388,20 @@ def route_partition(splitters, P: int, q, stream=None):
     _check(lib().harmonia_route_partition(sp, P, q.data_ptr(), n, routed.data_ptr(), pos.data_ptr(), counts,
                                           ws.data_ptr(), ws_b, _stream_ptr(stream, dev)), "harmonia_route_partition")
     return routed, pos, [int(c) for c in counts]
+
+
+def route_update_payload(ops, values, pos, rank: int, stream=None):
+    """Routed update payload (harmonia_route_update_payload): ops/values in routed order and the
+    global sequence number rank << 32 | original position of every routed op."""
+    torch = _torch()
+    n = pos.numel()
+    o = torch.empty(n, dtype=torch.uint8, device=pos.device)
+    v = torch.empty(n, dtype=torch.uint64, device=pos.device)
+    sq = torch.empty(n, dtype=torch.uint64, device=pos.device)
+    _check(lib().harmonia_route_update_payload(ops.data_ptr(), values.data_ptr(), pos.data_ptr(), n, rank,
+                                               o.data_ptr(), v.data_ptr(), sq.data_ptr(),
+                                               _stream_ptr(stream, pos.device)), "harmonia_route_update_payload")
+    return o, v, sq
 
 
 def scatter_results(vals, pos, out=None, stream=None):

@@ -41,6 +41,26 @@ __global__ void k_iota(uint32_t* __restrict__ p, uint64_t n) {
     p[i] = (uint32_t)i;
 }
 
+__global__ void k_gather_keys(const uint64_t* __restrict__ src, const uint32_t* __restrict__ idx, uint64_t n,
+                              uint64_t* __restrict__ dst) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    dst[i] = src[idx[i]];
+}
+
+// routed update payload: op, value and sequence number of routed entry i come from batch
+// position pos[i]; seq = rank << 32 | pos (global batch order = rank-major, C-A18)
+__global__ void k_route_update_payload(const uint8_t* __restrict__ ops, const uint64_t* __restrict__ vals,
+                                       const uint32_t* __restrict__ pos, uint64_t n, uint64_t rank,
+                                       uint8_t* __restrict__ ops_out, uint64_t* __restrict__ vals_out,
+                                       uint64_t* __restrict__ seq_out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t p = pos[i];
+    ops_out[i] = ops[p];
+    vals_out[i] = vals[p];
+    seq_out[i] = rank << 32 | p;
+  }
+}
+
 // flag[i] = 1 if sorted entry i is the last op on its key
 __global__ void k_upd_winners(const uint64_t* __restrict__ sk, uint64_t n, uint32_t* __restrict__ flag) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
@@ -210,6 +230,12 @@ extern "C" size_t harmonia_update_workspace_bytes(const harmonia_tree* t, uint64
 extern "C" harmonia_status harmonia_update_batch(harmonia_tree* t, const uint8_t* d_ops, const uint64_t* d_keys,
                                                  const uint64_t* d_values, uint64_t n, void* ws, size_t ws_bytes,
                                                  void* stream) {
+  return harmonia_update_batch_seq(t, d_ops, d_keys, d_values, nullptr, n, ws, ws_bytes, stream);
+}
+
+extern "C" harmonia_status harmonia_update_batch_seq(harmonia_tree* t, const uint8_t* d_ops, const uint64_t* d_keys,
+                                                     const uint64_t* d_values, const uint64_t* d_seq, uint64_t n,
+                                                     void* ws, size_t ws_bytes, void* stream) {
   if (!t) return HARMONIA_ERR_INVALID_ARG;
   if (n == 0) return HARMONIA_OK;
   if (!d_ops || !d_keys || !d_values || !ws) return HARMONIA_ERR_INVALID_ARG;
@@ -247,9 +273,19 @@ extern "C" harmonia_status harmonia_update_batch(harmonia_tree* t, const uint8_t
   k_iota<<<grid_of(n, sm), kBlock, 0, st>>>(pos, n);
   HM_LAUNCHED();
   size_t cb = cubb;
-  HM_CUDA(cub::DeviceRadixSort::SortPairs(P(L.cub), cb, d_keys, sk2, pos, pos2, (int)n, 0, 64, st));
-  count_launch(4);
-  (void)sk;
+  if (d_seq) {  // batch order = ascending seq: present the keys in that order to the stable key sort
+    HM_CUDA(cub::DeviceRadixSort::SortPairs(P(L.cub), cb, d_seq, sk, pos, pos2, (int)n, 0, 64, st));
+    count_launch(4);
+    k_gather_keys<<<grid_of(n, sm), kBlock, 0, st>>>(d_keys, pos2, n, sk);
+    HM_LAUNCHED();
+    cb = cubb;
+    HM_CUDA(cub::DeviceRadixSort::SortPairs(P(L.cub), cb, sk, sk2, pos2, pos, (int)n, 0, 64, st));
+    count_launch(4);
+    std::swap(pos, pos2);  // pos2 = original batch index of each key-sorted entry
+  } else {
+    HM_CUDA(cub::DeviceRadixSort::SortPairs(P(L.cub), cb, d_keys, sk2, pos, pos2, (int)n, 0, 64, st));
+    count_launch(4);
+  }
   // 3. winners (last op per key) and their compaction
   uint32_t *flag = (uint32_t*)P(L.flag), *at = (uint32_t*)P(L.at);
   k_upd_winners<<<grid_of(n, sm), kBlock, 0, st>>>(sk2, n, flag);
@@ -344,5 +380,21 @@ extern "C" harmonia_status harmonia_update_batch(harmonia_tree* t, const uint8_t
     t->min_key = kPad;
     t->max_key = 0;
   }
+  return HARMONIA_OK;
+}
+
+extern "C" harmonia_status harmonia_route_update_payload(const uint8_t* d_ops, const uint64_t* d_values,
+                                                         const uint32_t* d_pos, uint64_t n, uint32_t rank,
+                                                         uint8_t* d_ops_out, uint64_t* d_values_out,
+                                                         uint64_t* d_seq_out, void* stream) {
+  if (n == 0) return HARMONIA_OK;
+  if (!d_ops || !d_values || !d_pos || !d_ops_out || !d_values_out || !d_seq_out || n >= (1ull << 32))
+    return HARMONIA_ERR_INVALID_ARG;
+  int dev = 0, sm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
+  k_route_update_payload<<<grid_of(n, sm), kBlock, 0, (cudaStream_t)stream>>>(d_ops, d_values, d_pos, n, rank,
+                                                                              d_ops_out, d_values_out, d_seq_out);
+  HM_LAUNCHED();
   return HARMONIA_OK;
 }

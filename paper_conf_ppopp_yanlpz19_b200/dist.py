@@ -27,7 +27,7 @@ from __future__ import annotations
 import torch
 import torch.distributed as dist
 
-from . import Tree, route_partition, scatter_results
+from . import Tree, route_partition, route_update_payload, scatter_results
 
 __all__ = ["ReplicatedTree", "PartitionedTree", "PeerPartitionedTree", "CudaOps", "CudaPeerOps", "key_splitters",
            "peer_offsets"]
@@ -73,6 +73,43 @@ class CudaOps:
 
     def scatter(self, vals, pos):
         return scatter_results(vals, pos)
+
+    def route_update(self, ops, keys, values, rank: int):
+        rk, pos, counts = route_partition(self.split, self.P, keys)
+        ro, rv, rs = route_update_payload(ops, values, pos, rank)
+        return rk, ro, rv, rs, counts
+
+    def update(self, ops, keys, values, seq):
+        self.tree.update(ops, keys, values, seq=seq)
+
+
+def _routed_update(tree_like, ops, keys, values):
+    """Batched updates on a key-range partitioned tree (updates are routed like
+    queries).  Each op goes to the shard owning its key, with its global sequence number
+    rank << 32 | position, so a shard applies the ops it receives in the global batch order
+    (rank-major, then each rank's batch order; C-A18 last-op-wins) whatever order routing
+    and the exchange deliver them in.  Collective: every rank calls it (possibly with 0 ops)."""
+    ops_ = tree_like.ops
+    group, P = tree_like.group, tree_like.world
+    rk, ro, rv, rs, counts = ops_.route_update(ops, keys, values, tree_like.rank)
+    dev = keys.device
+    send = torch.tensor(counts, dtype=torch.int64, device=dev)
+    recv = torch.empty(P, dtype=torch.int64, device=dev)
+    dist.all_to_all_single(recv, send, group=group)
+    rc = recv.tolist()
+    m = sum(rc)
+
+    def a2a(x, dtype):
+        out = torch.empty(m, dtype=dtype, device=dev)
+        dist.all_to_all_single(out, x, output_split_sizes=rc, input_split_sizes=counts, group=group)
+        return out
+
+    k = a2a(_i64(rk), torch.int64)
+    v = a2a(_i64(rv), torch.int64)
+    sq = a2a(_i64(rs), torch.int64)
+    o = a2a(ro, torch.uint8)
+    if m:
+        ops_.update(o, _u64(k), _u64(v), _u64(sq))
 
 
 class ReplicatedTree:
@@ -129,6 +166,11 @@ class PartitionedTree:
         dist.all_to_all_single(back, _i64(vals), output_split_sizes=counts, input_split_sizes=rc,
                                group=self.group)               # C5: return values
         return self.ops.scatter(_u64(back), pos)               # caller's order
+
+    # ------------------------------------------------------------------ updates
+    def update(self, ops, keys, values):
+        """Batched upsert (op 0) / delete (op 1) routed to the owning shards (collective)."""
+        _routed_update(self, ops, keys, values)
 
     # ------------------------------------------------------------------ range queries
     def range(self, lo: torch.Tensor, hi: torch.Tensor, cap: int):
@@ -294,6 +336,14 @@ class CudaPeerOps:
     def fence(self):
         torch.cuda.current_stream(self.dev).synchronize()  # the pushes of this rank are complete
 
+    def route_update(self, ops, keys, values, rank: int):
+        rk, pos, counts = route_partition(self.split, self.P, keys)
+        ro, rv, rs = route_update_payload(ops, values, pos, rank)
+        return rk, ro, rv, rs, counts
+
+    def update(self, ops, keys, values, seq):
+        self.tree.update(ops, keys, values, seq=seq)
+
 
 class PeerPartitionedTree:
     """Key-range partitioned layout whose query exchange runs over peer memory (no NCCL data
@@ -338,6 +388,10 @@ class PeerPartitionedTree:
         self.ops.fence()
         dist.barrier(group=self.group)                         # every result has arrived
         return self.ops.route_return(n)                        # kernel: caller's order
+
+    def update(self, ops, keys, values):
+        """Batched upsert (op 0) / delete (op 1) routed to the owning shards (collective)."""
+        _routed_update(self, ops, keys, values)
 
     def close(self):
         if hasattr(self.ops, "close"):

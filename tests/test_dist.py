@@ -65,6 +65,24 @@ class CpuOps:
         out[pos] = vals.view(torch.int64)
         return out.view(torch.uint64)
 
+    def route_update(self, ops, keys, values, rank):
+        kn = keys.view(torch.int64).numpy().view(np.uint64)
+        dest = np.searchsorted(self.split, kn, side="right")
+        pos = np.argsort(dest, kind="stable")[::-1].copy()  # any order: the seq numbers carry it
+        pos = pos[np.argsort(dest[pos], kind="stable")]
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy())
+        seq = (np.uint64(rank) << np.uint64(32)) | pos.astype(np.uint64)
+        return (t(kn[pos]).view(torch.uint64), torch.from_numpy(ops.numpy()[pos].copy()),
+                t(values.view(torch.int64).numpy().view(np.uint64)[pos]).view(torch.uint64), t(seq).view(torch.uint64),
+                np.bincount(dest, minlength=self.P).tolist())
+
+    def update(self, ops, keys, values, seq):
+        order = np.argsort(seq.view(torch.int64).numpy().view(np.uint64), kind="stable")
+        m = self.orc.UpdateMap(self.keys, self.vals)
+        m.apply(ops.numpy()[order], keys.view(torch.int64).numpy().view(np.uint64)[order],
+                values.view(torch.int64).numpy().view(np.uint64)[order])
+        self.keys, self.vals = m.dump()
+
 
 def _worker(rank, world, port, T, cap, result_q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
@@ -237,3 +255,56 @@ def test_peer_offsets():
     assert push == [1, 2, 3]          # rank 0's runs precede rank 1's in every receive buffer
     assert roff == [0, 2, 7] and rn == 15  # segments from ranks 0, 1, 2 of shard 1's buffer
     assert boff == [1, 4, 7]          # shard 1's run in each source's routed order
+
+
+def _update_worker(rank, world, port, T, result_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree, key_splitters
+
+        keys = gen.uniform_keys(T)
+        vals = gen.values_for(keys)
+        sp = key_splitters(keys, world)
+        bounds = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
+        lk, lv = keys[bounds[rank]:bounds[rank + 1]], vals[bounds[rank]:bounds[rank + 1]]
+        pt = PartitionedTree(lk, lv, sp, ops=CpuOps(lk, lv, sp, world))
+        ref = oracle.UpdateMap(keys, vals)
+        batches = []
+        for r in range(world):  # every rank builds every batch (same seeds) for the reference
+            n = 0 if r == world - 1 and world > 2 else 3000 + 100 * r
+            o, k, v = gen.update_ops(keys, n, insert_frac=0.1, delete_frac=0.2, seed=gen.SEED_OPS + r)
+            if n:  # the same key several times inside one batch and across batches
+                k[-200:] = k[:200]
+                k[:50] = batches[0][1][:50] if batches and len(batches[0][1]) else k[:50]
+                o[k == gen.uniform_keys(T)[0]] = 1
+            batches.append((o, k, v))
+        for o, k, v in batches:
+            ref.apply(o, k, v)
+        o, k, v = batches[rank]
+        t64 = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy()).view(torch.uint64)
+        pt.update(torch.from_numpy(o.copy()), t64(k), t64(v))
+        ek, ev = ref.dump()
+        q = np.concatenate([keys, np.concatenate([b[1] for b in batches]), gen.edge_queries(keys)])
+        got = pt.search(t64(q)).view(torch.int64).numpy().view(np.uint64)
+        ok = bool(np.array_equal(got, oracle.sorted_search(ek, ev, q)))
+        result_q.put((rank, ok))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_partitioned_update_gloo(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_update_worker, args=(r, world, port, 8000, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, ok in res:
+        assert ok, f"rank {rank}: routed updates differ from the global-order oracle"

@@ -117,3 +117,39 @@ def test_paper_scale_update_batch(hm, orc):
     sel = gen._stream(5, 0, 1 << 18) % np.uint64(rk.shape[0])
     probe = np.concatenate([rk[sel], ks[: 1 << 18]])
     assert np.array_equal(t.search(cu(probe)).cpu().numpy(), orc.sorted_search(rk, rv, probe))
+
+
+@pytest.mark.parametrize("F", [8, 64])
+def test_update_batch_seq_order(hm, orc, F):
+    """harmonia_update_batch_seq: ops take effect in ascending seq, not in array order; with
+    many ops per key (upserts and deletes interleaved) the last by seq must win."""
+    keys = gen.uniform_keys(20000)
+    vals = gen.values_for(keys)
+    t = hm.Tree(cu(keys), cu(vals), fanout=F)
+    ops, k, v = gen.update_ops(keys, 30000, insert_frac=0.1, delete_frac=0.3)
+    k[10000:20000] = k[:10000]  # every key of the first third appears two or three times
+    k[20000:25000] = k[:5000]
+    rng = np.random.default_rng(F)
+    seq = (rng.permutation(30000).astype(np.uint64) << np.uint64(20)) | np.uint64(7)
+    t.update(cu(ops), cu(k), cu(v), seq=cu(seq))
+    order = np.argsort(seq, kind="stable")
+    ref = orc.UpdateMap(keys, vals)
+    ref.apply(ops[order], k[order], v[order])
+    rk, rv = ref.dump()
+    probe = np.concatenate([keys, k, gen.edge_queries(keys)])
+    check_tree(hm, orc, t, F, rk, rv, probe)
+
+
+def test_route_update_payload(hm):
+    import torch
+
+    n = 10007
+    rng = np.random.default_rng(3)
+    ops = rng.integers(0, 2, n).astype(np.uint8)
+    vals = gen._stream(9, 0, n)
+    pos = rng.permutation(n).astype(np.uint32)
+    o, v, s = hm.route_update_payload(cu(ops), cu(vals), torch.from_numpy(pos.view(np.int32)).cuda().view(torch.uint32),
+                                      5)
+    assert np.array_equal(o.cpu().numpy(), ops[pos])
+    assert np.array_equal(v.cpu().numpy(), vals[pos])
+    assert np.array_equal(s.cpu().numpy(), (np.uint64(5) << np.uint64(32)) | pos.astype(np.uint64))
