@@ -61,6 +61,46 @@ struct ProfScope {
   }
 };
 
+// ---- 1-D TMA bulk copies (cp.async.bulk, global -> shared) on an mbarrier ----------------
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+// one thread: the phase's single arrival, announcing `bytes` of transactions
+__device__ __forceinline__ void bulk_expect(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes) : "memory");
+}
+// copy `bytes` (% 16 == 0, both addresses 16-byte aligned) completing on bar; chunks of at
+// most 64 KiB per instruction.  Every copy of a phase must be covered by its bulk_expect.
+__device__ __forceinline__ void bulk_copy(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  const uint32_t b = smem_addr(bar);
+  for (uint32_t off = 0; off < bytes; off += 65536) {
+    const uint32_t sz = bytes - off < 65536 ? bytes - off : 65536;
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_addr((char*)dst + off)),
+        "l"((const char*)src + off), "r"(sz), "r"(b)
+        : "memory");
+  }
+}
+// one copy per phase: arrival + copy
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  bulk_expect(bar, bytes);
+  bulk_copy(dst, src, bytes, bar);
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  const uint32_t b = smem_addr(bar);
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(b), "r"(parity)
+        : "memory");
+  }
+}
+
 // ---- PSA bucket function (C-A11): bits [span-Nb, span) of clamp(q, kmin, kmax) -------
 struct BucketBits {
   uint64_t kmin, kmax;

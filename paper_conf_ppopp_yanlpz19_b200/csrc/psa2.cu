@@ -138,6 +138,18 @@ __device__ __forceinline__ void l1_tile_range(uint64_t n, uint32_t tile, uint64_
   *te = (uint64_t)(blockIdx.x + 1) * T / gridDim.x;
 }
 
+// ---- tile prefetch: every level-1 CTA walks a contiguous tile range, so the next tile's
+// inputs stream into shared memory by TMA bulk copies (one thread) while the current tile is
+// processed -- the per-tile load latency was exposed (ncu: long-scoreboard stalls).
+#ifndef HM_L1_PREFETCH
+#define HM_L1_PREFETCH 0  // measured: neutral to -2 % (the level-1 passes are bound by shared-store conflicts)
+#endif
+template <class C>
+__device__ __forceinline__ uint32_t tile_bytes(uint64_t tile, uint64_t n, uint32_t elem) {
+  const uint64_t m = std::min<uint64_t>(C::TILE, n - tile * C::TILE);
+  return (uint32_t)((m * elem + 15) & ~15ull);  // the tail rounds up inside its 16-byte block
+}
+
 // ---- level 1, pass 1: per-tile digit ranks ---------------------------------------------
 // Each query's coarse digit d and its rank among the tile's queries with digit d are taken
 // once, with a shared-memory atomic, and stored packed (d | rank << BITS) so that the move
@@ -152,22 +164,37 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_rank(const uint64_t* __
                                                               uint32_t* __restrict__ packed,
                                                               uint32_t* __restrict__ cta_counts) {
   __shared__ uint32_t cnt[C::BINS];
+  __shared__ __align__(16) uint64_t sq[HM_L1_PREFETCH ? C::TILE : 2];
+  __shared__ __align__(8) uint64_t bar;
   uint64_t tb, te;
   l1_tile_range(n, C::TILE, &tb, &te);
+  const bool pf = HM_L1_PREFETCH && ((uintptr_t)q & 15) == 0;
+  if (pf && threadIdx.x == 0) {
+    mbar_init(&bar, 1);
+    if (tb < te) bulk_load(sq, q + tb * C::TILE, tile_bytes<C>(tb, n, 8), &bar);
+  }
+  __syncthreads();
+  uint32_t phase = 0;
   uint32_t acc[C::BPT];
 #pragma unroll
   for (int k = 0; k < C::BPT; ++k) acc[k] = 0;
   for (uint64_t tile = tb; tile < te; ++tile) {
     const uint64_t t0 = tile * C::TILE;
     uint64_t v[C::PER];
+    if (pf) {
+      mbar_wait(&bar, phase);
+      phase ^= 1;
+    }
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {  // all loads first (PER in flight per thread)
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
-      v[k] = e < n ? __ldg(q + e) : 0;
+      v[k] = e < n ? (pf ? sq[k * C::NT + threadIdx.x] : __ldg(q + e)) : 0;
     }
 #pragma unroll
     for (int k = 0; k < C::BPT; ++k) cnt[k * C::NT + threadIdx.x] = 0;
     __syncthreads();
+    if (pf && threadIdx.x == 0 && tile + 1 < te)
+      bulk_load(sq, q + (tile + 1) * C::TILE, tile_bytes<C>(tile + 1, n, 8), &bar);
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
@@ -223,9 +250,24 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
   uint32_t* gbase = bin_start + C::BINS;
   uint32_t* st_i = gbase + C::BINS;                                       // kIdx
   uint8_t* st_d = reinterpret_cast<uint8_t*>(st_i + (kIdx ? C::TILE : 0));  // !kRecompute
+  // prefetch stage (16-byte aligned): next tile's queries and packed ranks
+  uint64_t* pq = reinterpret_cast<uint64_t*>(l1_smem + ((C::TILE * 8 + 2 * C::BINS * 4 + (kIdx ? C::TILE * 4 : 0) +
+                                                          (kRecompute ? 0 : C::TILE) + 15) & ~15));
+  uint32_t* pp = reinterpret_cast<uint32_t*>(pq + C::TILE);
   __shared__ uint32_t tmp[C::NT / 32 + 1];
+  __shared__ __align__(8) uint64_t bar;
   uint64_t tb, te;
   l1_tile_range(n, C::TILE, &tb, &te);
+  const bool pf = HM_L1_PREFETCH && ((uintptr_t)q & 15) == 0;
+  if (pf && threadIdx.x == 0) {
+    mbar_init(&bar, 1);
+    if (tb < te) {
+      bulk_expect(&bar, tile_bytes<C>(tb, n, 8) + tile_bytes<C>(tb, n, 4));
+      bulk_copy(pq, q + tb * C::TILE, tile_bytes<C>(tb, n, 8), &bar);
+      bulk_copy(pp, packed + tb * C::TILE, tile_bytes<C>(tb, n, 4), &bar);
+    }
+  }
+  uint32_t phase = 0;
   uint32_t run[C::BPT];  // next free global slot of bins threadIdx.x * BPT + k for this CTA
   {
     uint32_t cv[C::BPT];
@@ -245,11 +287,15 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
     const uint64_t t0 = tile * C::TILE;
     uint64_t v[C::PER];
     uint32_t pk[C::PER];
+    if (pf) {
+      mbar_wait(&bar, phase);
+      phase ^= 1;
+    }
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
-      v[k] = e < n ? __ldg(q + e) : 0;
-      pk[k] = e < n ? __ldg(packed + e) : 0;
+      v[k] = e < n ? (pf ? pq[k * C::NT + threadIdx.x] : __ldg(q + e)) : 0;
+      pk[k] = e < n ? (pf ? pp[k * C::NT + threadIdx.x] : __ldg(packed + e)) : 0;
     }
     {
       uint32_t cv[C::BPT], ex[C::BPT];
@@ -264,6 +310,11 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
       }
     }
     __syncthreads();
+    if (pf && threadIdx.x == 0 && tile + 1 < te) {  // every thread has read the stage
+      bulk_expect(&bar, tile_bytes<C>(tile + 1, n, 8) + tile_bytes<C>(tile + 1, n, 4));
+      bulk_copy(pq, q + (tile + 1) * C::TILE, tile_bytes<C>(tile + 1, n, 8), &bar);
+      bulk_copy(pp, packed + (tile + 1) * C::TILE, tile_bytes<C>(tile + 1, n, 4), &bar);
+    }
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
@@ -295,7 +346,8 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
 }
 template <class C, bool kIdx, bool kRecompute>
 constexpr size_t move_smem() {
-  return (size_t)C::TILE * 8 + 2 * C::BINS * 4 + (kIdx ? C::TILE * 4 : 0) + (kRecompute ? 0 : C::TILE);
+  return (((size_t)C::TILE * 8 + 2 * C::BINS * 4 + (kIdx ? C::TILE * 4 : 0) + (kRecompute ? 0 : C::TILE) + 15) & ~15) +
+         (HM_L1_PREFETCH ? (size_t)C::TILE * 12 : 0);
 }
 
 // ---- staged return: inverse of the move -------------------------------------------------
@@ -315,19 +367,32 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* 
   uint32_t* st_od = reinterpret_cast<uint32_t*>(l1_smem + C::TILE * 8);  // offset | bin << TILE_SHIFT
   uint32_t* bin_start = st_od + C::TILE;
   uint32_t* gbase = bin_start + C::BINS;
+  uint32_t* pp = gbase + C::BINS;  // prefetch stage: the next tile's packed ranks
   __shared__ uint32_t tmp[C::NT / 32 + 1];
+  __shared__ __align__(8) uint64_t bar;
   uint64_t tb, te;
   l1_tile_range(n, C::TILE, &tb, &te);
+  const bool pf = HM_L1_PREFETCH;
+  if (pf && threadIdx.x == 0) {
+    mbar_init(&bar, 1);
+    if (tb < te) bulk_load(pp, packed + tb * C::TILE, tile_bytes<C>(tb, n, 4), &bar);
+  }
+  __syncthreads();  // barrier initialised before anyone waits on it
+  uint32_t phase = 0;
   uint32_t run[C::BPT];
 #pragma unroll
   for (int k = 0; k < C::BPT; ++k) run[k] = cta_base[(uint64_t)blockIdx.x * C::BINS + threadIdx.x * C::BPT + k];
   for (uint64_t tile = tb; tile < te; ++tile) {
     const uint64_t t0 = tile * C::TILE;
     uint32_t pk[C::PER];
+    if (pf) {
+      mbar_wait(&bar, phase);
+      phase ^= 1;
+    }
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
-      pk[k] = e < n ? __ldg(packed + e) : 0;
+      pk[k] = e < n ? (pf ? pp[k * C::NT + threadIdx.x] : __ldg(packed + e)) : 0;
     }
     {
       uint32_t cv[C::BPT], ex[C::BPT];
@@ -342,6 +407,8 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* 
       }
     }
     __syncthreads();
+    if (pf && threadIdx.x == 0 && tile + 1 < te)
+      bulk_load(pp, packed + (tile + 1) * C::TILE, tile_bytes<C>(tile + 1, n, 4), &bar);
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
@@ -374,7 +441,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* 
 }
 template <class C>
 constexpr size_t unmove_smem() {
-  return (size_t)C::TILE * 12 + 2 * C::BINS * 4;
+  return (size_t)C::TILE * 12 + 2 * C::BINS * 4 + (HM_L1_PREFETCH ? (size_t)C::TILE * 4 : 0);
 }
 
 // ---- level 2: chunk-local sort by the N-bit bucket (two stable LSD passes) ---------------
@@ -494,7 +561,11 @@ __global__ void __launch_bounds__(kSortThreads, 2) k_psa2_local_sort(uint64_t* _
 }
 
 constexpr int kLocalBins = 1 << kLocalBits;
-constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12;
+#ifndef HM_SORT_PREFETCH
+#define HM_SORT_PREFETCH 1
+#endif
+// local histogram, sorted keys + positions, and (prefetch) the next chunk's staged queries
+constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12 + (HM_SORT_PREFETCH ? kChunk * 8 : 0);
 #include "psa2_count_sort.inc"
 
 // level-1 grid: persistent CTAs, ~2048 resident threads per SM, at most one CTA per tile
