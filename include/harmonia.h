@@ -274,6 +274,39 @@ harmonia_status harmonia_route_return(uint32_t P, const uint64_t* d_back, uint64
 harmonia_status harmonia_segments_push(const uint64_t* d_src, uint32_t nseg, const uint64_t* h_src_off,
                                        const uint64_t* h_len, const uint64_t* h_dst, void* d_workspace,
                                        size_t workspace_bytes, void* stream);
+/* ---------------------------------------------------------------------------------------
+ * Range queries over key-range shards (partitioned mode; C-A10).  A range
+ * [lo, hi] is cut at every splitter it crosses: its piece on shard d is
+ * [max(lo, s_{d-1}), min(hi, s_d - 1)] (s = d_splitters, P-1 strictly increasing; shard d owns
+ * [s_{d-1}, s_d)); lo > hi gives one piece on dest(lo) that answers count 0.  Pieces of range
+ * i get ids pbase[i] .. pbase[i+1]-1 in shard (= key) order.
+ * harmonia_range_split_count: d_npieces[n+1] (per range, [n] = 0), d_pbase[n+1] (exclusive
+ *   prefix: piece ids), h_counts[P] pieces per destination, *h_total = pieces (host, sync).
+ * harmonia_range_split_emit (same workspace, after _count): the pieces destination-major:
+ *   d_plo/d_phi[total] and their ids d_pid[total]; order inside a destination's run is
+ *   unspecified.
+ *   (caller) route the pieces to their shards, run harmonia_range_batch there with the same
+ *   cap, bring the answers back in the routed order.
+ * harmonia_range_assemble: for the m = total routed answers (d_counts[m] true totals,
+ *   d_keys/d_values[m][cap] slabs, d_pid[m] their piece ids), range i receives its pieces'
+ *   records in shard order, cut at cap (d_keys_out/d_values_out[n][cap]; entries past the
+ *   count are not written) and d_total_out[i] = the summed true count.  d_row_scratch: m
+ *   uint32.  Asynchronous.
+ * ------------------------------------------------------------------------------------- */
+size_t harmonia_range_split_workspace_bytes(uint64_t n);
+harmonia_status harmonia_range_split_count(const uint64_t* d_splitters, uint32_t P, const uint64_t* d_lo,
+                                           const uint64_t* d_hi, uint64_t n, uint32_t* d_npieces,
+                                           uint32_t* d_pbase, uint64_t* h_counts, uint64_t* h_total,
+                                           void* d_workspace, size_t workspace_bytes, void* stream);
+harmonia_status harmonia_range_split_emit(const uint64_t* d_splitters, uint32_t P, const uint64_t* d_lo,
+                                          const uint64_t* d_hi, uint64_t n, const uint32_t* d_pbase,
+                                          uint64_t* d_plo, uint64_t* d_phi, uint32_t* d_pid,
+                                          void* d_workspace, size_t workspace_bytes, void* stream);
+harmonia_status harmonia_range_assemble(uint64_t n, uint32_t cap, const uint32_t* d_pbase,
+                                        const uint32_t* d_pid, uint64_t m, const uint32_t* d_counts,
+                                        const uint64_t* d_keys, const uint64_t* d_values,
+                                        uint32_t* d_row_scratch, uint64_t* d_keys_out,
+                                        uint64_t* d_values_out, uint64_t* d_total_out, void* stream);
 harmonia_status harmonia_peer_alloc(size_t bytes, void** d_ptr, void* handle_out);
 harmonia_status harmonia_peer_open(const void* handle, void** d_ptr);
 harmonia_status harmonia_peer_close(void* d_ptr);

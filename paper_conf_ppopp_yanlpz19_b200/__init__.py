@@ -108,6 +108,13 @@ def lib():
             "harmonia_route_return": (C.c_int, [C.c_uint32, _vp, _u64, _vp, _vp, _sz, _vp]),
             "harmonia_segments_push": (C.c_int, [_vp, C.c_uint32, _vp, _vp, _vp, _vp, _sz, _vp]),
             "harmonia_peer_alloc": (C.c_int, [_sz, C.POINTER(_vp), _vp]),
+            "harmonia_range_split_workspace_bytes": (_sz, [_u64]),
+            "harmonia_range_split_count": (C.c_int, [_vp, C.c_uint32, _vp, _vp, _u64, _vp, _vp, _vp,
+                                                     C.POINTER(_u64), _vp, _sz, _vp]),
+            "harmonia_range_split_emit": (C.c_int, [_vp, C.c_uint32, _vp, _vp, _u64, _vp, _vp, _vp, _vp, _vp,
+                                                    _sz, _vp]),
+            "harmonia_range_assemble": (C.c_int, [_u64, C.c_uint32, _vp, _vp, _u64, _vp, _vp, _vp, _vp, _vp, _vp,
+                                                  _vp, _vp]),
             "harmonia_peer_open": (C.c_int, [_vp, C.POINTER(_vp)]),
             "harmonia_peer_close": (C.c_int, [_vp]),
             "harmonia_peer_free": (C.c_int, [_vp]),
@@ -489,3 +496,49 @@ class PeerBuffer:
         if self.ptr.value:
             _check(lib().harmonia_peer_free(self.ptr), "harmonia_peer_free")
             self.ptr = C.c_void_p()
+
+
+# ----------------------------------------------------------------------------- range routing
+def range_split(splitters, P: int, lo, hi, stream=None):
+    """Cut ranges at the shard splitters (harmonia_range_split_count + _emit).
+    Returns (plo, phi, pid, counts per destination, pbase): the pieces destination-major."""
+    torch = _torch()
+    dev, n = lo.device, lo.numel()
+    npieces = torch.empty(n + 1, dtype=torch.uint32, device=dev)
+    pbase = torch.empty(n + 1, dtype=torch.uint32, device=dev)
+    ws_b = lib().harmonia_range_split_workspace_bytes(n)
+    ws = torch.empty(ws_b, dtype=torch.uint8, device=dev)
+    counts, total = (C.c_uint64 * P)(), C.c_uint64(0)
+    sp = splitters.data_ptr() if P > 1 else None
+    st = _stream_ptr(stream, dev)
+    _check(lib().harmonia_range_split_count(sp, P, lo.data_ptr(), hi.data_ptr(), n, npieces.data_ptr(),
+                                            pbase.data_ptr(), counts, C.byref(total), ws.data_ptr(), ws_b, st),
+           "harmonia_range_split_count")
+    m = int(total.value)
+    plo = torch.empty(m, dtype=torch.uint64, device=dev)
+    phi = torch.empty(m, dtype=torch.uint64, device=dev)
+    pid = torch.empty(m, dtype=torch.uint32, device=dev)
+    if n:
+        _check(lib().harmonia_range_split_emit(sp, P, lo.data_ptr(), hi.data_ptr(), n, pbase.data_ptr(),
+                                               plo.data_ptr(), phi.data_ptr(), pid.data_ptr(), ws.data_ptr(), ws_b,
+                                               st), "harmonia_range_split_emit")
+    return plo, phi, pid, [int(c) for c in counts], pbase
+
+
+def range_assemble(n: int, cap: int, pbase, pid, counts, keys, values, stream=None):
+    """Reassemble routed range answers (harmonia_range_assemble): (keys [n, cap], values [n, cap],
+    totals [n] uint64); slab entries past a range's count hold PAD / NOT_FOUND."""
+    torch = _torch()
+    dev = pbase.device
+    m = pid.numel()
+    ko = torch.full((n, cap), KEY_PAD, dtype=torch.uint64, device=dev) if cap else None
+    vo = torch.full((n, cap), NOT_FOUND, dtype=torch.uint64, device=dev) if cap else None
+    tot = torch.empty(n, dtype=torch.uint64, device=dev)
+    rows = torch.empty(max(m, 1), dtype=torch.uint32, device=dev)
+    _check(lib().harmonia_range_assemble(n, cap, pbase.data_ptr(), pid.data_ptr() if m else None, m,
+                                         counts.data_ptr() if m else None,
+                                         keys.data_ptr() if (cap and m) else None,
+                                         values.data_ptr() if (cap and m) else None, rows.data_ptr(),
+                                         ko.data_ptr() if cap else None, vo.data_ptr() if cap else None,
+                                         tot.data_ptr(), _stream_ptr(stream, dev)), "harmonia_range_assemble")
+    return ko, vo, tot

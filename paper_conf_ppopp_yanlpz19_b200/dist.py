@@ -27,7 +27,7 @@ from __future__ import annotations
 import torch
 import torch.distributed as dist
 
-from . import Tree, route_partition, route_update_payload, scatter_results
+from . import Tree, range_assemble, range_split, route_partition, route_update_payload, scatter_results
 
 __all__ = ["ReplicatedTree", "PartitionedTree", "PeerPartitionedTree", "CudaOps", "CudaPeerOps", "key_splitters",
            "peer_offsets"]
@@ -81,6 +81,12 @@ class CudaOps:
 
     def update(self, ops, keys, values, seq):
         self.tree.update(ops, keys, values, seq=seq)
+
+    def range_split(self, lo, hi):
+        return range_split(self.split, self.P, lo, hi)
+
+    def range_assemble(self, n, cap, pbase, pid, counts, keys, values):
+        return range_assemble(n, cap, pbase, pid, counts, keys, values)
 
 
 def _routed_update(tree_like, ops, keys, values):
@@ -175,36 +181,16 @@ class PartitionedTree:
     # ------------------------------------------------------------------ range queries
     def range(self, lo: torch.Tensor, hi: torch.Tensor, cap: int):
         """Inclusive ranges; a range crossing splitters is answered piecewise by every shard it
-        touches; pieces are concatenated in shard order (= key order) and the slab is cut at
-        `cap`.  Returns (keys [n, cap] uint64, values [n, cap] uint64, counts [n] int64 = true
-        totals); slab entries past the count hold PAD / NOT_FOUND."""
-        P, dev, n = self.world, lo.device, lo.numel()
-        sign = torch.tensor(-(1 << 63), dtype=torch.int64, device=dev)
-        ulo, uhi = _i64(lo) ^ sign, _i64(hi) ^ sign          # unsigned order as signed order
-        spi = _u64_words(self.splitters, dev)
-        if P > 1:
-            d_lo = torch.searchsorted(spi ^ sign, ulo, right=True)
-            d_hi = torch.searchsorted(spi ^ sign, uhi, right=True)
-        else:
-            d_lo = d_hi = torch.zeros(n, dtype=torch.int64, device=dev)
-        npieces = torch.where(ulo > uhi, torch.ones_like(d_lo), d_hi - d_lo + 1)
-        first_of_q = torch.cumsum(npieces, 0) - npieces
-        qid = torch.repeat_interleave(torch.arange(n, device=dev), npieces)
-        off = torch.arange(qid.numel(), device=dev) - first_of_q[qid]
-        shard = d_lo[qid] + off
-        plo, phi = _i64(lo)[qid].clone(), _i64(hi)[qid].clone()
-        if P > 1:
-            first = off > 0
-            plo[first] = spi[shard[first] - 1]
-            last = off < (npieces[qid] - 1)
-            phi[last] = spi[shard[last]] - 1                # splitter keys belong to the upper shard
-        order = torch.argsort(shard, stable=True)
-        counts = torch.bincount(shard, minlength=P)
-        send_n = counts.tolist()
-        recv_counts = torch.empty(P, dtype=torch.int64, device=dev)
-        dist.all_to_all_single(recv_counts, counts.to(torch.int64), group=self.group)
+        touches (harmonia_range_split_*), pieces are concatenated in shard order (= key order)
+        and the slab is cut at `cap` (harmonia_range_assemble).  Returns (keys [n, cap] uint64,
+        values [n, cap] uint64, counts [n] = true totals); slab entries past the count hold
+        PAD / NOT_FOUND."""
+        n, dev = lo.numel(), lo.device
+        plo, phi, pid, send_n, pbase = self.ops.range_split(lo, hi)   # kernels: cut + dest-major
+        recv_counts = torch.empty(self.world, dtype=torch.int64, device=dev)
+        dist.all_to_all_single(recv_counts, torch.tensor(send_n, dtype=torch.int64, device=dev), group=self.group)
         rc = recv_counts.tolist()
-        pieces = torch.stack([plo[order], phi[order]], 1).contiguous()
+        pieces = torch.stack([_i64(plo), _i64(phi)], 1).contiguous()
         recv_p = torch.empty(sum(rc), 2, dtype=torch.int64, device=dev)
         dist.all_to_all_single(recv_p, pieces, output_split_sizes=rc, input_split_sizes=send_n, group=self.group)
         m = recv_p.shape[0]
@@ -213,24 +199,12 @@ class PartitionedTree:
         if cap:
             cols = [_i64(ko).reshape(m, cap), _i64(vo).reshape(m, cap)] + cols
         payload = torch.cat(cols, 1).contiguous()
-        back = torch.empty(qid.numel(), payload.shape[1], dtype=torch.int64, device=dev)
+        back = torch.empty(plo.numel(), payload.shape[1], dtype=torch.int64, device=dev)
         dist.all_to_all_single(back, payload, output_split_sizes=send_n, input_split_sizes=rc, group=self.group)
-        res = torch.empty_like(back)
-        res[order] = back                                     # pieces back in (query, shard) order
-        pc = res[:, -1]
-        total = torch.zeros(n, dtype=torch.int64, device=dev).index_add_(0, qid, pc)
-        out_k = torch.full((n, cap), -1, dtype=torch.int64, device=dev)
-        out_v = torch.full((n, cap), -1, dtype=torch.int64, device=dev)
-        if cap:
-            S = torch.cumsum(pc, 0) - pc
-            before = S - S[first_of_q[qid]]                   # records of earlier pieces of the query
-            t = torch.arange(cap, device=dev)
-            slot = before[:, None] + t[None, :]
-            valid = (t[None, :] < torch.clamp(pc, max=cap)[:, None]) & (slot < cap)
-            rows = qid[:, None].expand(-1, cap)[valid]
-            out_k[rows, slot[valid]] = res[:, :cap][valid]
-            out_v[rows, slot[valid]] = res[:, cap:2 * cap][valid]
-        return _u64(out_k), _u64(out_v), total
+        bc = back[:, -1].to(torch.int32).contiguous()
+        bk = _u64(back[:, :cap].contiguous()) if cap else None
+        bv = _u64(back[:, cap:2 * cap].contiguous()) if cap else None
+        return self.ops.range_assemble(n, cap, pbase, pid, bc, bk, bv)   # kernel: shard order, cap
 
 
 # ------------------------------------------------------------------ fused routing (peer memory)

@@ -65,6 +65,54 @@ class CpuOps:
         out[pos] = vals.view(torch.int64)
         return out.view(torch.uint64)
 
+    def range_split(self, lo, hi):
+        # cut at the splitters (the semantics of harmonia_range_split_*), destination-major,
+        # and deliberately scrambled inside each destination's run (the kernel's order is
+        # unspecified; the piece ids carry the order)
+        l = lo.view(torch.int64).numpy().view(np.uint64)
+        h = hi.view(torch.int64).numpy().view(np.uint64)
+        d0 = np.searchsorted(self.split, l, side="right")
+        np_ = np.where(l > h, 1, np.searchsorted(self.split, h, side="right") - d0 + 1)
+        pbase = np.concatenate([[0], np.cumsum(np_)]).astype(np.uint32)
+        plo, phi, dest, pid = [], [], [], []
+        for i in range(len(l)):
+            for j in range(int(np_[i])):
+                d = int(d0[i]) + j
+                a, b = l[i], h[i]
+                if l[i] <= h[i]:
+                    if j > 0:
+                        a = self.split[d - 1]
+                    if j + 1 < np_[i]:
+                        b = self.split[d] - np.uint64(1)
+                plo.append(a), phi.append(b), dest.append(d), pid.append(pbase[i] + j)
+        dest = np.asarray(dest, dtype=np.int64)
+        order = np.lexsort((-np.arange(len(dest)), dest))
+        t = lambda a, dt: torch.from_numpy(np.asarray(a, dtype=dt)[order].copy())
+        return (t(plo, np.uint64).view(torch.int64).view(torch.uint64), t(phi, np.uint64).view(torch.int64).view(torch.uint64),
+                t(pid, np.uint32).to(torch.int64), np.bincount(dest, minlength=self.P).tolist(), torch.from_numpy(pbase))
+
+    def range_assemble(self, n, cap, pbase, pid, counts, keys, values):
+        pb, pid = pbase.numpy(), pid.numpy()
+        row_of = np.empty(len(pid), dtype=np.int64)
+        row_of[pid] = np.arange(len(pid))
+        c = counts.numpy().astype(np.int64)
+        k = keys.view(torch.int64).numpy().reshape(-1, cap) if cap else None
+        v = values.view(torch.int64).numpy().reshape(-1, cap) if cap else None
+        ko = np.full((n, cap), -1, dtype=np.int64)
+        vo = np.full((n, cap), -1, dtype=np.int64)
+        tot = np.zeros(n, dtype=np.int64)
+        for i in range(n):
+            f = 0
+            for p in range(pb[i], pb[i + 1]):
+                r = row_of[p]
+                tot[i] += c[r]
+                take = min(c[r], cap - f) if f < cap else 0
+                if take:
+                    ko[i, f:f + take] = k[r, :take]
+                    vo[i, f:f + take] = v[r, :take]
+                f += take
+        return torch.from_numpy(ko).view(torch.uint64), torch.from_numpy(vo).view(torch.uint64), torch.from_numpy(tot)
+
     def route_update(self, ops, keys, values, rank):
         kn = keys.view(torch.int64).numpy().view(np.uint64)
         dest = np.searchsorted(self.split, kn, side="right")
@@ -109,8 +157,8 @@ def _worker(rank, world, port, T, cap, result_q):
         # ranges: short, long (crossing several shards), empty, lo > hi, full span
         lo1, hi1 = gen.ranges(keys, 200, 40, seed=gen.SEED_RANGE + rank)
         lo2, hi2 = gen.random_ranges(keys, 200, seed=gen.SEED_RANGE + 7 * rank, max_width_keys=T)
-        lo = np.concatenate([lo1, lo2, [0, 5, int(keys[-1])], np.asarray(sp, dtype=np.uint64)])
-        hi = np.concatenate([hi1, hi2, [(1 << 64) - 1, 4, (1 << 64) - 1],
+        lo = np.concatenate([lo1, lo2, np.array([0, 5, int(keys[-1])], dtype=np.uint64), np.asarray(sp, dtype=np.uint64)])
+        hi = np.concatenate([hi1, hi2, np.array([(1 << 64) - 1, 4, (1 << 64) - 1], dtype=np.uint64),
                              np.asarray(sp, dtype=np.uint64) + np.uint64(3)])
         lo, hi = lo.astype(np.uint64), hi.astype(np.uint64)
         tl = torch.from_numpy(lo.view(np.int64).copy()).view(torch.uint64)

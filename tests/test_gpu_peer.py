@@ -123,3 +123,46 @@ def test_peer_partitioned_two_processes_ipc(world):
         p.join(timeout=120)
     for rank, ok, err in res:
         assert ok, f"rank {rank}: {err or 'peer-routed results differ from the oracle'}"
+
+
+@pytest.mark.parametrize("P,cap", [(1, 16), (3, 0), (4, 64), (16, 32)])
+def test_range_split_assemble_single_process(hm, orc, P, cap):
+    """harmonia_range_split_count/_emit cut ranges at the splitters, P shard trees answer their
+    pieces (harmonia_range_batch), harmonia_range_assemble reassembles: equal to the oracle on
+    the whole key set (slab contents up to min(count, cap) and true totals)."""
+    T = 40000
+    keys = gen.uniform_keys(T)
+    vals = gen.values_for(keys)
+    sp = [int(keys[(p * T) // P]) for p in range(1, P)]
+    bnd = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
+    trees = [hm.Tree(_u64(keys[bnd[d]:bnd[d + 1]]), _u64(vals[bnd[d]:bnd[d + 1]]), fanout=16) for d in range(P)]
+    lo1, hi1 = gen.ranges(keys, 3000, 40)
+    lo2, hi2 = gen.random_ranges(keys, 3000, max_width_keys=T)
+    spa = np.asarray(sp, dtype=np.uint64)
+    lo = np.concatenate([lo1, lo2, np.array([0, 5, int(keys[-1])], dtype=np.uint64), spa, spa - np.uint64(1)]).astype(np.uint64)
+    hi = np.concatenate([hi1, hi2, np.array([(1 << 64) - 1, 4, (1 << 64) - 1], dtype=np.uint64), spa + np.uint64(3), spa]).astype(np.uint64)
+    spd = _u64(spa if P > 1 else np.zeros(1, np.uint64))
+    plo, phi, pid, counts, pbase = hm.range_split(spd, P, _u64(lo), _u64(hi))
+    m = plo.numel()
+    assert sum(counts) == m
+    rc = torch.empty(m, dtype=torch.int32, device="cuda")
+    rk = torch.empty(max(m * cap, 1), dtype=torch.uint64, device="cuda")
+    rv = torch.empty(max(m * cap, 1), dtype=torch.uint64, device="cuda")
+    start = 0
+    for d in range(P):  # each destination run answered by its shard
+        c = counts[d]
+        if c:
+            ko, vo, cnt = trees[d].range(plo[start:start + c], phi[start:start + c], cap)
+            rc[start:start + c] = cnt.view(torch.int32)
+            if cap:
+                rk[start * cap:(start + c) * cap] = ko.reshape(-1)
+                rv[start * cap:(start + c) * cap] = vo.reshape(-1)
+        start += c
+    ko, vo, tot = hm.range_assemble(len(lo), cap, pbase, pid, rc, rk, rv)
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, cap)
+    assert np.array_equal(_np(tot), ecnt.astype(np.uint64))
+    if cap:
+        mk = np.arange(cap)[None, :] < np.minimum(ecnt.astype(np.int64), cap)[:, None]
+        gk, gv = _np(ko).reshape(-1, cap), _np(vo).reshape(-1, cap)
+        assert np.array_equal(gk[mk], eko.reshape(-1, cap)[mk]) and np.array_equal(gv[mk], evo.reshape(-1, cap)[mk])
+        assert np.all(gk[~mk] == np.uint64((1 << 64) - 1))
