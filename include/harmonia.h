@@ -95,6 +95,10 @@ typedef struct {
                                       the default warp-shared descent (the warp's PSA-ordered
                                       queries share the path down to the level where their
                                       key interval splits)                           */
+#define HARMONIA_QF_RANGE_GROUP 2048u /* ranges: the G-lane group walk of the leaves (one
+                                      load-ballot-store step per 2G slots) instead of the
+                                      default warp-per-range resolve-then-copy kernel; also
+                                      implied by an explicit group_size                      */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic

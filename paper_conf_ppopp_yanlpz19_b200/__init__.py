@@ -30,6 +30,7 @@ QF_FUSE_SORT = 128
 QF_SCATTER_RETURN = 256
 QF_PSA_WIDE = 512
 QF_PER_LANE = 1024
+QF_RANGE_GROUP = 2048
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
            6: "DEVICE_MISMATCH", 7: "TOO_LARGE"}
 
@@ -340,14 +341,20 @@ class Tree:
                                                 ws.data_ptr(), ws_b, C.byref(o), st), "harmonia_search_batch_host")
         return out_host
 
-    def range(self, lo, hi, cap: int, *, opts: QueryOpts | None = None, stream=None, **kw):
-        """Inclusive range queries: (keys [n, cap], values [n, cap], counts [n] uint32)."""
+    def range(self, lo, hi, cap: int, *, out=None, opts: QueryOpts | None = None, stream=None, **kw):
+        """Inclusive range queries: (keys [n, cap], values [n, cap], counts [n] uint32).
+        Without `out`, fresh slabs pre-filled with PAD / NOT_FOUND are returned; with
+        out=(keys, values, counts) those buffers are written as the C ABI does (slab entries
+        past a range's count are left untouched)."""
         torch = _torch()
         lo, hi = _as_u64_dev(lo, self.device), _as_u64_dev(hi, self.device)
         n = lo.numel()
-        ko = torch.full((n, cap), KEY_PAD, dtype=torch.uint64, device=self.device) if cap else None
-        vo = torch.full((n, cap), NOT_FOUND, dtype=torch.uint64, device=self.device) if cap else None
-        cnt = torch.empty(n, dtype=torch.uint32, device=self.device)
+        if out is not None:
+            ko, vo, cnt = out
+        else:
+            ko = torch.full((n, cap), KEY_PAD, dtype=torch.uint64, device=self.device) if cap else None
+            vo = torch.full((n, cap), NOT_FOUND, dtype=torch.uint64, device=self.device) if cap else None
+            cnt = torch.empty(n, dtype=torch.uint32, device=self.device)
         o = opts if opts is not None else make_opts(**kw)
         ws_b = lib().harmonia_range_workspace_bytes(self._h, n, C.byref(o))
         ws = self._workspace(ws_b)

@@ -88,6 +88,9 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
           2 * (round_up(P.smem_bytes, 16) + kPsaChunk * 8 + 1024) <= t->smem_per_sm;
   P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
   P.coop = P.ret && !(o->flags & HARMONIA_QF_PER_LANE);
+  // ranges: the warp-per-range copy kernel unless a group size was requested explicitly or
+  // the G-lane group walk is asked for (HARMONIA_QF_RANGE_GROUP)
+  P.range_warp = o->group_size == 0 && !(o->flags & HARMONIA_QF_RANGE_GROUP);
   *p = P;
   return HARMONIA_OK;
 }
@@ -347,6 +350,10 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   a.smem_nodes = p.smem_nodes;
   a.ps_smem_bytes = p.ps_smem ? p.ps_smem_bytes : 0;
   a.cap = cap;
+  // long slabs: one warp per range, resolve then stream-copy (164 vs 128 G records/s at
+  // len 1024, 137 vs 123 at 256); short ones: several ranges per warp in G-lane groups (43 vs
+  // 22 G records/s at len 16), measured at c2
+  p.range_warp = p.range_warp && cap >= 128;
   if (p.g_auto) {  // the leaf scan wants wide groups for long ranges (measured)
     int G = 8;
     while (G < 32 && (uint32_t)(4 * G) < cap) G *= 2;

@@ -139,6 +139,15 @@ struct harmonia_tree {
   uint64_t* d_vals = nullptr;       // leaf-aligned values, L*F
   uint64_t* d_leaf_base = nullptr;  // records before leaf j, L+1 entries (range counts)
   uint64_t min_key = 0, max_key = 0;
+  // capacities of the live arrays, spare arrays of the previous layout (an update builds into
+  // them and hands the old ones back: no cudaMalloc/cudaFree per batch in steady state), and
+  // build scratch (per-level subtree minima)
+  size_t cap_keys = 0, cap_vals = 0, cap_ps = 0, cap_lb = 0;
+  uint64_t *sp_keys = nullptr, *sp_vals = nullptr, *sp_lb = nullptr;
+  uint32_t* sp_ps = nullptr;
+  size_t sp_cap_keys = 0, sp_cap_vals = 0, sp_cap_ps = 0, sp_cap_lb = 0;
+  uint64_t* scratch = nullptr;
+  size_t scratch_cap = 0;
   float fill = 1.0f;
   int sm_count = 148;
   size_t smem_optin = 0;
@@ -175,6 +184,7 @@ struct Plan {
   bool ret = false;          // staged inverse return (chunk-local result staging + unmove)
   bool wide = false;         // staged return with the 11-bit level-1 partition
   bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
+  bool range_warp = true;    // ranges: one warp per range, resolve then stream-copy (k_range_warp)
 };
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
@@ -288,6 +298,10 @@ harmonia_status launch_scatter_back(const uint64_t* vals, const uint32_t* pos, u
 // layout construction (tree.cu)
 harmonia_status build_layout(harmonia_tree* t, const uint64_t* d_keys, const uint64_t* d_vals,
                              uint64_t n, cudaStream_t st);
+// grow a device buffer to >= need bytes (contents not kept); 1/8 headroom on reallocation
+harmonia_status reserve_bytes(void** p, size_t* cap, size_t need);
+// the live arrays become the spares and the spares the live arrays (pointers and capacities)
+void swap_layout_buffers(harmonia_tree* t);
 uint32_t level_shape(uint64_t n, uint32_t F, double fill, uint64_t* bottom_up_nodes);
 
 }  // namespace hm

@@ -957,6 +957,158 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(co
   }
 }
 
+// ---- range scan, one warp per range (default) -------------------------------------------
+// The range is resolved first and copied second (find the first target key, scan the
+// key region to the last):
+//   1. a joint warp-cooperative descent of lo and hi (one 128-bit load per lane and two
+//      ballots per level while both bounds share the node) gives their leaves and in-leaf
+//      ranks, so R0 = rank of the first key >= lo and R1 = rank past the last key <= hi come
+//      from leaf_base: count = R1 - R0 exactly, with no second pass for truncated slabs;
+//   2. min(count, cap) records are copied leaf by leaf, kRangeBatch leaves per round with
+//      all their key, value and leaf_base loads in flight at once -- the copy is a stream
+//      over contiguous leaves, so it runs at memory speed instead of one dependent
+//      load-ballot-store step per leaf.
+constexpr int kRangeLeaves = 4;  // leaves in flight per warp (F <= 64; fewer for wider nodes)
+
+template <int F, bool SMEM, bool STRICT>
+__device__ __forceinline__ uint32_t warp_rank1(const uint64_t* nk, uint64_t q) {
+  uint32_t rl, rh;
+  coop_rank<F, SMEM, STRICT>(nk, q, q, rl, rh);
+  return STRICT ? rl : rh;
+}
+
+template <int F>
+__global__ void __launch_bounds__(1024, 1) k_range_warp(const RangeArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  constexpr int NP = F >= 64 ? F / 64 : 1;  // 128-bit slot pairs per lane per leaf
+  constexpr int kRangeBatch = kRangeLeaves / NP > 0 ? kRangeLeaves / NP : 1;
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t cap = a.cap;
+  const uint64_t ls = a.leaf_start, nleaves = a.n_nodes - a.leaf_start;
+  for (uint64_t j = warp; j < a.n; j += nwarps) {
+    const uint64_t lo = ld_stream(a.lo + j);
+    const uint64_t slab = a.idx ? (uint64_t)ld_stream32(a.idx + j) : j;
+    uint64_t hi = __ldg(a.hi + slab);
+    uint64_t count = 0;
+    if (lo <= hi && lo != kPad) {
+      if (hi == kPad) hi = kPad - 1;  // no key equals PAD, and PAD slots must not count
+      // 1. joint descent of lo (rank: keys < lo at the leaf) and hi (keys <= hi)
+      uint32_t nlo = 0, nhi = 0;
+      for (uint32_t l = 0; l + 1 < a.h; ++l) {
+        const bool sm = l < a.smem_levels;
+        const uint64_t* base = sm ? s_keys : a.keys;
+        uint32_t rl, rh;
+        if (nlo == nhi) {
+          if (sm) coop_rank<F, true, false>(base + (uint64_t)nlo * F, lo, hi, rl, rh);
+          else coop_rank<F, false, false>(base + (uint64_t)nlo * F, lo, hi, rl, rh);
+        } else {
+          rl = sm ? warp_rank1<F, true, false>(base + (uint64_t)nlo * F, lo)
+                  : warp_rank1<F, false, false>(base + (uint64_t)nlo * F, lo);
+          rh = sm ? warp_rank1<F, true, false>(base + (uint64_t)nhi * F, hi)
+                  : warp_rank1<F, false, false>(base + (uint64_t)nhi * F, hi);
+        }
+        const uint32_t flo = ps_smem ? s_ps[nlo] : __ldg(a.ps + nlo);
+        const uint32_t fhi = ps_smem ? s_ps[nhi] : __ldg(a.ps + nhi);
+        nlo = flo + rl;  // Eq 1
+        nhi = fhi + rh;
+      }
+      uint32_t s0, s1;
+      {
+        const uint64_t* base = leaf_smem ? s_keys : a.keys;
+        if (nlo == nhi) {
+          if (leaf_smem) coop_rank<F, true, true>(base + (uint64_t)nlo * F, lo, hi, s0, s1);
+          else coop_rank<F, false, true>(base + (uint64_t)nlo * F, lo, hi, s0, s1);
+        } else {
+          s0 = leaf_smem ? warp_rank1<F, true, true>(base + (uint64_t)nlo * F, lo)
+                         : warp_rank1<F, false, true>(base + (uint64_t)nlo * F, lo);
+          s1 = leaf_smem ? warp_rank1<F, true, false>(base + (uint64_t)nhi * F, hi)
+                         : warp_rank1<F, false, false>(base + (uint64_t)nhi * F, hi);
+        }
+      }
+      const uint64_t r0 = __ldg(a.leaf_base + (nlo - ls)) + s0;
+      const uint64_t r1 = __ldg(a.leaf_base + (nhi - ls)) + s1;
+      count = r1 - r0;
+      // 2. copy min(count, cap) records, leaf by leaf from (nlo, s0)
+      const uint64_t ncopy = count < cap ? count : cap;
+      uint64_t* ko = a.kout + slab * cap;
+      uint64_t* vo = a.vout + slab * cap;
+      uint64_t leaf = nlo - ls, o = 0;
+      uint32_t sfirst = s0;
+      while (o < ncopy) {
+        // leaf_base[leaf .. leaf + kRangeBatch] (record counts of the batch's leaves)
+        const uint64_t lbi = leaf + lane;
+        const uint64_t lbv = (lane <= (unsigned)kRangeBatch && lbi <= nleaves) ? __ldg(a.leaf_base + lbi) : 0;
+        ulonglong2 kk[kRangeBatch][NP], vv[kRangeBatch][NP];
+#pragma unroll
+        for (int b = 0; b < kRangeBatch; ++b)
+#pragma unroll
+          for (int p = 0; p < NP; ++p) {
+            const uint32_t slot = p * 64 + 2 * lane;
+            const bool ok = leaf + b < nleaves && (F >= 64 || slot < F);
+            kk[b][p] = ok ? ld_pair_global(a.keys + (ls + leaf + b) * F + slot) : make_ulonglong2(kPad, kPad);
+            vv[b][p] = ok ? ld_pair_global(a.vals + (leaf + b) * F + slot) : make_ulonglong2(0, 0);
+          }
+#pragma unroll
+        for (int b = 0; b < kRangeBatch; ++b) {
+          const uint64_t b0 = __shfl_sync(kFull, lbv, b), b1 = __shfl_sync(kFull, lbv, b + 1);
+          if (o < ncopy && leaf + b < nleaves) {
+            const uint32_t c = (uint32_t)(b1 - b0);  // valid keys occupy slots [0, c) (I6)
+            const uint32_t st = b == 0 ? sfirst : 0;
+            const uint64_t room = ncopy - o;
+            const uint32_t end = (uint64_t)(c - (st < c ? st : c)) < room ? c : st + (uint32_t)room;
+            const int64_t base = (int64_t)o - st;  // output index of slot 0
+#pragma unroll
+            for (int p = 0; p < NP; ++p) {
+              const uint32_t slot = p * 64 + 2 * lane;
+              if (slot >= st && slot < end) {
+                ko[base + slot] = kk[b][p].x;
+                vo[base + slot] = vv[b][p].x;
+              }
+              if (slot + 1 >= st && slot + 1 < end) {
+                ko[base + slot + 1] = kk[b][p].y;
+                vo[base + slot + 1] = vv[b][p].y;
+              }
+            }
+            o += end > st ? end - st : 0;
+          }
+        }
+        leaf += kRangeBatch;
+        sfirst = 0;
+      }
+    }
+    if (lane == 0) a.counts[slab] = (uint32_t)(count > 0xFFFFFFFFull ? 0xFFFFFFFFull : count);
+  }
+}
+
+template <int F>
+harmonia_status launch_range_warp_f(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
+  auto kern = k_range_warp<F>;
+  static int configured_smem = -1;
+  if ((int)p.smem_bytes > configured_smem) {
+    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
+    configured_smem = (int)p.smem_bytes;
+  }
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, p.smem_bytes));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t need = ceil_div(a.n, (uint64_t)32);
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
+  {
+    ProfScope ps_(HARMONIA_PROF_RANGE, st);
+    kern<<<grid, 1024, p.smem_bytes, st>>>(a);
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
 template <int F>
 harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
   auto kern = a.staged ? k_sort_search<F, true> : k_sort_search<F, false>;
@@ -1140,6 +1292,18 @@ harmonia_status launch_search(const harmonia_tree* t, const Plan& p, const Searc
 
 harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
   if (a.n == 0) return HARMONIA_OK;
+  if (p.range_warp) {
+    switch (t->F) {
+      case 4: return launch_range_warp_f<4>(t, p, a, st);
+      case 8: return launch_range_warp_f<8>(t, p, a, st);
+      case 16: return launch_range_warp_f<16>(t, p, a, st);
+      case 32: return launch_range_warp_f<32>(t, p, a, st);
+      case 64: return launch_range_warp_f<64>(t, p, a, st);
+      case 128: return launch_range_warp_f<128>(t, p, a, st);
+      case 256: return launch_range_warp_f<256>(t, p, a, st);
+    }
+    return HARMONIA_ERR_INVALID_ARG;
+  }
   const int G = p.G == 1 ? 2 : p.G;  // ranges scan leaves with at least a lane pair
   HM_DISPATCH(launch_range_fg, t->F, G, t, p, a, st)
 }

@@ -138,10 +138,12 @@ harmonia_status build_layout(harmonia_tree* t, const uint64_t* d_keys, const uin
 
   const size_t kr_bytes = (size_t)t->N * F * 8, lv_bytes = (size_t)t->L * F * 8;
   const size_t ps_bytes = round_up((t->I + 1) * 4, 16);
-  HM_CUDA(cudaMalloc(&t->d_keys, kr_bytes));
-  HM_CUDA(cudaMalloc(&t->d_vals, lv_bytes));
-  HM_CUDA(cudaMalloc(&t->d_ps, ps_bytes));
-  HM_CUDA(cudaMalloc(&t->d_leaf_base, (t->L + 1) * 8));
+  // the layout is built into the tree's current arrays, grown only when too small
+  harmonia_status rs;
+  if ((rs = reserve_bytes((void**)&t->d_keys, &t->cap_keys, kr_bytes)) != HARMONIA_OK) return rs;
+  if ((rs = reserve_bytes((void**)&t->d_vals, &t->cap_vals, lv_bytes)) != HARMONIA_OK) return rs;
+  if ((rs = reserve_bytes((void**)&t->d_ps, &t->cap_ps, ps_bytes)) != HARMONIA_OK) return rs;
+  if ((rs = reserve_bytes((void**)&t->d_leaf_base, &t->cap_lb, (t->L + 1) * 8)) != HARMONIA_OK) return rs;
   HM_CUDA(cudaMemsetAsync(t->d_keys, 0xFF, kr_bytes, st));
   HM_CUDA(cudaMemsetAsync(t->d_vals, 0xFF, lv_bytes, st));
   HM_CUDA(cudaMemsetAsync(t->d_ps, 0, ps_bytes, st));
@@ -151,9 +153,9 @@ harmonia_status build_layout(harmonia_tree* t, const uint64_t* d_keys, const uin
   uint64_t nrec = n;
   HM_CUDA(cudaMemcpyAsync(t->d_leaf_base + t->L, &nrec, 8, cudaMemcpyHostToDevice, st));
 
-  uint64_t *mins_a = nullptr, *mins_b = nullptr;
-  HM_CUDA(cudaMalloc(&mins_a, t->L * 8));
-  HM_CUDA(cudaMalloc(&mins_b, t->L * 8));
+  if ((rs = reserve_bytes((void**)&t->scratch, &t->scratch_cap, 2 * round_up(t->L * 8, 256))) != HARMONIA_OK)
+    return rs;
+  uint64_t *mins_a = t->scratch, *mins_b = t->scratch + round_up(t->L * 8, 256) / 8;
   harmonia_status s = HARMONIA_OK;
   if (n > 0) {
     k_fill_leaves<<<grid_for(n, t->sm_count), kBlock, 0, st>>>(
@@ -172,10 +174,45 @@ harmonia_status build_layout(harmonia_tree* t, const uint64_t* d_keys, const uin
   }
   cudaError_t e = cudaGetLastError();
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  cudaFree(mins_a);
-  cudaFree(mins_b);
   if (e != cudaSuccess) s = cuda_fail(e);
   return s;
+}
+
+harmonia_status reserve_bytes(void** p, size_t* cap, size_t need) {
+  need = std::max<size_t>(need, 16);
+  if (*p && *cap >= need) return HARMONIA_OK;
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  const size_t want = need + need / 8;
+  cudaError_t e = cudaMalloc(p, want);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    *p = nullptr;
+    if (e == cudaErrorMemoryAllocation) {  // retry without headroom
+      if (cudaMalloc(p, need) == cudaSuccess) {
+        *cap = need;
+        return HARMONIA_OK;
+      }
+      cudaGetLastError();
+      *p = nullptr;
+      return HARMONIA_ERR_OUT_OF_MEMORY;
+    }
+    return cuda_fail(e);
+  }
+  *cap = want;
+  return HARMONIA_OK;
+}
+
+void swap_layout_buffers(harmonia_tree* t) {
+  std::swap(t->d_keys, t->sp_keys);
+  std::swap(t->cap_keys, t->sp_cap_keys);
+  std::swap(t->d_vals, t->sp_vals);
+  std::swap(t->cap_vals, t->sp_cap_vals);
+  std::swap(t->d_ps, t->sp_ps);
+  std::swap(t->cap_ps, t->sp_cap_ps);
+  std::swap(t->d_leaf_base, t->sp_lb);
+  std::swap(t->cap_lb, t->sp_cap_lb);
 }
 
 int psa_bits_for(uint64_t n_keys) {
@@ -199,6 +236,11 @@ static void free_tree(harmonia_tree* t) {
   cudaFree(t->d_vals);
   cudaFree(t->d_ps);
   cudaFree(t->d_leaf_base);
+  cudaFree(t->sp_keys);
+  cudaFree(t->sp_vals);
+  cudaFree(t->sp_ps);
+  cudaFree(t->sp_lb);
+  cudaFree(t->scratch);
   if (t->s_h2d) cudaStreamDestroy(t->s_h2d);
   if (t->s_d2h) cudaStreamDestroy(t->s_d2h);
   if (t->ev_start) cudaEventDestroy(t->ev_start);

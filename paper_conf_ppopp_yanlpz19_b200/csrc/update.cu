@@ -344,22 +344,13 @@ extern "C" harmonia_status harmonia_update_batch_seq(harmonia_tree* t, const uin
     k_upd_merge_ins<<<grid_of(nins, sm), kBlock, 0, st>>>(ik, iv, nins, K, kpos, nk, NK, NV);
     HM_LAUNCHED();
   }
-  // 7. rebuild the layout (new arrays; the old ones are released after the build)
+  // 7. rebuild the layout into the spare arrays (the previous layout's buffers, kept by the
+  // tree); on success the old arrays become the spares, on failure the tree is unchanged
   harmonia_tree old = *t;
-  t->d_keys = nullptr;
-  t->d_vals = nullptr;
-  t->d_ps = nullptr;
-  t->d_leaf_base = nullptr;
+  swap_layout_buffers(t);
   harmonia_status s = build_layout(t, NK, NV, nn, st);
   if (s != HARMONIA_OK) {
-    cudaFree(t->d_keys);
-    cudaFree(t->d_vals);
-    cudaFree(t->d_ps);
-    cudaFree(t->d_leaf_base);
-    t->d_keys = old.d_keys;  // tree unchanged on failure
-    t->d_vals = old.d_vals;
-    t->d_ps = old.d_ps;
-    t->d_leaf_base = old.d_leaf_base;
+    swap_layout_buffers(t);  // live arrays back; whatever build_layout grew stays spare
     t->h = old.h;
     t->N = old.N;
     t->I = old.I;
@@ -368,10 +359,6 @@ extern "C" harmonia_status harmonia_update_batch_seq(harmonia_tree* t, const uin
     for (int l = 0; l <= HARMONIA_MAX_LEVELS; ++l) t->level_start[l] = old.level_start[l];
     return s;
   }
-  cudaFree(old.d_keys);
-  cudaFree(old.d_vals);
-  cudaFree(old.d_ps);
-  cudaFree(old.d_leaf_base);
   if (nn > 0) {
     HM_CUDA(cudaMemcpyAsync(&t->min_key, NK, 8, cudaMemcpyDeviceToHost, st));
     HM_CUDA(cudaMemcpyAsync(&t->max_key, NK + nn - 1, 8, cudaMemcpyDeviceToHost, st));

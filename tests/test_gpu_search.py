@@ -229,6 +229,30 @@ def test_range_parity(hm, orc, F, G, length, cap):
         _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
 
 
+@pytest.mark.parametrize("F,fill", [(4, 1.0), (8, 0.69), (16, 1.0), (32, 0.69), (64, 1.0), (64, 0.69), (128, 1.0),
+                                    (256, 0.69)])
+@pytest.mark.parametrize("length,cap", [(1, 128), (16, 200), (128, 128), (300, 130), (1024, 1024), (5000, 256),
+                                        (50, 0), (64, 64)])
+def test_range_warp_kernel(hm, orc, F, fill, length, cap):
+    """Default range path (k_range_warp: joint descent of lo/hi, counts from leaf_base ranks,
+    batched leaf copy): exact slabs and true totals, ranges starting mid-leaf, spanning many
+    leaves, truncated by the cap, empty, lo > hi, unbounded and PAD bounds."""
+    keys = gen.uniform_keys(50000) if F != 4 else gen.uniform_keys(6000)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F, fill)
+    lo, hi = gen.ranges(keys, 2000, min(length, len(keys)))
+    lo2, hi2 = gen.random_ranges(keys, 2000, max_width_keys=3 * max(cap, 8))
+    lo3 = np.array([0, 0, int(keys[500]), int(keys[-1]), MAX, 5, MAX - 1, int(keys[7]) + 1], dtype=np.uint64)
+    hi3 = np.array([MAX, int(keys[99]), MAX, MAX, MAX, 4, MAX, int(keys[9])], dtype=np.uint64)
+    lo, hi = np.concatenate([lo, lo2, lo3]), np.concatenate([hi, hi2, hi3])
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, cap)
+    for kw in ({}, {"psa_bits": -1}, {"window": 2048}, {"smem_levels": -1}):
+        ko, vo, cnt = t.range(cu(lo), cu(hi), cap, **kw)
+        _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
+    ko, vo, cnt = t.range(cu(lo), cu(hi), cap, flags=hm.QF_RANGE_GROUP)  # the G-lane group walk
+    _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
+
+
 def test_range_unbounded_counts(hm, orc):
     keys = gen.uniform_keys(100000)
     vals = gen.values_for(keys)

@@ -52,10 +52,16 @@ def range_bench(T=1 << 23, F=64, reps=5, groups=(0,), flags=0):
     for length, Qr in ((16, 1 << 22), (64, 1 << 21), (256, 1 << 20), (1024, 1 << 18)):
         lo, hi = gen.ranges(keys, Qr, length)
         lo, hi = torch.from_numpy(lo).cuda(), torch.from_numpy(hi).cuda()
+        outb = (torch.empty((Qr, length), dtype=torch.uint64, device="cuda"),
+                torch.empty((Qr, length), dtype=torch.uint64, device="cuda"),
+                torch.empty(Qr, dtype=torch.uint32, device="cuda"))
         for G in groups:
             o = hm.make_opts(group_size=G, flags=flags)
-            ms = timed(lambda: t.range(lo, hi, length, opts=o), reps)
+            ms = timed(lambda: t.range(lo, hi, length, out=outb, opts=o), reps)  # slabs preallocated
+            cnt = outb[2].cpu().numpy()
+            ok = bool((cnt == length).all())  # lo = key[p], hi = key[p+len-1]: exactly len records
             res.append({"what": "range_batch", "T": T, "F": F, "G": G, "len": length, "Qr": Qr, "ms": ms,
+                        "kernel": "group" if (G or flags & hm.QF_RANGE_GROUP or length < 128) else "warp", "counts_ok": ok,
                         "Gq_per_s": Qr / ms / 1e6, "G_records_per_s": Qr * length / ms / 1e6,
                         "GB_per_s_out": Qr * length * 16 / ms / 1e6})
             print(json.dumps(res[-1]), flush=True)
@@ -94,6 +100,7 @@ if __name__ == "__main__":
     for w in a.what.split(","):
         rows = {"update": update_bench, "range": range_bench,
                 "range_sweep": lambda: range_bench(groups=(2, 4, 8, 16, 32)),
+                "range_group": lambda: range_bench(flags=hm.QF_RANGE_GROUP),
                 "sweep": lambda: sweep_bench(dist=a.sweep_dist)}[w]()
         for r in rows:
             print(json.dumps(r), flush=True)
