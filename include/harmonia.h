@@ -75,7 +75,8 @@ typedef struct {
                            window"): 0 = auto; otherwise rounded to a multiple of 1024 */
   uint32_t lane_queries; /* group_size = 1 only: independent queries interleaved per lane
                            (1, 2 or 4; 0 = auto)                                            */
-  uint32_t reserved0;
+  uint32_t sort_chunk;   /* staged-return PSA: level-2 chunk in queries, 4096 or 8192; 0 = auto
+                           (8192 when the window holds >= 192 queries per leaf)            */
   uint64_t reserved1;
 } harmonia_query_opts;
 
@@ -324,7 +325,7 @@ typedef struct {
   uint32_t staged_return;  /* 1: results return through the chunk-local stage + inverse move */
   uint32_t lane_queries;   /* G = 1: queries interleaved per lane */
   uint32_t warp_shared;    /* 1: G = 1 warp-shared descent (see HARMONIA_QF_PER_LANE) */
-  uint32_t reserved;
+  uint32_t sort_chunk;     /* staged return: level-2 chunk (queries); 0 when not staged */
 } harmonia_plan;
 harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
                                     const harmonia_query_opts* opts, harmonia_plan* out);

@@ -52,14 +52,14 @@ class BuildOpts(C.Structure):
 class QueryOpts(C.Structure):
     _fields_ = [("group_size", C.c_int32), ("psa_bits", C.c_int32), ("smem_levels", C.c_int32),
                 ("flags", C.c_int32), ("window", C.c_uint64), ("lane_queries", C.c_uint32),
-                ("reserved0", C.c_uint32), ("reserved1", C.c_uint64)]
+                ("sort_chunk", C.c_uint32), ("reserved1", C.c_uint64)]
 
 
 class PlanInfo(C.Structure):
     _fields_ = [("group_size", C.c_int32), ("psa_bits", C.c_int32), ("smem_levels", C.c_int32),
                 ("ps_in_smem", C.c_int32), ("window", C.c_uint64), ("smem_bytes", C.c_uint32),
                 ("smem_nodes", C.c_uint32), ("staged_return", C.c_uint32), ("lane_queries", C.c_uint32),
-                ("warp_shared", C.c_uint32), ("reserved", C.c_uint32)]
+                ("warp_shared", C.c_uint32), ("sort_chunk", C.c_uint32)]
 
 
 class Info(C.Structure):
@@ -204,10 +204,12 @@ def _as_u64_dev(t, device):
     return t.contiguous()
 
 
-def make_opts(group_size=0, psa_bits=0, smem_levels=0, window=0, flags=0, lane_queries=0) -> QueryOpts:
+def make_opts(group_size=0, psa_bits=0, smem_levels=0, window=0, flags=0, lane_queries=0,
+              sort_chunk=0) -> QueryOpts:
     o = QueryOpts()
     o.group_size, o.psa_bits, o.smem_levels, o.flags, o.window = group_size, psa_bits, smem_levels, flags, window
     o.lane_queries = lane_queries
+    o.sort_chunk = sort_chunk
     return o
 
 

@@ -57,7 +57,10 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.ilp2 = (o->flags & HARMONIA_QF_ILP1) == 0;
   if (o->lane_queries != 0 && o->lane_queries != 1 && o->lane_queries != 2 && o->lane_queries != 4)
     return HARMONIA_ERR_INVALID_ARG;
-  P.lane_ilp = o->lane_queries ? (int)o->lane_queries : 2;
+#ifndef HM_LANE_ILP
+#define HM_LANE_ILP 2
+#endif
+  P.lane_ilp = o->lane_queries ? (int)o->lane_queries : HM_LANE_ILP;
   P.psa_level2 = (o->flags & HARMONIA_QF_PSA_COARSE) ? 2 : ((o->flags & HARMONIA_QF_PSA_LSD) ? 1 : 0);
   P.fuse = (o->flags & HARMONIA_QF_FUSE_SORT) != 0;  // measured slower
   P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
@@ -81,11 +84,18 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.smem_nodes = (uint32_t)t->level_start[lv];
   P.smem_bytes = used + P.smem_nodes * t->F * 8;
   // staged return (default for the G = 1 PSA path): results leave the search in level-1
-  // order through a kPsaChunk x 8-byte shared-memory stage, k_psa2_unmove restores the
-  // caller's order; two 1024-thread CTAs per SM must still fit
+  // order through a chunk x 8-byte shared-memory stage, k_psa2_unmove restores the caller's
+  // order; two 1024-thread CTAs per SM must still fit.  Chunk: 8192 queries when the window
+  // holds >= 192 queries per leaf (a warp's 64 queries then span ~4 leaves instead of ~8;
+  // measured +5 % at 504 and 252 queries per leaf), else 4096 (at 126, 63 and 32 the 8192
+  // chunk loses 3-30 %: the denser warps gain little and the 8192 sort runs 1 CTA/SM).
+  const uint64_t qpl = t->L ? std::min<uint64_t>(n, P.window) / t->L : 0;
+  P.chunk = o->sort_chunk == kPsaChunkMax || (o->sort_chunk == 0 && qpl >= kChunk8kMinQueriesPerLeaf)
+                ? kPsaChunkMax : kPsaChunk;
   P.ret = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather &&
           !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
-          2 * (round_up(P.smem_bytes, 16) + kPsaChunk * 8 + 1024) <= t->smem_per_sm;
+          2 * (round_up(P.smem_bytes, 16) + P.chunk * 8 + 1024) <= t->smem_per_sm;
+  if (!P.ret || P.fuse) P.chunk = kPsaChunk;
   P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
   P.coop = P.ret && !(o->flags & HARMONIA_QF_PER_LANE);
   // ranges: the warp-per-range copy kernel unless a group size was requested explicitly or
@@ -149,12 +159,13 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       continue;
     }
     if (p.ret) {  // staged return: level-1-order results, then the inverse move
-      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : 0, true, p.wide);
+      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : 0, true, p.wide, p.chunk);
       if (s != HARMONIA_OK) return s;
       a.idx = w.idx;
       a.out = w.sorted_out;
       a.staged = 1;
       a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
+      a.chunk = p.chunk;
       a.bucket = p.bucket;
       if ((s = fused ? launch_sort_search(t, p, a, st) : launch_search(t, p, a, st)) != HARMONIA_OK) return s;
       if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, t->sm_count, st, p.wide)) != HARMONIA_OK) return s;
@@ -233,6 +244,7 @@ extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t 
   out->staged_return = p.ret ? 1u : 0u;
   out->lane_queries = p.G == 1 ? (uint32_t)p.lane_ilp : 0u;
   out->warp_shared = p.coop ? 1u : 0u;
+  out->sort_chunk = p.ret ? p.chunk : 0u;
   return HARMONIA_OK;
 }
 

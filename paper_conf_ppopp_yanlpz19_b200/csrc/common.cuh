@@ -185,6 +185,7 @@ struct Plan {
   bool wide = false;         // staged return with the 11-bit level-1 partition
   bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
   bool range_warp = true;    // ranges: one warp per range, resolve then stream-copy (k_range_warp)
+  uint32_t chunk = 4096;     // staged return: level-2 chunk (4096 or kPsaChunkMax queries)
 };
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
@@ -213,7 +214,12 @@ inline uint64_t l1_rows_bytes(uint64_t window) {
                  c = (window + 8191) / 8192 * 2048 * 4;
   return a > b ? (a > c ? a : c) : (b > c ? b : c);
 }
-constexpr uint32_t kPsaChunk = 4096;  // level-2 chunk (queries)
+constexpr uint32_t kPsaChunk = 4096;     // level-2 chunk (queries): the LSD / non-staged sorts
+constexpr uint32_t kPsaChunkMax = 8192;  // staged-return chunk sizes: 4096 or 8192 (Plan::chunk)
+#ifndef HM_CHUNK8K_QPL
+#define HM_CHUNK8K_QPL 192
+#endif
+constexpr uint64_t kChunk8kMinQueriesPerLeaf = HM_CHUNK8K_QPL;  // auto 8192 chunks from this density
 constexpr uint32_t kScanTile = 4096;
 size_t psa_ws_bytes(const Plan& p);
 PsaWs psa_ws_carve(const Plan& p, void* base);
@@ -242,6 +248,7 @@ struct SearchArgs {
                            // go through shared memory (at dynamic-smem offset res_smem_off)
                            // to out[] in level-1 order, chunk by chunk (kPsaChunk)
   uint32_t res_smem_off;
+  uint32_t chunk;          // staged return: level-2 chunk (queries), 4096 or 8192
   // warp-shared descent (G = 1 PSA path): clamp(q) -> (clamp(q) - kmin) >> cshift is a
   // monotone 32-bit image of the key, so two 32-bit warp reductions bound the warp's queries
   uint32_t coop;
@@ -252,7 +259,7 @@ harmonia_status launch_sort_search(const harmonia_tree* t, const struct Plan& p,
                                    cudaStream_t st);
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
                                int sm_count, cudaStream_t st, int level2 = 0, bool local = false,
-                               bool wide = false);
+                               bool wide = false, uint32_t chunk = kPsaChunk);
 // inverse of the level-1 move for the staged return: out[e] = res1[level-1 position of e]
 harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
                                  cudaStream_t st, bool wide);

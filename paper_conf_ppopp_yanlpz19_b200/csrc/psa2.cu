@@ -29,8 +29,9 @@ constexpr int kCoarseTile = kBlock * kBatches;           // 2048 queries per sca
 #define HM_SORT_THREADS 512
 #endif
 constexpr int kSortThreads = HM_SORT_THREADS, kSortWarps = kSortThreads / 32;
-constexpr int kChunk = kSortThreads * kBatches;          // 4096 queries per local-sort chunk
-static_assert(kCoarseTile == (int)kPsaTile && kChunk == (int)kPsaChunk, "tile sizes shared with search.cu");
+constexpr int kChunk = (int)kPsaChunk;                   // queries per LSD local-sort chunk (4096)
+constexpr int kSortBatches = kChunk / kSortThreads;      // 32-query batches per warp per chunk
+static_assert(kCoarseTile == (int)kPsaTile && kChunk == kSortThreads * kSortBatches, "tile sizes shared with search.cu");
 constexpr int kLocalBits = 11, kLoBits = 6, kHiBits = kLocalBits - kLoBits;
 constexpr size_t kSortSmem = (size_t)kChunk * (8 + 4 + 2);  // keys, positions, local digits
 
@@ -446,17 +447,17 @@ constexpr size_t unmove_smem() {
 
 // ---- level 2: chunk-local sort by the N-bit bucket (two stable LSD passes) ---------------
 template <int BITS, int SHIFT>
-__device__ __forceinline__ void lsd_pass(uint64_t (&v)[kBatches], uint32_t (&ix)[kBatches], uint32_t (&lk)[kBatches],
+__device__ __forceinline__ void lsd_pass(uint64_t (&v)[kSortBatches], uint32_t (&ix)[kSortBatches], uint32_t (&lk)[kSortBatches],
                                          uint32_t m, uint32_t (*wcnt)[1 << kLoBits], uint32_t* bin_start, uint32_t* tmp,
                                          uint64_t* s_q, uint32_t* s_i, uint16_t* s_k) {
   constexpr int NB = 1 << BITS;
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (int i = threadIdx.x; i < kSortWarps * NB; i += kSortThreads) wcnt[i / NB][i % NB] = 0;
   __syncthreads();
-  uint32_t pos[kBatches], dg[kBatches];
+  uint32_t pos[kSortBatches], dg[kSortBatches];
 #pragma unroll
-  for (int k = 0; k < kBatches; ++k) {  // element order = (warp, batch, lane): stable ranks
-    const uint32_t e = warp * (32 * kBatches) + k * 32 + lane;
+  for (int k = 0; k < kSortBatches; ++k) {  // element order = (warp, batch, lane): stable ranks
+    const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
     const bool valid = e < m;
     dg[k] = (lk[k] >> SHIFT) & (NB - 1);
     const unsigned peers = peers_of<BITS>(dg[k], __ballot_sync(kFull, valid));
@@ -480,8 +481,8 @@ __device__ __forceinline__ void lsd_pass(uint64_t (&v)[kBatches], uint32_t (&ix)
   if (threadIdx.x < NB) bin_start[threadIdx.x] = bs;
   __syncthreads();
 #pragma unroll
-  for (int k = 0; k < kBatches; ++k) {
-    const uint32_t e = warp * (32 * kBatches) + k * 32 + lane;
+  for (int k = 0; k < kSortBatches; ++k) {
+    const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
     if (e < m) {
       const uint32_t dst = bin_start[dg[k]] + wcnt[warp][dg[k]] + pos[k];
       s_q[dst] = v[k];
@@ -491,8 +492,8 @@ __device__ __forceinline__ void lsd_pass(uint64_t (&v)[kBatches], uint32_t (&ix)
   }
   __syncthreads();
 #pragma unroll
-  for (int k = 0; k < kBatches; ++k) {  // reload in the new order for the next pass
-    const uint32_t e = warp * (32 * kBatches) + k * 32 + lane;
+  for (int k = 0; k < kSortBatches; ++k) {  // reload in the new order for the next pass
+    const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
     if (e < m) {
       v[k] = s_q[e];
       ix[k] = s_i[e];
@@ -513,12 +514,12 @@ __global__ void __launch_bounds__(kSortThreads, 2) k_psa2_local_sort(uint64_t* _
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (uint64_t c0 = (uint64_t)blockIdx.x * kChunk; c0 < n; c0 += (uint64_t)gridDim.x * kChunk) {
     const uint32_t m = (uint32_t)std::min<uint64_t>(kChunk, n - c0);
-    uint64_t v[kBatches];
-    uint32_t ix[kBatches], lk[kBatches];
+    uint64_t v[kSortBatches];
+    uint32_t ix[kSortBatches], lk[kSortBatches];
     uint32_t bmin = 0xFFFFFFFFu, bmax = 0;
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {
-      const uint32_t e = warp * (32 * kBatches) + k * 32 + lane;
+    for (int k = 0; k < kSortBatches; ++k) {
+      const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
       if (e < m) {
         v[k] = sorted_q[c0 + e];
         ix[k] = idx[c0 + e];
@@ -546,12 +547,12 @@ __global__ void __launch_bounds__(kSortThreads, 2) k_psa2_local_sort(uint64_t* _
     uint32_t sh = 0;
     while (((bmax - bmin) >> sh) >= (1u << kLocalBits)) ++sh;
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) lk[k] = (lk[k] - bmin) >> sh;
+    for (int k = 0; k < kSortBatches; ++k) lk[k] = (lk[k] - bmin) >> sh;
     lsd_pass<kLoBits, 0>(v, ix, lk, m, wcnt, bin_start, tmp, s_q, s_i, s_k);
     lsd_pass<kHiBits, kLoBits>(v, ix, lk, m, wcnt, bin_start, tmp, s_q, s_i, s_k);
 #pragma unroll
-    for (int k = 0; k < kBatches; ++k) {  // write back (coalesced)
-      const uint32_t e = warp * (32 * kBatches) + k * 32 + lane;
+    for (int k = 0; k < kSortBatches; ++k) {  // write back (coalesced)
+      const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
       if (e < m) {
         sorted_q[c0 + e] = v[k];
         idx[c0 + e] = ix[k];
@@ -565,7 +566,10 @@ constexpr int kLocalBins = 1 << kLocalBits;
 #define HM_SORT_PREFETCH 1
 #endif
 // local histogram, sorted keys + positions, and (prefetch) the next chunk's staged queries
-constexpr size_t kCountSortSmem = (size_t)kLocalBins * 4 + (size_t)kChunk * 12 + (HM_SORT_PREFETCH ? kChunk * 8 : 0);
+template <int kCh>
+constexpr size_t count_sort_smem() {
+  return (size_t)kLocalBins * 4 + (size_t)kCh * 12 + (HM_SORT_PREFETCH ? (size_t)kCh * 8 : 0);
+}
 #include "psa2_count_sort.inc"
 
 // level-1 grid: persistent CTAs, ~2048 resident threads per SM, at most one CTA per tile
@@ -728,7 +732,7 @@ harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSpli
 }
 
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
-                               cudaStream_t st, int level2, bool local, bool wide) {
+                               cudaStream_t st, int level2, bool local, bool wide, uint32_t chunk) {
   harmonia_status s;
   if (wide) {  // staged-return mode only (no idx)
     const uint32_t b1 = (uint32_t)std::min(nb, Wide::BITS);
@@ -746,22 +750,28 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
     static bool configured = false;
     if (!configured) {
       HM_CUDA(cudaFuncSetAttribute(k_psa2_local_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSortSmem));
-      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)kCountSortSmem));
-      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)kCountSortSmem));
+      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<false, kChunk>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)count_sort_smem<kChunk>()));
+      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<true, kChunk>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)count_sort_smem<kChunk>()));
+      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<true, (int)kPsaChunkMax>,
+                                   cudaFuncAttributeMaxDynamicSharedMemorySize, (int)count_sort_smem<kPsaChunkMax>()));
       configured = true;
     }
 #ifndef HM_SORT_CTAS_PER_SM
 #define HM_SORT_CTAS_PER_SM 4
 #endif
-    const int g = (int)std::min<uint64_t>(ceil_div(n, kChunk), (uint64_t)sm * HM_SORT_CTAS_PER_SM);
+    const uint32_t ch = (local && level2 == 0 && chunk == kPsaChunkMax) ? kPsaChunkMax : (uint32_t)kChunk;
+    const int g = (int)std::min<uint64_t>(ceil_div(n, ch), (uint64_t)sm * HM_SORT_CTAS_PER_SM);
     if (level2 == 1)  // two stable LSD passes of ballot multisplit (ablation)
       k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
+    else if (local && ch == kPsaChunkMax)  // 8192-query chunks (denser key ranges per warp)
+      k_psa2_count_sort<true, (int)kPsaChunkMax>
+          <<<std::max(g, 1), kSortThreads, count_sort_smem<kPsaChunkMax>(), st>>>(ws.sorted_q, ws.idx, n, f);
     else if (local)   // one counting pass with shared-memory atomics (default, measured faster)
-      k_psa2_count_sort<true><<<std::max(g, 1), kSortThreads, kCountSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
+      k_psa2_count_sort<true, kChunk><<<std::max(g, 1), kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted_q, ws.idx, n, f);
     else
-      k_psa2_count_sort<false><<<std::max(g, 1), kSortThreads, kCountSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
+      k_psa2_count_sort<false, kChunk><<<std::max(g, 1), kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted_q, ws.idx, n, f);
   }
   HM_LAUNCHED();
   return HARMONIA_OK;

@@ -438,6 +438,54 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
   }
 }
 
+// 256-bit read-only load of 4 consecutive keys (sm_100a LDG.E.ENL2.256; 32-byte aligned)
+__device__ __forceinline__ void ld_quad_global(const uint64_t* p, uint64_t (&k)[4]) {
+  asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
+               : "=l"(k[0]), "=l"(k[1]), "=l"(k[2]), "=l"(k[3])
+               : "l"(p));
+}
+
+#ifndef HM_LEAF_TAIL
+#define HM_LEAF_TAIL 4  // measured: 4 > 8 > 16 > off at c2 and c3
+#endif
+// Per-lane rank in a global node with a vector tail: binary-lifting steps down to TL keys,
+// then the TL-key block [r, r+TL) is read with TL/4 independent 256-bit loads and counted
+// (keys below r are <= q, keys from r+TL on are > q, so r + #(block <= q) is the rank).
+// log2(F/TL) + 1 dependent round trips instead of log2(F).  best = the last key <= q.
+template <int F, int U, int TL>
+__device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint32_t (&node)[U],
+                                               const uint64_t (&q)[U], uint32_t (&r)[U], uint64_t (&best)[U]) {
+#pragma unroll
+  for (int s = F / 2; s >= TL; s >>= 1) {
+    uint64_t k[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) k[u] = ld_key_global(keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool le = k[u] <= q[u];
+      r[u] += le ? s : 0;
+      best[u] = le ? k[u] : best[u];
+    }
+  }
+  uint64_t k[U][TL];
+#pragma unroll
+  for (int u = 0; u < U; ++u)
+#pragma unroll
+    for (int j = 0; j < TL / 4; ++j)
+      ld_quad_global(keys + (uint64_t)node[u] * F + r[u] + 4 * j, *reinterpret_cast<uint64_t(*)[4]>(&k[u][4 * j]));
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    uint32_t c = 0;
+#pragma unroll
+    for (int j = 0; j < TL; ++j) {
+      const bool le = k[u][j] <= q[u];
+      c += le ? 1u : 0u;
+      best[u] = le ? k[u][j] : best[u];
+    }
+    r[u] += c;
+  }
+}
+
 // G = 1 with U independent queries per lane, interleaved step by step: the single-lane
 // search is latency-bound (few instructions, few wavefronts), so U chains per thread raise
 // the memory-level parallelism without adding work.  A warp takes 32*U consecutive
@@ -464,13 +512,21 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
         for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
       }
     } else {
+#if HM_LEAF_TAIL > 0 && HM_TAIL_INTERNAL
+      if constexpr (F >= 2 * HM_LEAF_TAIL) {
+        uint64_t bst[U];
+        lane_rank_tail<F, U, HM_LEAF_TAIL>(a.keys, node, q, r, bst);
+      } else
+#endif
+      {
 #pragma unroll
-      for (int s = F / 2; s >= 1; s >>= 1) {
-        uint64_t k[U];
+        for (int s = F / 2; s >= 1; s >>= 1) {
+          uint64_t k[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+          for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
 #pragma unroll
-        for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+          for (int u = 0; u < U; ++u) r[u] += k[u] <= q[u] ? s : 0;
+        }
       }
     }
 #pragma unroll
@@ -485,18 +541,25 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
     r[u] = 0;
     best[u] = 0;
   }
+#if HM_LEAF_TAIL > 0
+  if (F >= 2 * HM_LEAF_TAIL && !leaf_smem) {
+    lane_rank_tail<F, U, (F >= 2 * HM_LEAF_TAIL ? HM_LEAF_TAIL : 4)>(a.keys, node, q, r, best);
+  } else
+#endif
+  {
 #pragma unroll
-  for (int s = F / 2; s >= 1; s >>= 1) {
-    uint64_t k[U];
+    for (int s = F / 2; s >= 1; s >>= 1) {
+      uint64_t k[U];
 #pragma unroll
-    for (int u = 0; u < U; ++u)
-      k[u] = leaf_smem ? s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)]
-                       : ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+      for (int u = 0; u < U; ++u)
+        k[u] = leaf_smem ? s_keys[(uint64_t)node[u] * F + (r[u] + s - 1)]
+                         : ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const bool le = k[u] <= q[u];
-      r[u] += le ? s : 0;
-      best[u] = le ? k[u] : best[u];
+      for (int u = 0; u < U; ++u) {
+        const bool le = k[u] <= q[u];
+        r[u] += le ? s : 0;
+        best[u] = le ? k[u] : best[u];
+      }
     }
   }
 #pragma unroll
@@ -695,8 +758,8 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
   const bool ps_smem = a.ps_smem_bytes != 0;
   const bool leaf_smem = a.h - 1 < a.smem_levels;
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t c0 = (uint64_t)blockIdx.x * kPsaChunk; c0 < a.n; c0 += (uint64_t)gridDim.x * kPsaChunk) {
-    const uint32_t m = (uint32_t)(a.n - c0 < kPsaChunk ? a.n - c0 : kPsaChunk);
+  for (uint64_t c0 = (uint64_t)blockIdx.x * a.chunk; c0 < a.n; c0 += (uint64_t)gridDim.x * a.chunk) {
+    const uint32_t m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
@@ -1136,7 +1199,7 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   const int U = p.lane_ilp;
   auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
                      : (U >= 4 ? k_lane_search_c<F, 4, false> : (U == 2 ? k_lane_search_c<F, 2, false> : k_lane_search_c<F, 1, false>));
-  const uint32_t smem = a.res_smem_off + kPsaChunk * 8;
+  const uint32_t smem = a.res_smem_off + a.chunk * 8;
   static int configured_smem[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
   const int ci = (U >= 4 ? 4 : U) + (a.coop ? 5 : 0);
   if ((int)smem > configured_smem[ci]) {
@@ -1146,7 +1209,7 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, smem));
   per_sm = std::max(per_sm, 1);
-  const uint64_t need = ceil_div(a.n, kPsaChunk);
+  const uint64_t need = ceil_div(a.n, (uint64_t)a.chunk);
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);

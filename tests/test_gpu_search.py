@@ -135,7 +135,9 @@ def test_lane_search_queries_per_lane(hm, orc, F, lane_queries):
                {"flags": hm.QF_FUSE_SORT, "window": 5120, "smem_levels": 1}, {"flags": hm.QF_SCATTER_RETURN},
                {"flags": hm.QF_SCATTER_RETURN, "window": 7168}, {"window": 7168, "smem_levels": -1},
                {"flags": hm.QF_PSA_WIDE}, {"flags": hm.QF_PSA_WIDE, "window": 13312},
-               {"flags": hm.QF_PER_LANE}, {"flags": hm.QF_PER_LANE, "window": 7168, "smem_levels": -1}):
+               {"flags": hm.QF_PER_LANE}, {"flags": hm.QF_PER_LANE, "window": 7168, "smem_levels": -1},
+               {"sort_chunk": 8192}, {"sort_chunk": 8192, "window": 13312}, {"sort_chunk": 4096},
+               {"sort_chunk": 8192, "smem_levels": -1}, {"sort_chunk": 8192, "flags": hm.QF_PER_LANE}):
         got = host(t.search(cu(q), group_size=1, lane_queries=lane_queries, **kw))
         assert np.array_equal(got, exp), kw
 
@@ -165,9 +167,25 @@ def test_warp_shared_descent(hm, orc, F, keyset):
     q = np.concatenate(parts)
     exp = orc.sorted_search(keys, vals, q)
     for kw in ({}, {"window": 5120}, {"smem_levels": -1}, {"smem_levels": 1}, {"lane_queries": 1},
-               {"lane_queries": 4}, {"flags": hm.QF_PER_LANE}):
+               {"lane_queries": 4}, {"flags": hm.QF_PER_LANE}, {"sort_chunk": 8192},
+               {"sort_chunk": 8192, "window": 9216}, {"sort_chunk": 4096}):
         assert np.array_equal(host(t.search(cu(q), group_size=1, **kw)), exp), kw
     assert t.plan(len(q))["warp_shared"] == 1 and t.plan(len(q), flags=hm.QF_PER_LANE)["warp_shared"] == 0
+
+
+def test_sort_chunk_plan(hm):
+    """Auto level-2 chunk: 8192 queries when the window holds >= 192 queries per leaf, else
+    4096; an explicit sort_chunk wins; non-staged plans report 0."""
+    keys = gen.uniform_keys(1 << 16)
+    t = tree(hm, keys, gen.values_for(keys), 64)
+    inf = t.info()
+    leaves = inf["n_nodes"] - inf["level_start"][inf["height"] - 1]
+    dense, sparse = 192 * leaves, 191 * leaves
+    assert t.plan(dense)["sort_chunk"] == 8192
+    assert t.plan(sparse)["sort_chunk"] == 4096
+    assert t.plan(dense, sort_chunk=4096)["sort_chunk"] == 4096
+    assert t.plan(sparse, sort_chunk=8192)["sort_chunk"] == 8192
+    assert t.plan(dense, psa_bits=-1)["sort_chunk"] == 0
 
 
 @pytest.mark.parametrize("F,G", FG)

@@ -1,6 +1,6 @@
 # A/B the default library against gpurun_variants/*.so on c2 (device-resident bench, no e2e/cpu)
 mkdir -p gpurun_out
-for v in default $(ls gpurun_variants | sed 's/\.so$//'); do
+for v in default $(cd gpurun_variants && ls *.so | sed "s/\.so$//"); do
   if [ $v = default ]; then unset HARMONIA_LIB; else export HARMONIA_LIB=gpurun_variants/$v.so; fi
   python bench.py --no-e2e --no-cpu --steps 20 "$@" > gpurun_out/ab_$v.json 2>/dev/null
   python -c "
