@@ -562,15 +562,14 @@ __global__ void __launch_bounds__(kSortThreads, 2) k_psa2_local_sort(uint64_t* _
 }
 
 constexpr int kLocalBins = 1 << kLocalBits;
-#ifndef HM_SORT_PREFETCH
-#define HM_SORT_PREFETCH 1
-#endif
 // local histogram, sorted keys + positions, and (prefetch) the next chunk's staged queries
 template <int kCh>
-constexpr size_t count_sort_smem() {
-  return (size_t)kLocalBins * 4 + (size_t)kCh * 12 + (HM_SORT_PREFETCH ? (size_t)kCh * 8 : 0);
-}
+constexpr size_t count_sort_smem();
 #include "psa2_count_sort.inc"
+template <int kCh>
+constexpr size_t count_sort_smem() {
+  return (size_t)kLocalBins * 4 + (size_t)kCh * 12 + (sort_prefetch<kCh>() ? (size_t)kCh * 8 : 0);
+}
 
 // level-1 grid: persistent CTAs, ~2048 resident threads per SM, at most one CTA per tile
 template <class C>
