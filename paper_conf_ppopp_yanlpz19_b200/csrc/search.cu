@@ -438,6 +438,15 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
   }
 }
 
+#ifndef HM_SEARCH_PF_L2
+#define HM_SEARCH_PF_L2 0
+#endif
+// bulk L2 prefetch (TMA unit; bytes a multiple of 16, address 16-byte aligned)
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  if (bytes == 0 || ((uintptr_t)p & 15)) return;
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
 // 256-bit read-only load of 4 consecutive keys (sm_100a LDG.E.ENL2.256; 32-byte aligned)
 __device__ __forceinline__ void ld_quad_global(const uint64_t* p, uint64_t (&k)[4]) {
   asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
@@ -597,12 +606,18 @@ __device__ __forceinline__ void lane_core(const SearchArgs& a, const uint64_t* s
 // the lane searches only that window, then goes on alone.  At the leaf the window is
 // [#keys < qlo, #keys <= qhi]: a key equal to q can only lie inside it.
 
-// ranks of qlo and qhi in node nk: #keys (< or <=) qlo and #keys <= qhi, warp-cooperatively
+// ranks of qlo and qhi in node nk: #keys (< or <=) qlo and #keys <= qhi, warp-cooperatively.
+// The node's keys stay in kk (lane l holds slots p*64 + 2l, +1 of load p) for the window rank.
+template <int F>
+struct NodeRegs {
+  static constexpr int NP = F >= 64 ? F / 64 : 1;  // 128-bit loads per lane
+  ulonglong2 k[NP];
+};
 template <int F, bool SMEM, bool STRICT_LO>
 __device__ __forceinline__ void coop_rank(const uint64_t* nk, uint64_t qlo, uint64_t qhi, uint32_t& rlo,
-                                          uint32_t& rhi) {
+                                          uint32_t& rhi, NodeRegs<F>& kk) {
   const unsigned lane = threadIdx.x & 31;
-  constexpr int NP = F >= 64 ? F / 64 : 1;  // 128-bit loads per lane
+  constexpr int NP = NodeRegs<F>::NP;
   rlo = 0;
   rhi = 0;
 #pragma unroll
@@ -610,9 +625,50 @@ __device__ __forceinline__ void coop_rank(const uint64_t* nk, uint64_t qlo, uint
     const uint32_t slot = p * 64 + 2 * lane;
     ulonglong2 k = make_ulonglong2(kPad, kPad);  // PAD > every bound
     if (F >= 64 || slot < F) k = ld_pair<SMEM>(nk + slot);
+    kk.k[p] = k;
     const bool lx = STRICT_LO ? k.x < qlo : k.x <= qlo, ly = STRICT_LO ? k.y < qlo : k.y <= qlo;
     rlo += __popc(ballot(lx)) + __popc(ballot(ly));
     rhi += __popc(ballot(k.x <= qhi)) + __popc(ballot(k.y <= qhi));
+  }
+}
+template <int F, bool SMEM, bool STRICT_LO>
+__device__ __forceinline__ void coop_rank(const uint64_t* nk, uint64_t qlo, uint64_t qhi, uint32_t& rlo,
+                                          uint32_t& rhi) {
+  NodeRegs<F> kk;
+  coop_rank<F, SMEM, STRICT_LO>(nk, qlo, qhi, rlo, rhi, kk);
+}
+
+#ifndef HM_SHFL_WINDOW
+#define HM_SHFL_WINDOW 16
+#endif
+#ifndef HM_SHFL_SMEM
+#define HM_SHFL_SMEM 1  // also at staged (shared-memory) levels (measured: equal or 0.5 % better)
+#endif
+// per-lane rank inside a narrow warp-uniform window [rlo, rhi] from the node keys the
+// cooperative load left in registers: the rhi - rlo undecided keys are broadcast one by one
+// (warp-uniform trip count, two 32-bit shuffles each) and counted -- no dependent memory
+// round trip after the cooperative load.  Same result as window_rank.  F <= 64 (larger
+// nodes would hold 4+ registers per lane past the 32-register budget of the search CTAs).
+template <int F, int U>
+__device__ __forceinline__ void window_rank_regs(const NodeRegs<F>& kk, const uint64_t (&q)[U], uint32_t rlo,
+                                                 uint32_t rhi, uint32_t (&r)[U], uint64_t (&best)[U]) {
+  constexpr int NP = NodeRegs<F>::NP;
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    r[u] = rlo;
+    best[u] = 0;
+  }
+  for (uint32_t j = rlo; j < rhi; ++j) {
+    ulonglong2 pr = kk.k[0];
+#pragma unroll
+    for (int p = 1; p < NP; ++p) pr = (int)(j >> 6) == p ? kk.k[p] : pr;
+    const uint64_t key = __shfl_sync(kFull, (j & 1) ? pr.y : pr.x, (int)((j & 63) >> 1));
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool le = key <= q[u];
+      r[u] += le ? 1u : 0u;
+      best[u] = le ? key : best[u];
+    }
   }
 }
 
@@ -676,8 +732,9 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
   for (; l + 1 < a.h; ++l) {
     const uint32_t first = ps_smem ? s_ps[node] : __ldg(a.ps + node);  // PS[node_idx]
     uint32_t rlo, rhi;
-    if (l < a.smem_levels) coop_rank<F, true, false>(s_keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
-    else coop_rank<F, false, false>(a.keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
+    NodeRegs<F> kk;
+    if (l < a.smem_levels) coop_rank<F, true, false>(s_keys + (uint64_t)node * F, qlo, qhi, rlo, rhi, kk);
+    else coop_rank<F, false, false>(a.keys + (uint64_t)node * F, qlo, qhi, rlo, rhi, kk);
     if (rlo == rhi) {
       node = first + rlo;  // Eq 1, the same child for the whole warp
       continue;
@@ -687,7 +744,9 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
     uint64_t off[U], best[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) off[u] = (uint64_t)node * F;
-    if (l < a.smem_levels) window_rank<F, U, true>(s_keys, off, q, rlo, rhi, r, best);
+    if (F <= 64 && rhi - rlo <= HM_SHFL_WINDOW && (HM_SHFL_SMEM || l >= a.smem_levels))
+      window_rank_regs<F, U>(kk, q, rlo, rhi, r, best);
+    else if (l < a.smem_levels) window_rank<F, U, true>(s_keys, off, q, rlo, rhi, r, best);
     else window_rank<F, U, false>(a.keys, off, q, rlo, rhi, r, best);
 #pragma unroll
     for (int u = 0; u < U; ++u) nd[u] = first + r[u];
@@ -696,13 +755,15 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
   }
   // the whole warp reached the same leaf
   uint32_t rlo, rhi;
-  if (leaf_smem) coop_rank<F, true, true>(s_keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
-  else coop_rank<F, false, true>(a.keys + (uint64_t)node * F, qlo, qhi, rlo, rhi);
+  NodeRegs<F> kk;
+  if (leaf_smem) coop_rank<F, true, true>(s_keys + (uint64_t)node * F, qlo, qhi, rlo, rhi, kk);
+  else coop_rank<F, false, true>(a.keys + (uint64_t)node * F, qlo, qhi, rlo, rhi, kk);
   uint32_t r[U];
   uint64_t off[U], best[U];
 #pragma unroll
   for (int u = 0; u < U; ++u) off[u] = (uint64_t)node * F;
-  if (leaf_smem) window_rank<F, U, true>(s_keys, off, q, rlo, rhi, r, best);
+  if (F <= 64 && rhi - rlo <= HM_SHFL_WINDOW && (HM_SHFL_SMEM || !leaf_smem)) window_rank_regs<F, U>(kk, q, rlo, rhi, r, best);
+  else if (leaf_smem) window_rank<F, U, true>(s_keys, off, q, rlo, rhi, r, best);
   else window_rank<F, U, false>(a.keys, off, q, rlo, rhi, r, best);
   const uint64_t* vrow = a.vals + (uint64_t)(node - a.leaf_start) * F;
 #pragma unroll
@@ -760,6 +821,16 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (uint64_t c0 = (uint64_t)blockIdx.x * a.chunk; c0 < a.n; c0 += (uint64_t)gridDim.x * a.chunk) {
     const uint32_t m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
+#if HM_SEARCH_PF_L2
+    if (threadIdx.x == 0) {  // the next chunk's queries and offsets: HBM -> L2 while this one runs
+      const uint64_t c1 = c0 + (uint64_t)gridDim.x * a.chunk;
+      if (c1 < a.n) {
+        const uint32_t m1 = (uint32_t)(a.n - c1 < a.chunk ? a.n - c1 : a.chunk);
+        prefetch_l2(a.q + c1, (m1 * 8) & ~15u);
+        prefetch_l2(a.idx + c1, (m1 * 4) & ~15u);
+      }
+    }
+#endif
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
