@@ -214,6 +214,9 @@ inline uint64_t l1_rows_bytes(uint64_t window) {
                  c = (window + 8191) / 8192 * 2048 * 4;
   return a > b ? (a > c ? a : c) : (b > c ? b : c);
 }
+#ifndef HM_IDX16
+#define HM_IDX16 1  // staged return: chunk-local level-1 offsets stored as uint16 (< 2^16)
+#endif
 constexpr uint32_t kPsaChunk = 4096;     // level-2 chunk (queries): the LSD / non-staged sorts
 constexpr uint32_t kPsaChunkMax = 8192;  // staged-return chunk sizes: 4096 or 8192 (Plan::chunk)
 #ifndef HM_CHUNK8K_QPL

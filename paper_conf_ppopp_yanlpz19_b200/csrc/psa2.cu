@@ -21,6 +21,13 @@
 
 namespace hm {
 
+#ifndef HM_L1_WAVES
+#define HM_L1_WAVES 8
+#endif
+#ifndef HM_L1_WAVES_MV
+#define HM_L1_WAVES_MV 16
+#endif
+
 namespace {
 
 constexpr int kBatches = 8;                              // 32-query batches per warp per tile
@@ -31,7 +38,7 @@ constexpr int kCoarseTile = kBlock * kBatches;           // 2048 queries per sca
 constexpr int kSortThreads = HM_SORT_THREADS, kSortWarps = kSortThreads / 32;
 constexpr int kChunk = (int)kPsaChunk;                   // queries per LSD local-sort chunk (4096)
 constexpr int kSortBatches = kChunk / kSortThreads;      // 32-query batches per warp per chunk
-static_assert(kCoarseTile == (int)kPsaTile && kChunk == kSortThreads * kSortBatches, "tile sizes shared with search.cu");
+static_assert(kChunk == kSortThreads * kSortBatches, "chunk = threads x batches");
 constexpr int kLocalBits = 11, kLoBits = 6, kHiBits = kLocalBits - kLoBits;
 constexpr size_t kSortSmem = (size_t)kChunk * (8 + 4 + 2);  // keys, positions, local digits
 
@@ -109,7 +116,13 @@ struct L1Cfg {
   static_assert(BINS % NT_ == 0 && TILE_ % NT_ == 0 && (1 << TILE_SHIFT) == TILE_, "L1Cfg");
   static_assert(BITS_ + TILE_SHIFT <= 32 && BITS_ + TILE_SHIFT + 0 <= 32, "packed digit|rank");
 };
-using Narrow = L1Cfg<8, 2048, 256>;
+#ifndef HM_NARROW_TILE
+#define HM_NARROW_TILE 2048
+#endif
+#ifndef HM_NARROW_NT
+#define HM_NARROW_NT 256
+#endif
+using Narrow = L1Cfg<8, HM_NARROW_TILE, HM_NARROW_NT>;
 #ifndef HM_WIDE_TILE
 #define HM_WIDE_TILE 4096
 #endif
@@ -244,6 +257,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
                                                               uint32_t* __restrict__ idx,
                                                               const uint64_t* __restrict__ push_dst = nullptr) {
   constexpr bool kRecompute = std::is_same<Digit, CoarseDigit>::value;
+  constexpr bool kCtaSums = HM_L1_WAVES_MV != HM_L1_WAVES;
   __shared__ uint64_t s_push[kPush ? C::BINS : 1];  // push_dst[d] - 8 * (first global slot of bin d)
   extern __shared__ __align__(16) unsigned char l1_smem[];
   uint64_t* st_q = reinterpret_cast<uint64_t*>(l1_smem);
@@ -279,7 +293,14 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __
     for (int k = 0; k < C::BPT; ++k) {
       const uint64_t b = threadIdx.x * C::BPT + k;
       if constexpr (kPush) s_push[b] = push_dst[b] - 8ull * run[k];  // run[k] = bin start here
-      const uint32_t cc = cta_counts[(uint64_t)blockIdx.x * C::BINS + b];
+      // this CTA's total in bin b, from the per-tile counts of its own tile range: the move
+      // grid need not equal the rank grid (cta_counts is only read when it does)
+      uint32_t cc = 0;
+      if (kCtaSums) {
+        for (uint64_t tt = tb; tt < te; ++tt) cc += tile_counts[tt * C::BINS + b];
+      } else {
+        cc = cta_counts[(uint64_t)blockIdx.x * C::BINS + b];
+      }
       run[k] = cc ? run[k] + atomicAdd(cursor + b, cc) : 0u;
       cta_base[(uint64_t)blockIdx.x * C::BINS + b] = run[k];  // for the staged return
     }
@@ -571,14 +592,18 @@ constexpr size_t count_sort_smem() {
   return (size_t)kLocalBins * 4 + (size_t)kCh * 12 + (sort_prefetch<kCh>() ? (size_t)kCh * 8 : 0);
 }
 
-// level-1 grid: persistent CTAs, ~2048 resident threads per SM, at most one CTA per tile
+// level-1 grids: CTAs own contiguous tile ranges, ~2048 resident threads per SM, waves x the
+// resident CTAs.  The rank pass and the move/unmove pair may use different wave counts (the
+// move then sums its CTA's per-tile counts itself): measured best 8 for the rank pass, 16 for
+// the move and its inverse.
 template <class C>
-int l1_grid(uint64_t n, int sm) {
-#ifndef HM_L1_WAVES
-#define HM_L1_WAVES 8
-#endif
-  const uint64_t g = std::min<uint64_t>((uint64_t)sm * (2048 / C::NT) * HM_L1_WAVES, kL1CtaRows / C::BINS);
+int l1_grid(uint64_t n, int sm, int waves = HM_L1_WAVES) {
+  const uint64_t g = std::min<uint64_t>((uint64_t)sm * (2048 / C::NT) * waves, kL1CtaRows / C::BINS);
   return (int)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(n, C::TILE), g));
+}
+template <class C>
+int l1_grid_mv(uint64_t n, int sm) {
+  return l1_grid<C>(n, sm, HM_L1_WAVES_MV);
 }
 
 // level-1 partition by a C::BITS-bit digit: rank pass, then the staged move.
@@ -589,7 +614,7 @@ harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg,
                                  uint32_t nbins) {
   constexpr bool kRecompute = std::is_same<Digit, CoarseDigit>::value;
   HM_CUDA(cudaMemsetAsync(ws.counts, 0, 2 * C::BINS * 4, st));
-  const int g = l1_grid<C>(n, sm);
+  const int g = l1_grid<C>(n, sm), gm = l1_grid_mv<C>(n, sm);
   {
     ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
     k_psa2_rank<Digit, C><<<g, C::NT, 0, st>>>(q, n, dg, ws.counts, ws.tile_counts, ws.packed, ws.cta_counts);
@@ -610,7 +635,7 @@ harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg,
         HM_CUDA(cudaFuncSetAttribute(k_psa2_move<Digit, C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
         cfg = true;
       }
-      k_psa2_move<Digit, C, true><<<g, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
+      k_psa2_move<Digit, C, true><<<gm, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
                                                          ws.packed, ws.cta_counts, ws.cta_base, sorted_q, idx);
     } else {
       constexpr size_t smb = move_smem<C, false, kRecompute>();
@@ -619,7 +644,7 @@ harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg,
         HM_CUDA(cudaFuncSetAttribute(k_psa2_move<Digit, C, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
         cfg = true;
       }
-      k_psa2_move<Digit, C, false><<<g, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
+      k_psa2_move<Digit, C, false><<<gm, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
                                                           ws.packed, ws.cta_counts, ws.cta_base, sorted_q, nullptr);
     }
   }
@@ -637,7 +662,7 @@ harmonia_status unpartition(const PsaWs& ws, const uint64_t* res1, uint64_t n, u
     cfg = true;
   }
   ProfScope ps_(HARMONIA_PROF_RETURN, st);
-  k_psa2_unmove<C><<<l1_grid<C>(n, sm), C::NT, smb, st>>>(ws.tile_counts, ws.cta_base, ws.packed, res1, n, out);
+  k_psa2_unmove<C><<<l1_grid_mv<C>(n, sm), C::NT, smb, st>>>(ws.tile_counts, ws.cta_base, ws.packed, res1, n, out);
   HM_LAUNCHED();
   return HARMONIA_OK;
 }
@@ -696,7 +721,7 @@ harmonia_status route_push2(const uint64_t* q, uint64_t n, const BucketSplit& f,
   }
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
-    k_psa2_move<BucketSplit, C, false, true><<<l1_grid<C>(n, sm), C::NT, smb, st>>>(
+    k_psa2_move<BucketSplit, C, false, true><<<l1_grid_mv<C>(n, sm), C::NT, smb, st>>>(
         q, n, f, ws.counts, ws.counts + C::BINS, ws.tile_counts, ws.packed, ws.cta_counts, ws.cta_base, nullptr,
         nullptr, d_push);
   }

@@ -80,6 +80,11 @@ __device__ __forceinline__ uint64_t ld_stream(const uint64_t* p) {
   asm volatile("ld.global.cs.u64 %0, [%1];" : "=l"(v) : "l"(p));
   return v;
 }
+__device__ __forceinline__ uint16_t ld_stream16(const uint16_t* p) {
+  uint16_t v;
+  asm volatile("ld.global.cs.u16 %0, [%1];" : "=h"(v) : "l"(p));
+  return v;
+}
 __device__ __forceinline__ uint32_t ld_stream32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.global.cs.u32 %0, [%1];" : "=r"(v) : "l"(p));
@@ -438,6 +443,9 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
   }
 }
 
+#ifndef HM_LEAF_VSPEC
+#define HM_LEAF_VSPEC 0
+#endif
 #ifndef HM_SEARCH_PF_L2
 #define HM_SEARCH_PF_L2 0
 #endif
@@ -541,6 +549,36 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
 #pragma unroll
     for (int u = 0; u < U; ++u) node[u] = first[u] + r[u];  // Eq 1
   }
+#if HM_LEAF_VSPEC
+  // leaf, speculative value block: binary lifting on #keys < q down to a 4-slot block; then
+  // (invariant r <= #keys < q < r + 4) a key equal to q can only sit in [r, r+4), so the
+  // block's 4 keys and its 4 values (each one 32-byte sector) are read together -- the
+  // value no longer waits for the rank.  Keys are unique: at most one slot matches.
+  if (F >= 8 && !leaf_smem) {
+    uint32_t r[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) r[u] = 0;
+#pragma unroll
+    for (int s = F / 2; s >= 4; s >>= 1) {
+      uint64_t k[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
+#pragma unroll
+      for (int u = 0; u < U; ++u) r[u] += k[u] < q[u] ? s : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      uint64_t kb[4], vb[4];
+      ld_quad_global(a.keys + (uint64_t)node[u] * F + r[u], kb);
+      ld_quad_global(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + r[u], vb);
+      uint64_t v = kNotFound;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) v = kb[j] == q[u] ? vb[j] : v;
+      res[u] = live[u] ? v : kNotFound;
+    }
+    return;
+  }
+#endif
   // leaf: r = #keys <= q; the last key that compared <= q is key[r-1] (the successful
   // steps of the power-of-two search visit increasing slots), so the probe needs no reload
   uint32_t r[U];
@@ -840,7 +878,11 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
         const uint32_t j = b0 + u * 32 + lane;
         act[u] = j < m;
         q0[u] = act[u] ? ld_stream(a.q + c0 + j) : kPad;
+#if HM_IDX16
+        o[u] = act[u] ? (uint32_t)ld_stream16(reinterpret_cast<const uint16_t*>(a.idx) + c0 + j) : 0u;
+#else
         o[u] = act[u] ? ld_stream32(a.idx + c0 + j) : 0u;
+#endif
       }
       uint64_t res[U];
       if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
