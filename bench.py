@@ -416,8 +416,15 @@ def main():
     l2_bytes = torch.cuda.get_device_properties(dev).L2_cache_size
     nw = plan["window"] if plan["window"] else c["Q"]
     bytes_launch, noreuse_bpq = roofline_model(info, plan, nw, l2_bytes)
+    # profiling classes of the C ABI -> the kernels they time on the default staged-return path
+    kernels = {"search": "k_lane_search_c (Eq-1 descent + leaf probe, results to level-1 order)",
+               "psa_hist": "k_psa2_rank (level-1 digit + rank in tile)",
+               "psa_scatter": "k_psa2_move (level-1 staged move)",
+               "psa_scan": "k_psa2_count_sort (level-2 chunk counting sort)",
+               "return": "k_psa2_unmove (inverse move to caller order)"}
     breakdown = {k: {"ms_per_step": v[0] / a.steps, "launches_per_step": v[1] / a.steps,
-                     "share": v[0] / max(1e-9, sum(x[0] for x in prof.values()))} for k, v in prof.items()}
+                     "share": v[0] / max(1e-9, sum(x[0] for x in prof.values())),
+                     "kernels": kernels.get(k, k)} for k, v in prof.items()}
     roof = None
     if dom_kind == "search":
         avg_ms = dom_ms / dom_n

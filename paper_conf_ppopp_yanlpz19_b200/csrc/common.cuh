@@ -89,6 +89,22 @@ __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t b
   bulk_expect(bar, bytes);
   bulk_copy(dst, src, bytes, bar);
 }
+// shared -> global bulk copy (TMA store; bytes % 16 == 0, 16-byte aligned), one bulk group
+__device__ __forceinline__ void bulk_store(void* gdst, const void* ssrc, uint32_t bytes) {
+  for (uint32_t off = 0; off < bytes; off += 65536) {
+    const uint32_t sz = bytes - off < 65536 ? bytes - off : 65536;
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"((char*)gdst + off),
+                 "r"(smem_addr((const char*)ssrc + off)), "r"(sz)
+                 : "memory");
+  }
+}
+__device__ __forceinline__ void bulk_store_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+// the issuing thread: every committed bulk store has finished READING shared memory
+__device__ __forceinline__ void bulk_store_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+// the issuing thread: every committed bulk store has completed (global writes performed)
+__device__ __forceinline__ void bulk_store_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+// generic-proxy shared-memory writes become visible to the async (TMA) proxy
+__device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t b = smem_addr(bar);
   uint32_t done = 0;

@@ -21,6 +21,9 @@
 
 namespace hm {
 
+#ifndef HM_UNMOVE_TMA_STORE
+#define HM_UNMOVE_TMA_STORE 1
+#endif
 #ifndef HM_L1_WAVES
 #define HM_L1_WAVES 8
 #endif
@@ -440,6 +443,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* 
         st_od[lp] = (uint32_t)(k * C::NT + threadIdx.x) | (d << C::TILE_SHIFT);
       }
     }
+    if (HM_UNMOVE_TMA_STORE && threadIdx.x == 0) bulk_store_wait_read();  // st_r free again
     __syncthreads();
     const uint32_t tile_n = (uint32_t)std::min<uint64_t>(C::TILE, n - t0);
     uint64_t rv[C::PER];
@@ -456,10 +460,21 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* 
 #pragma unroll
     for (int k = 0; k < C::PER; ++k)
       if (k * C::NT + threadIdx.x < tile_n) st_r[oo[k]] = rv[k];
+    // TMA store of a full tile (one thread, async); the next tile's st_r writes wait above
+    const bool tma = HM_UNMOVE_TMA_STORE && tile_n == (uint32_t)C::TILE && ((uintptr_t)(out + t0) & 15) == 0;
+    if (tma) fence_proxy_async_smem();
     __syncthreads();
-    for (uint32_t i = threadIdx.x; i < tile_n; i += C::NT) out[t0 + i] = st_r[i];
-    __syncthreads();
+    if (tma) {
+      if (threadIdx.x == 0) {
+        bulk_store(out + t0, st_r, C::TILE * 8);
+        bulk_store_commit();
+      }
+    } else {
+      for (uint32_t i = threadIdx.x; i < tile_n; i += C::NT) out[t0 + i] = st_r[i];
+      __syncthreads();
+    }
   }
+  if (HM_UNMOVE_TMA_STORE && threadIdx.x == 0) bulk_store_wait_all();
 }
 template <class C>
 constexpr size_t unmove_smem() {
