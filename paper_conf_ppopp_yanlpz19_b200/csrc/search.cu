@@ -446,15 +446,9 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
 #ifndef HM_LEAF_VSPEC
 #define HM_LEAF_VSPEC 0
 #endif
-#ifndef HM_SEARCH_PF_L2
-#define HM_SEARCH_PF_L2 0
+#ifndef HM_SEARCH_TMA_STORE
+#define HM_SEARCH_TMA_STORE 0
 #endif
-// bulk L2 prefetch (TMA unit; bytes a multiple of 16, address 16-byte aligned)
-__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
-  if (bytes == 0 || ((uintptr_t)p & 15)) return;
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
-}
-
 // 256-bit read-only load of 4 consecutive keys (sm_100a LDG.E.ENL2.256; 32-byte aligned)
 __device__ __forceinline__ void ld_quad_global(const uint64_t* p, uint64_t (&k)[4]) {
   asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
@@ -859,16 +853,15 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (uint64_t c0 = (uint64_t)blockIdx.x * a.chunk; c0 < a.n; c0 += (uint64_t)gridDim.x * a.chunk) {
     const uint32_t m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
-#if HM_SEARCH_PF_L2
-    if (threadIdx.x == 0) {  // the next chunk's queries and offsets: HBM -> L2 while this one runs
-      const uint64_t c1 = c0 + (uint64_t)gridDim.x * a.chunk;
-      if (c1 < a.n) {
-        const uint32_t m1 = (uint32_t)(a.n - c1 < a.chunk ? a.n - c1 : a.chunk);
-        prefetch_l2(a.q + c1, (m1 * 8) & ~15u);
-        prefetch_l2(a.idx + c1, (m1 * 4) & ~15u);
-      }
+    // TMA store of the chunk's results (HM_SEARCH_TMA_STORE): the stage may be rewritten once
+    // the previous chunk's bulk store has read it -- checked after the first iteration's search
+    // when every warp runs the same number of iterations, else at the chunk start
+    const bool full = HM_SEARCH_TMA_STORE && m == a.chunk && a.chunk % (blockDim.x * U) == 0;
+    if (HM_SEARCH_TMA_STORE && !full) {
+      if (threadIdx.x == 0) bulk_store_wait_read();
+      __syncthreads();
     }
-#endif
+    bool first = true;
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
@@ -887,14 +880,29 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
       uint64_t res[U];
       if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
       else lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      if (full && first) {
+        if (threadIdx.x == 0) bulk_store_wait_read();
+        __syncthreads();
+      }
+      first = false;
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (act[u]) s_res[o[u]] = res[u];
     }
-    __syncthreads();
-    for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) a.out[c0 + i] = s_res[i];
-    __syncthreads();
+    if (full) {
+      fence_proxy_async_smem();
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        bulk_store(a.out + c0, s_res, m * 8);
+        bulk_store_commit();
+      }
+    } else {
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) a.out[c0 + i] = s_res[i];
+      __syncthreads();
+    }
   }
+  if (HM_SEARCH_TMA_STORE && threadIdx.x == 0) bulk_store_wait_all();
 }
 
 // ---- level-2 PSA fused with the G = 1 search (default search path) -----------------------
