@@ -69,3 +69,43 @@ def test_null_and_invalid_args_without_gpu():
     bo = hm.BuildOpts(3, 1.0, 0, 0)  # fanout not a power of two
     h = C.c_void_p()
     assert L.harmonia_build(None, None, 0, C.byref(bo), None, C.byref(h)) == 1
+
+
+def test_struct_layouts_match_the_header(tmp_path):
+    """The ctypes mirrors of the ABI structs have the header's size and field offsets (compiled
+    with gcc against include/harmonia.h; no GPU)."""
+    import ctypes as C
+
+    import paper_conf_ppopp_yanlpz19_b200 as hm
+
+    structs = {"harmonia_build_opts": hm.BuildOpts, "harmonia_query_opts": hm.QueryOpts,
+               "harmonia_plan": hm.PlanInfo, "harmonia_info": hm.Info}
+    lines = ['#include <stdio.h>', '#include "harmonia.h"', "int main(void) {"]
+    for cname, py in structs.items():
+        lines.append(f'  printf("{cname} size %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'  printf("{cname} {f} %zu\\n", offsetof({cname}, {f}));')
+    lines += ["  return 0;", "}"]
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    got = {}
+    for line in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.splitlines():
+        s, f, v = line.split()
+        got[(s, f)] = int(v)
+    for cname, py in structs.items():
+        assert got[(cname, "size")] == C.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert got[(cname, f)] == getattr(py, f).offset, (cname, f)
+
+
+def test_sass_uses_blackwell_memory_instructions():
+    """The search kernel's 256-bit leaf-block loads, the TMA bulk stores of the PSA write-outs
+    and the warp shuffles of the window rank are in the built library."""
+    from paper_conf_ppopp_yanlpz19_b200 import _build
+
+    sass = subprocess.run(["cuobjdump", "-sass", _build.LIB], capture_output=True, text=True).stdout
+    assert "LDG.E.ENL2.256" in sass  # ld.global.nc.v4.u64 (sm_100a 256-bit load)
+    assert "UBLKCP.G.S" in sass      # cp.async.bulk shared -> global (TMA store)
+    assert "SHFL.IDX" in sass
