@@ -10,9 +10,6 @@
 namespace hm {
 
 namespace {
-#ifndef HM_SMEM_ADAPTIVE
-#define HM_SMEM_ADAPTIVE 0
-#endif
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
 constexpr uint64_t kAutoWindow = 1ull << 27;  // auto PSA window (queries): measured best, DESIGN.md §8
 
@@ -71,18 +68,12 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   // top levels in BFS order while they fit
   const uint32_t ps_bytes = (uint32_t)round_up((t->I + 1) * 4, 16);
   const uint32_t limit = (uint32_t)std::min<size_t>(t->smem_optin > 1024 ? t->smem_optin - 1024 : 0, 200 * 1024);
-  uint32_t budget = o->smem_levels > 0 ? limit : std::min(kSmemBudget, limit);
-  // staged-return G = 1 path: two 1024-thread CTAs per SM share the SM's shared memory with
-  // their chunk stages, so the top plan may take what the stages leave (PS of larger trees)
+  const uint32_t budget = o->smem_levels > 0 ? limit : std::min(kSmemBudget, limit);
+  // (a larger budget that stages the PS of bigger trees was measured 1.7-2.4x slower at c3:
+  // the shared memory it takes comes out of the L1 that caches the leaves)
   const uint64_t qpl = t->L ? std::min<uint64_t>(n, P.window) / t->L : 0;
   P.chunk = o->sort_chunk == kPsaChunkMax || (o->sort_chunk == 0 && qpl >= kChunk8kMinQueriesPerLeaf)
                 ? kPsaChunkMax : kPsaChunk;
-  const bool staged_cand = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather && !P.fuse &&
-                           !(o->flags & HARMONIA_QF_SCATTER_RETURN);
-  if (HM_SMEM_ADAPTIVE && staged_cand && o->smem_levels == 0) {
-    const int64_t room = (int64_t)t->smem_per_sm / 2 - (int64_t)P.chunk * 8 - 2048;
-    if (room > (int64_t)budget) budget = (uint32_t)std::min<int64_t>(room, limit);
-  }
   uint32_t used = 0;
   int lv = 0;
   if (o->smem_levels >= 0) {

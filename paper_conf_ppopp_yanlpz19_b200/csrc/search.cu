@@ -446,6 +446,9 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
 #ifndef HM_LEAF_VSPEC
 #define HM_LEAF_VSPEC 0
 #endif
+#ifndef HM_CARVEOUT
+#define HM_CARVEOUT 0
+#endif
 #ifndef HM_SEARCH_TMA_STORE
 #define HM_SEARCH_TMA_STORE 0
 #endif
@@ -1327,6 +1330,18 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     configured_smem[ci] = (int)smem;
   }
+#if HM_CARVEOUT
+  {  // ask for the smallest shared-memory carveout that holds two CTAs: the rest is L1, which
+     // caches the tree lines PSA neighbours share
+    static int last_pct[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
+    const size_t need = 2 * ((size_t)smem + 1024);
+    const int pct = (int)std::min<size_t>(100, (need * 100 + t->smem_per_sm - 1) / std::max<size_t>(t->smem_per_sm, 1));
+    if (pct != last_pct[ci]) {
+      HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, pct));
+      last_pct[ci] = pct;
+    }
+  }
+#endif
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, smem));
   per_sm = std::max(per_sm, 1);
