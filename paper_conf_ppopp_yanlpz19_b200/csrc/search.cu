@@ -443,15 +443,6 @@ __global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_lane_search(
   }
 }
 
-#ifndef HM_LEAF_VSPEC
-#define HM_LEAF_VSPEC 0
-#endif
-#ifndef HM_CARVEOUT
-#define HM_CARVEOUT 0
-#endif
-#ifndef HM_SEARCH_TMA_STORE
-#define HM_SEARCH_TMA_STORE 0
-#endif
 // 256-bit read-only load of 4 consecutive keys (sm_100a LDG.E.ENL2.256; 32-byte aligned)
 __device__ __forceinline__ void ld_quad_global(const uint64_t* p, uint64_t (&k)[4]) {
   asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];"
@@ -546,36 +537,6 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
 #pragma unroll
     for (int u = 0; u < U; ++u) node[u] = first[u] + r[u];  // Eq 1
   }
-#if HM_LEAF_VSPEC
-  // leaf, speculative value block: binary lifting on #keys < q down to a 4-slot block; then
-  // (invariant r <= #keys < q < r + 4) a key equal to q can only sit in [r, r+4), so the
-  // block's 4 keys and its 4 values (each one 32-byte sector) are read together -- the
-  // value no longer waits for the rank.  Keys are unique: at most one slot matches.
-  if (F >= 8 && !leaf_smem) {
-    uint32_t r[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) r[u] = 0;
-#pragma unroll
-    for (int s = F / 2; s >= 4; s >>= 1) {
-      uint64_t k[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) k[u] = ld_key_global(a.keys + (uint64_t)node[u] * F + (r[u] + s - 1));
-#pragma unroll
-      for (int u = 0; u < U; ++u) r[u] += k[u] < q[u] ? s : 0;
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      uint64_t kb[4], vb[4];
-      ld_quad_global(a.keys + (uint64_t)node[u] * F + r[u], kb);
-      ld_quad_global(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + r[u], vb);
-      uint64_t v = kNotFound;
-#pragma unroll
-      for (int j = 0; j < 4; ++j) v = kb[j] == q[u] ? vb[j] : v;
-      res[u] = live[u] ? v : kNotFound;
-    }
-    return;
-  }
-#endif
   // leaf: r = #keys <= q; the last key that compared <= q is key[r-1] (the successful
   // steps of the power-of-two search visit increasing slots), so the probe needs no reload
   uint32_t r[U];
@@ -856,15 +817,6 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   for (uint64_t c0 = (uint64_t)blockIdx.x * a.chunk; c0 < a.n; c0 += (uint64_t)gridDim.x * a.chunk) {
     const uint32_t m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
-    // TMA store of the chunk's results (HM_SEARCH_TMA_STORE): the stage may be rewritten once
-    // the previous chunk's bulk store has read it -- checked after the first iteration's search
-    // when every warp runs the same number of iterations, else at the chunk start
-    const bool full = HM_SEARCH_TMA_STORE && m == a.chunk && a.chunk % (blockDim.x * U) == 0;
-    if (HM_SEARCH_TMA_STORE && !full) {
-      if (threadIdx.x == 0) bulk_store_wait_read();
-      __syncthreads();
-    }
-    bool first = true;
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
@@ -883,29 +835,14 @@ __global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
       uint64_t res[U];
       if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
       else lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
-      if (full && first) {
-        if (threadIdx.x == 0) bulk_store_wait_read();
-        __syncthreads();
-      }
-      first = false;
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (act[u]) s_res[o[u]] = res[u];
     }
-    if (full) {
-      fence_proxy_async_smem();
-      __syncthreads();
-      if (threadIdx.x == 0) {
-        bulk_store(a.out + c0, s_res, m * 8);
-        bulk_store_commit();
-      }
-    } else {
-      __syncthreads();
-      for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) a.out[c0 + i] = s_res[i];
-      __syncthreads();
-    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) a.out[c0 + i] = s_res[i];
+    __syncthreads();
   }
-  if (HM_SEARCH_TMA_STORE && threadIdx.x == 0) bulk_store_wait_all();
 }
 
 // ---- level-2 PSA fused with the G = 1 search (default search path) -----------------------
@@ -1330,18 +1267,6 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
     HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     configured_smem[ci] = (int)smem;
   }
-#if HM_CARVEOUT
-  {  // ask for the smallest shared-memory carveout that holds two CTAs: the rest is L1, which
-     // caches the tree lines PSA neighbours share
-    static int last_pct[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
-    const size_t need = 2 * ((size_t)smem + 1024);
-    const int pct = (int)std::min<size_t>(100, (need * 100 + t->smem_per_sm - 1) / std::max<size_t>(t->smem_per_sm, 1));
-    if (pct != last_pct[ci]) {
-      HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, pct));
-      last_pct[ci] = pct;
-    }
-  }
-#endif
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, smem));
   per_sm = std::max(per_sm, 1);
