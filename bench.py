@@ -262,6 +262,11 @@ def main():
     if world > 1 or a.mode in ("partitioned", "peer"):
         import torch.distributed as dist
 
+        if world == 1:  # a one-rank group without torchrun (--mode partitioned/peer at N = 1)
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", str(29500 + os.getpid() % 1000))
+            os.environ.setdefault("RANK", "0")
+            os.environ.setdefault("WORLD_SIZE", "1")
         dist.init_process_group("nccl", device_id=dev)
         pg = dist
 

@@ -77,7 +77,11 @@ typedef struct {
                            (1, 2 or 4; 0 = auto)                                            */
   uint32_t sort_chunk;   /* staged-return PSA: level-2 chunk in queries, 4096 or 8192; 0 = auto
                            (8192 when the window holds >= 192 queries per leaf)            */
-  uint64_t reserved1;
+  uint64_t l2_window_bytes; /* search kernels: bytes of the unstaged internal key region pinned
+                           in L2 by an access-policy window (persisting hits, streaming
+                           misses): 0 = auto = all of it (capped by the device's window and
+                           persisting-L2 limits); disable with HARMONIA_QF_NO_L2_WINDOW.  The
+                           first windowed call sets the device's cudaLimitPersistingL2CacheSize. */
 } harmonia_query_opts;
 
 #define HARMONIA_QF_NO_PS_SMEM 1u  /* do not stage the prefix-sum array in shared memory     */
@@ -100,6 +104,7 @@ typedef struct {
                                       load-ballot-store step per 2G slots) instead of the
                                       default warp-per-range resolve-then-copy kernel; also
                                       implied by an explicit group_size                      */
+#define HARMONIA_QF_NO_L2_WINDOW 4096u /* no L2 access-policy window on the search kernels   */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic
@@ -326,6 +331,7 @@ typedef struct {
   uint32_t lane_queries;   /* G = 1: queries interleaved per lane */
   uint32_t warp_shared;    /* 1: G = 1 warp-shared descent (see HARMONIA_QF_PER_LANE) */
   uint32_t sort_chunk;     /* staged return: level-2 chunk (queries); 0 when not staged */
+  uint64_t l2_window_bytes; /* bytes of the internal key region pinned in L2 (0 = none) */
 } harmonia_plan;
 harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
                                     const harmonia_query_opts* opts, harmonia_plan* out);

@@ -29,6 +29,7 @@ QF_PSA_LSD = 64
 QF_FUSE_SORT = 128
 QF_SCATTER_RETURN = 256
 QF_PSA_WIDE = 512
+QF_NO_L2_WINDOW = 4096
 QF_PER_LANE = 1024
 QF_RANGE_GROUP = 2048
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
@@ -52,14 +53,15 @@ class BuildOpts(C.Structure):
 class QueryOpts(C.Structure):
     _fields_ = [("group_size", C.c_int32), ("psa_bits", C.c_int32), ("smem_levels", C.c_int32),
                 ("flags", C.c_int32), ("window", C.c_uint64), ("lane_queries", C.c_uint32),
-                ("sort_chunk", C.c_uint32), ("reserved1", C.c_uint64)]
+                ("sort_chunk", C.c_uint32), ("l2_window_bytes", C.c_uint64)]
 
 
 class PlanInfo(C.Structure):
     _fields_ = [("group_size", C.c_int32), ("psa_bits", C.c_int32), ("smem_levels", C.c_int32),
                 ("ps_in_smem", C.c_int32), ("window", C.c_uint64), ("smem_bytes", C.c_uint32),
                 ("smem_nodes", C.c_uint32), ("staged_return", C.c_uint32), ("lane_queries", C.c_uint32),
-                ("warp_shared", C.c_uint32), ("sort_chunk", C.c_uint32)]
+                ("warp_shared", C.c_uint32), ("sort_chunk", C.c_uint32),
+                ("l2_window_bytes", C.c_uint64)]
 
 
 class Info(C.Structure):
@@ -205,11 +207,12 @@ def _as_u64_dev(t, device):
 
 
 def make_opts(group_size=0, psa_bits=0, smem_levels=0, window=0, flags=0, lane_queries=0,
-              sort_chunk=0) -> QueryOpts:
+              sort_chunk=0, l2_window_bytes=0) -> QueryOpts:
     o = QueryOpts()
     o.group_size, o.psa_bits, o.smem_levels, o.flags, o.window = group_size, psa_bits, smem_levels, flags, window
     o.lane_queries = lane_queries
     o.sort_chunk = sort_chunk
+    o.l2_window_bytes = l2_window_bytes
     return o
 
 

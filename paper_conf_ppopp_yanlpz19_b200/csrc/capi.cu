@@ -10,6 +10,9 @@
 namespace hm {
 
 namespace {
+#ifndef HM_L2_WINDOW
+#define HM_L2_WINDOW 1
+#endif
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
 constexpr uint64_t kAutoWindow = 1ull << 27;  // auto PSA window (queries): measured best, DESIGN.md §8
 
@@ -98,6 +101,21 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
           !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
           2 * (round_up(P.smem_bytes, 16) + P.chunk * 8 + 1024) <= t->smem_per_sm;
   if (!P.ret || P.fuse) P.chunk = kPsaChunk;
+  // L2 access-policy window over the internal levels below the staged top (north_star (c):
+  // the upper levels are pinned in L2 while leaves, values and query streams pass through)
+  if (HM_L2_WINDOW && !(o->flags & HARMONIA_QF_NO_L2_WINDOW) && t->l2_window_max && t->l2_persist_max && t->h > 1 &&
+      t->d_keys) {
+    const uint64_t leaf0 = t->level_start[t->h - 1];
+    const uint64_t first = std::min<uint64_t>(P.smem_nodes, leaf0);
+    uint64_t bytes = (leaf0 - first) * t->F * 8;
+    if (o->l2_window_bytes) bytes = std::min<uint64_t>(bytes, o->l2_window_bytes);
+    bytes = std::min<uint64_t>(bytes, t->l2_window_max);
+    if (bytes) {
+      P.l2_base = t->d_keys + first * t->F;
+      P.l2_bytes = bytes;
+      P.l2_hit = (float)std::min(1.0, (double)t->l2_persist_max / (double)bytes);
+    }
+  }
   P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
   P.coop = P.ret && !(o->flags & HARMONIA_QF_PER_LANE);
   // ranges: the warp-per-range copy kernel unless a group size was requested explicitly or
@@ -125,9 +143,30 @@ static SearchArgs search_args(const harmonia_tree* t, const Plan& p) {
   return a;
 }
 
+// The device's persisting-L2 set-aside must cover the window (cudaLimitPersistingL2CacheSize
+// is device-wide; raised once, never lowered by the library).  false: no window this call.
+static bool ensure_l2_persist(const harmonia_tree* tc, size_t bytes) {
+  harmonia_tree* t = const_cast<harmonia_tree*>(tc);
+  const size_t want = std::min(bytes, t->l2_persist_max);
+  if (t->l2_persist_set >= want) return true;
+  size_t cur = 0;
+  if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess && cur >= want) {
+    t->l2_persist_set = cur;
+    return true;
+  }
+  if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  t->l2_persist_set = want;
+  return true;
+}
+
 static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, uint64_t n, uint64_t* out,
-                                     void* ws, const Plan& p, cudaStream_t st) {
+                                     void* ws, const Plan& p_in, cudaStream_t st) {
   if (n == 0) return HARMONIA_OK;
+  Plan p = p_in;
+  if (p.l2_bytes && !ensure_l2_persist(t, p.l2_bytes)) p.l2_bytes = 0;
   if (t->n_keys == 0) {  // C-A17: empty tree, every query is absent
     HM_CUDA(cudaMemsetAsync(out, 0xFF, n * 8, st));
     return HARMONIA_OK;
@@ -247,6 +286,7 @@ extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t 
   out->lane_queries = p.G == 1 ? (uint32_t)p.lane_ilp : 0u;
   out->warp_shared = p.coop ? 1u : 0u;
   out->sort_chunk = p.ret ? p.chunk : 0u;
+  out->l2_window_bytes = p.l2_bytes;
   return HARMONIA_OK;
 }
 
@@ -338,6 +378,7 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   cudaStream_t st = (cudaStream_t)stream;
   Plan p;
   harmonia_status s = make_plan(t, n, o, &p);
+  if (s == HARMONIA_OK && p.l2_bytes && !ensure_l2_persist(t, p.l2_bytes)) p.l2_bytes = 0;
   if (s != HARMONIA_OK) return s;
   if (t->n_keys == 0) {
     HM_CUDA(cudaMemsetAsync(d_counts, 0, n * 4, st));

@@ -169,6 +169,8 @@ struct harmonia_tree {
   size_t smem_optin = 0;
   size_t smem_per_sm = 0;
   size_t l2_bytes = 0;
+  size_t l2_persist_max = 0, l2_window_max = 0;  // device limits for the access-policy window
+  size_t l2_persist_set = 0;                     // cudaLimitPersistingL2CacheSize this tree set
   // host-pipeline streams/events (harmonia_search_batch_host)
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
   cudaEvent_t ev_start = nullptr, ev_in[2] = {}, ev_done[2] = {}, ev_out[2] = {};
@@ -202,7 +204,33 @@ struct Plan {
   bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
   bool range_warp = true;    // ranges: one warp per range, resolve then stream-copy (k_range_warp)
   uint32_t chunk = 4096;     // staged return: level-2 chunk (4096 or kPsaChunkMax queries)
+  const void* l2_base = nullptr;  // L2 access-policy window over the unstaged internal levels
+  size_t l2_bytes = 0;
+  float l2_hit = 0.f;
 };
+
+// Launch kern(a) on st, carrying the plan's L2 access-policy window (if any) as a launch
+// attribute: hits on the window persist in L2, everything else streams (north_star (c)).
+template <typename Kern, typename Args>
+cudaError_t launch_win(Kern kern, dim3 grid, dim3 block, size_t smem, cudaStream_t st, const Plan& p, const Args& a) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  if (p.l2_bytes) {
+    at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+    at[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(p.l2_base);
+    at[0].val.accessPolicyWindow.num_bytes = p.l2_bytes;
+    at[0].val.accessPolicyWindow.hitRatio = p.l2_hit;
+    at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+  }
+  return cudaLaunchKernelEx(&cfg, kern, a);
+}
 
 harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_query_opts* o,
                           Plan* p);

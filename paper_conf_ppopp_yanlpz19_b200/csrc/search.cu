@@ -1227,7 +1227,7 @@ harmonia_status launch_range_warp_f(const harmonia_tree* t, const Plan& p, const
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_RANGE, st);
-    kern<<<grid, 1024, p.smem_bytes, st>>>(a);
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(1024), p.smem_bytes, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
@@ -1249,7 +1249,7 @@ harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, cons
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    kern<<<grid, kFuseThreads, smem, st>>>(a);
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(kFuseThreads), smem, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
@@ -1274,7 +1274,7 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    kern<<<grid, 1024, smem, st>>>(a);
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(1024), smem, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
@@ -1299,7 +1299,7 @@ harmonia_status launch_lane_search(const harmonia_tree* t, const Plan& p, const 
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    kern<<<grid, bs, p.smem_bytes, st>>>(a);
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(bs), p.smem_bytes, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
@@ -1322,7 +1322,7 @@ harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const Se
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    kern<<<grid, kQueryBlock, p.smem_bytes, st>>>(a);
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(kQueryBlock), p.smem_bytes, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
@@ -1344,7 +1344,7 @@ harmonia_status launch_range_fg(const harmonia_tree* t, const Plan& p, const Ran
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_RANGE, st);
-    kern<<<grid, kQueryBlock, p.smem_bytes, st>>>(a);
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(kQueryBlock), p.smem_bytes, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;

@@ -283,6 +283,8 @@ extern "C" harmonia_status harmonia_build(const uint64_t* keys, const uint64_t* 
   t->smem_optin = prop.sharedMemPerBlockOptin;
   t->smem_per_sm = prop.sharedMemPerMultiprocessor;
   t->l2_bytes = prop.l2CacheSize;
+  t->l2_persist_max = prop.persistingL2CacheMaxSize;
+  t->l2_window_max = prop.accessPolicyMaxWindowSize;
 
   if (on_dev && n > 0) {
     cudaPointerAttributes pa;

@@ -338,3 +338,28 @@ def test_config2_full_size_sampled(hm, orc):
     assert np.array_equal(out, gen.values_for(q))
     sel = gen._stream(77, 0, 1 << 20) % np.uint64(Q)
     assert np.array_equal(out[sel], orc.sorted_search(keys, vals, q[sel]))
+
+
+def test_l2_access_policy_window(hm, orc):
+    """The search kernels carry an L2 access-policy window over the internal levels below the
+    staged top (north_star (c)); it changes no result.  Plan reporting, the opt-out flag and
+    an explicit byte cap."""
+    keys = gen.uniform_keys(1 << 18)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 16)
+    inf = t.info()
+    leaf0 = inf["level_start"][inf["height"] - 1]
+    pl = t.plan(1 << 18)
+    internal_unstaged = (leaf0 - min(pl["smem_nodes"], leaf0)) * 16 * 8
+    assert 0 < pl["l2_window_bytes"] <= internal_unstaged
+    assert t.plan(1 << 18, flags=hm.QF_NO_L2_WINDOW)["l2_window_bytes"] == 0
+    assert t.plan(1 << 18, l2_window_bytes=4096)["l2_window_bytes"] == 4096
+    q = np.concatenate([gen.uniform_queries(keys, 200003, miss_frac=0.3), gen.edge_queries(keys)])
+    exp = orc.sorted_search(keys, vals, q)
+    for kw in ({}, {"flags": hm.QF_NO_L2_WINDOW}, {"l2_window_bytes": 4096}, {"group_size": 4},
+               {"psa_bits": -1}):
+        assert np.array_equal(host(t.search(cu(q), **kw)), exp), kw
+    lo, hi = gen.ranges(keys, 5000, 64)
+    ko, vo, cnt = t.range(cu(lo), cu(hi), 64)
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, 64)
+    assert np.array_equal(host(cnt), ecnt) and np.array_equal(host(ko), eko) and np.array_equal(host(vo), evo)
