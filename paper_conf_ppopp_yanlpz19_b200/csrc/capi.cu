@@ -13,6 +13,9 @@ namespace {
 #ifndef HM_L2_WINDOW
 #define HM_L2_WINDOW 1
 #endif
+#ifndef HM_L2_WINDOW_DIV
+#define HM_L2_WINDOW_DIV 8
+#endif
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
 constexpr uint64_t kAutoWindow = 1ull << 27;  // auto PSA window (queries): measured best, DESIGN.md §8
 
@@ -110,6 +113,9 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
     uint64_t bytes = (leaf0 - first) * t->F * 8;
     if (o->l2_window_bytes) bytes = std::min<uint64_t>(bytes, o->l2_window_bytes);
     bytes = std::min<uint64_t>(bytes, t->l2_window_max);
+    // at most L2 / HM_L2_WINDOW_DIV: lines pinned across calls take L2 from the streaming PSA
+    // passes (an 88 MB window at c3 F8 made the move pass 3x slower)
+    bytes = std::min<uint64_t>(bytes, t->l2_bytes / HM_L2_WINDOW_DIV);
     if (bytes) {
       P.l2_base = t->d_keys + first * t->F;
       P.l2_bytes = bytes;
