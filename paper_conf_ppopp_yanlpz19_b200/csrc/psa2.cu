@@ -801,7 +801,11 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
 #define HM_SORT_CTAS_PER_SM 4
 #endif
     const uint32_t ch = (local && level2 == 0 && chunk == kPsaChunkMax) ? kPsaChunkMax : (uint32_t)kChunk;
-    const int g = (int)std::min<uint64_t>(ceil_div(n, ch), (uint64_t)sm * HM_SORT_CTAS_PER_SM);
+#ifndef HM_SORT_CTAS_PER_SM_8K
+#define HM_SORT_CTAS_PER_SM_8K 1  // one resident CTA per SM: persistent, one TMA prefetch chain each
+#endif
+    const int cps = ch == kPsaChunkMax ? HM_SORT_CTAS_PER_SM_8K : HM_SORT_CTAS_PER_SM;
+    const int g = (int)std::min<uint64_t>(ceil_div(n, ch), (uint64_t)sm * cps);
     if (level2 == 1)  // two stable LSD passes of ballot multisplit (ablation)
       k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
     else if (local && ch == kPsaChunkMax)  // 8192-query chunks (denser key ranges per warp)
