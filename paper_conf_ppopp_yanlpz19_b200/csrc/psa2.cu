@@ -212,10 +212,24 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_rank(const uint64_t* __
     __syncthreads();
     if (pf && threadIdx.x == 0 && tile + 1 < te)
       bulk_load(sq, q + (tile + 1) * C::TILE, tile_bytes<C>(tile + 1, n, 8), &bar);
+    // Router digits (few destinations): warp-aggregated ranks -- one shared atomic per distinct
+    // digit per warp (lanes with equal digits found by MATCH.ANY); with P <= 8 shards a warp
+    // otherwise serialises up to 32 atomics on one counter.  The PSA coarse digit (256 bins,
+    // ~30 distinct per warp) keeps one atomic per query.
+    constexpr bool kAgg = !std::is_same<Digit, CoarseDigit>::value;
 #pragma unroll
     for (int k = 0; k < C::PER; ++k) {
       const uint64_t e = t0 + k * C::NT + threadIdx.x;
-      if (e < n) {
+      if constexpr (kAgg) {
+        const bool in = e < n;  // every lane takes part in the match (tile tails)
+        const uint32_t d = in ? dg(v[k]) : 0xFFFFFFFFu;
+        const unsigned peers = __match_any_sync(kFull, d);
+        const unsigned lane = threadIdx.x & 31, leader = __ffs(peers) - 1;
+        uint32_t base = 0;
+        if (in && lane == leader) base = atomicAdd(&cnt[d], (uint32_t)__popc(peers));
+        base = __shfl_sync(kFull, base, leader);
+        if (in) packed[e] = d | ((base + __popc(peers & ((1u << lane) - 1))) << C::BITS);
+      } else if (e < n) {
         const uint32_t d = dg(v[k]);
         packed[e] = d | (atomicAdd(&cnt[d], 1u) << C::BITS);
       }
