@@ -17,9 +17,12 @@ import harmonia_gen as gen  # noqa: E402
 import paper_conf_ppopp_yanlpz19_b200 as hm  # noqa: E402
 
 
-def timed(fn, reps):
+def timed(fn, reps, warm=2):
+    # two warm-up calls: an update batch alternates the live and spare layout buffers, so the
+    # second call is the one that grows the spare set after the first call grew the tree
     s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    fn()
+    for _ in range(warm):
+        fn()
     torch.cuda.synchronize()
     s0.record()
     for _ in range(reps):
