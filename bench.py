@@ -462,6 +462,12 @@ def main():
             if "l1_wavefront_pct" in ent:  # the on-chip limiter of the search
                 roof["limiter"] = {"resource": "L1 data-pipe (LSU) wavefronts", "frac": ent["l1_wavefront_pct"] / 100,
                                    "source": ent.get("source")}
+            if ent.get("sol_pct"):  # ncu speed-of-light of every tier: none saturated -> latency-bound
+                roof["ncu_sol"] = {k: v / 100 for k, v in ent["sol_pct"].items()}
+                if ent.get("ncu_time_s"):  # DRAM GB/s of the captured launch vs the measured peak
+                    roof["ncu_sol"]["dram"] = ent["dram_bytes_per_launch"] / ent["ncu_time_s"] / 1e9 / hbm_peak
+                if "long_scoreboard_stall_share" in ent:
+                    roof["ncu_sol"]["long_scoreboard_stall_share"] = ent["long_scoreboard_stall_share"]
     except Exception:
         pass
 

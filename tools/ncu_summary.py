@@ -111,6 +111,17 @@ if __name__ == "__main__":
         l1 = d.get("l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed")
         if isinstance(l1, float):
             ent["l1_wavefront_pct"] = l1
+        # speed-of-light fractions of each tier / pipe (which one binds the kernel)
+        sol = {"l2": d.get("lts__throughput.avg.pct_of_peak_sustained_elapsed"),
+               "dram": d.get("dram__throughput.avg.pct_of_peak_sustained_elapsed"),
+               "l1_lsu": l1, "issue": d.get("smsp__issue_active.avg.pct_of_peak_sustained_active")}
+        ent["sol_pct"] = {k: v for k, v in sol.items() if isinstance(v, float)}
+        tv, tu = d.get("gpu__time_duration.sum"), d.get("gpu__time_duration.sum.unit", "nsecond")
+        if isinstance(tv, float):  # capture duration: DRAM GB/s of this launch = bytes / time
+            ent["ncu_time_s"] = tv * {"ns": 1e-9, "nsecond": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3, "msecond": 1e-3, "s": 1.0, "second": 1.0}.get(tu, 1e-9)
+        st = d.get("stall_share")
+        if isinstance(st, dict) and "long_scoreboard" in st:
+            ent["long_scoreboard_stall_share"] = st["long_scoreboard"]
         tr.setdefault(a.workload, {})[k] = ent  # the newest capture supersedes
     json.dump(tr, open(tr_path, "w"), indent=1)
     with open(a.out + ".md", "w") as f:
