@@ -24,6 +24,12 @@ namespace hm {
 #ifndef HM_UNMOVE_TMA_STORE
 #define HM_UNMOVE_TMA_STORE 1
 #endif
+#ifndef HM_MOVE_MINB
+#define HM_MOVE_MINB 4
+#endif
+#ifndef HM_UNMOVE_MINB
+#define HM_UNMOVE_MINB 4
+#endif
 #ifndef HM_L1_WAVES
 #define HM_L1_WAVES 8
 #endif
@@ -263,7 +269,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_rank(const uint64_t* __
 // straight into the receive buffer of rank d (a peer-mapped device pointer, NVLink stores),
 // push_dst[d] = address of this rank's segment there; nothing is written locally.
 template <class Digit, class C, bool kIdx, bool kPush = false>
-__global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
+__global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? HM_MOVE_MINB : C::MINB)) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
                                                               const uint32_t* __restrict__ counts,
                                                               uint32_t* __restrict__ cursor,
                                                               const uint32_t* __restrict__ tile_counts,
@@ -396,7 +402,7 @@ constexpr size_t move_smem() {
 // gbase rebuilt from the CTA base, so res1 is read in runs and out[] written contiguously --
 // no scattered global access on either side.
 template <class C>
-__global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_unmove(const uint32_t* __restrict__ tile_counts,
+__global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? HM_UNMOVE_MINB : C::MINB)) k_psa2_unmove(const uint32_t* __restrict__ tile_counts,
                                                                 const uint32_t* __restrict__ cta_base,
                                                                 const uint32_t* __restrict__ packed,
                                                                 const uint64_t* __restrict__ res1, uint64_t n,
