@@ -31,7 +31,7 @@ namespace hm {
 #define HM_UNMOVE_MINB 4
 #endif
 #ifndef HM_L1_WAVES
-#define HM_L1_WAVES 8
+#define HM_L1_WAVES 6
 #endif
 #ifndef HM_L1_WAVES_MV
 #define HM_L1_WAVES_MV 16
@@ -629,7 +629,7 @@ constexpr size_t count_sort_smem() {
 
 // level-1 grids: CTAs own contiguous tile ranges, ~2048 resident threads per SM, waves x the
 // resident CTAs.  The rank pass and the move/unmove pair may use different wave counts (the
-// move then sums its CTA's per-tile counts itself): measured best 8 for the rank pass, 16 for
+// move then sums its CTA's per-tile counts itself): measured best 6 for the rank pass (4-8 within 4 %), 16 for
 // the move and its inverse.
 template <class C>
 int l1_grid(uint64_t n, int sm, int waves = HM_L1_WAVES) {
