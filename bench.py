@@ -214,7 +214,8 @@ def roofline_model(info, plan, nq_window, l2_bytes):
     """Algorithmic bytes of the search kernel.
 
     Per launch over one PSA window of nw queries:
-      I/O: 8 B query + 4 B position + 8 B result per query (16 B without PSA);
+      I/O: 8 B query + position + 8 B result per query: the staged return reads a 2-B
+           chunk-local offset (18 B), the other PSA paths a 4-B position (20 B), no PSA 16 B;
       tree: every level not staged in shared memory is charged min(no-reuse, whole level):
             no-reuse = nw x (S + 32) (node + one 32-B PS / value sector), whole level =
             nodes x S (+ the level's values for the leaf level).
@@ -222,7 +223,7 @@ def roofline_model(info, plan, nq_window, l2_bytes):
     F, h = info["fanout"], info["height"]
     S = F * 8
     ls = info["level_start"]
-    io = 20 if plan["psa_bits"] > 0 else 16
+    io = (18 if plan.get("staged_return") else 20) if plan["psa_bits"] > 0 else 16
     tree = 0
     noreuse = io
     for lev in range(plan["smem_levels"], h):
