@@ -804,8 +804,11 @@ __global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const 
 // back to level-1 order in shared memory and written contiguously -- the scattered 8-byte
 // stores to out[original position] (measured: a third of the kernel) are replaced by
 // k_psa2_unmove's run-wise copy.
+#ifndef HM_SEARCH_NT
+#define HM_SEARCH_NT 1024  // threads per staged-search CTA (2 CTAs per SM)
+#endif
 template <int F, int U, bool COOP>
-__global__ void __launch_bounds__(1024, 2) k_lane_search_c(const SearchArgs a) {
+__global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
   stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
@@ -1260,6 +1263,9 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   const int U = p.lane_ilp;
   auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
                      : (U >= 4 ? k_lane_search_c<F, 4, false> : (U == 2 ? k_lane_search_c<F, 2, false> : k_lane_search_c<F, 1, false>));
+#if HM_SEARCH_U3
+  if (U == 3) kern = a.coop ? k_lane_search_c<F, 3, true> : k_lane_search_c<F, 3, false>;
+#endif
   const uint32_t smem = a.res_smem_off + a.chunk * 8;
   static int configured_smem[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
   const int ci = (U >= 4 ? 4 : U) + (a.coop ? 5 : 0);
@@ -1268,13 +1274,13 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
     configured_smem[ci] = (int)smem;
   }
   int per_sm = 0;
-  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, smem));
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, HM_SEARCH_NT, smem));
   per_sm = std::max(per_sm, 1);
   const uint64_t need = ceil_div(a.n, (uint64_t)a.chunk);
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    HM_CUDA(launch_win(kern, dim3(grid), dim3(1024), smem, st, p, a));
+    HM_CUDA(launch_win(kern, dim3(grid), dim3(HM_SEARCH_NT), smem, st, p, a));
   }
   HM_LAUNCHED();
   return HARMONIA_OK;
