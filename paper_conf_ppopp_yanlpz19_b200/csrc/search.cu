@@ -1263,9 +1263,6 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   const int U = p.lane_ilp;
   auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
                      : (U >= 4 ? k_lane_search_c<F, 4, false> : (U == 2 ? k_lane_search_c<F, 2, false> : k_lane_search_c<F, 1, false>));
-#if HM_SEARCH_U3
-  if (U == 3) kern = a.coop ? k_lane_search_c<F, 3, true> : k_lane_search_c<F, 3, false>;
-#endif
   const uint32_t smem = a.res_smem_off + a.chunk * 8;
   static int configured_smem[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
   const int ci = (U >= 4 ? 4 : U) + (a.coop ? 5 : 0);
