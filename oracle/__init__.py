@@ -67,6 +67,7 @@ def lib():
             "orc_bpt_size": (C.c_uint64, [C.c_void_p]),
             "orc_bpt_height": (C.c_uint32, [C.c_void_p]),
             "orc_bpt_check": (C.c_int, [C.c_void_p]),
+            "orc_bpt_debug_mutate": (C.c_int, [C.c_void_p, C.c_int]),
             "orc_bpt_dump": (None, [C.c_void_p, u64p, u64p]),
             "orc_bpt_level_stats": (None, [C.c_void_p, u64p, u64p, C.c_uint32]),
             "orc_bpt_quarter_stats": (None, [C.c_void_p, u64p, C.c_uint64, u64p]),
@@ -84,9 +85,9 @@ def lib():
             "orc_psa_order": (None, [u64p, C.c_uint64, C.c_uint32, C.c_uint64, C.c_uint64, u64p]),
             "orc_ntg_steps": (C.c_uint32, [C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32]),
             "orc_ntg_warp_steps": (C.c_double, [u64p, u32p, C.c_uint32, C.c_uint32, u64p, u64p, C.c_uint64,
-                                                C.c_uint32, C.c_uint32, C.c_uint32]),
+                                                C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32]),
             "orc_ntg_choose_gs": (C.c_uint32, [u64p, u32p, C.c_uint32, C.c_uint32, u64p, u64p, C.c_uint64,
-                                               C.c_uint32, C.c_uint32, C.c_uint32]),
+                                               C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32]),
             "orc_warp_transactions": (C.c_double, [u64p, u32p, C.c_uint32, C.c_uint32, u64p, u64p,
                                                    C.c_uint64, C.c_uint32]),
             "orc_map_create": (C.c_void_p, [u64p, u64p, C.c_uint64]),
@@ -197,6 +198,10 @@ class BPlusTree:
     def check(self) -> int:
         return int(lib().orc_bpt_check(self._h))
 
+    def debug_mutate(self, kind: int) -> bool:
+        """Test hook: corrupt the tree one way (bptree.cc orc_bpt_debug_mutate)."""
+        return bool(lib().orc_bpt_debug_mutate(self._h, kind))
+
     def dump(self):
         n = len(self)
         k = np.empty(n, dtype=np.uint64)
@@ -270,15 +275,15 @@ class Layout:
     def _args(self):
         return (_p64(self.key_region), _p32(self.ps), self.F, self.h, _p64(self.level_start))
 
-    def ntg_warp_steps(self, q, gs, kpl=2, lev0=0) -> float:
+    def ntg_warp_steps(self, q, gs, kpl=2, lev0=0, warp=32) -> float:
         q = _u64(q)
         kr, ps, F, h, ls = self._args()
-        return float(lib().orc_ntg_warp_steps(kr, ps, F, h, ls, _p64(q), q.shape[0], gs, kpl, lev0))
+        return float(lib().orc_ntg_warp_steps(kr, ps, F, h, ls, _p64(q), q.shape[0], gs, kpl, lev0, warp))
 
-    def ntg_choose_gs(self, q, gs0, kpl=2, lev0=0) -> int:
+    def ntg_choose_gs(self, q, gs0, kpl=2, lev0=0, warp=32) -> int:
         q = _u64(q)
         kr, ps, F, h, ls = self._args()
-        return int(lib().orc_ntg_choose_gs(kr, ps, F, h, ls, _p64(q), q.shape[0], gs0, kpl, lev0))
+        return int(lib().orc_ntg_choose_gs(kr, ps, F, h, ls, _p64(q), q.shape[0], gs0, kpl, lev0, warp))
 
     def warp_transactions(self, q, queries_per_warp) -> float:
         q = _u64(q)

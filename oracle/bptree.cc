@@ -333,6 +333,59 @@ extern "C" int orc_bpt_check(void* tp) {
   return cnt == t->size ? 0 : 6;
 }
 
+// Test hook for the checker's own pin: corrupt the tree in one targeted way so that a test
+// can assert orc_bpt_check reports the rule it breaks.  Returns 1 if the mutation applied
+// (the tree must have height >= 2 and a leaf with >= 2 records for kinds 1-5).
+//  1 swap two keys of a leaf (order)        2 underfill a leaf (occupancy)
+//  3 move a leaf key outside its separator bounds (bounds)
+//  4 break the leaf sibling chain (chain)   5 size counter off by one (size)
+//  6 drop a child of an internal node (occupancy: children != keys + 1)
+extern "C" int orc_bpt_debug_mutate(void* tp, int kind) {
+  Tree* t = (Tree*)tp;
+  Node* n = t->root;
+  if (n->leaf) return 0;
+  Node* parent = n;
+  while (!n->leaf) {
+    parent = n;
+    n = n->child[n->child.size() / 2];
+  }
+  Node* leaf = n;  // a middle leaf: it has a predecessor and separator bounds on both sides
+  if (leaf->keys.size() < 2) return 0;
+  switch (kind) {
+    case 1:
+      std::swap(leaf->keys[0], leaf->keys[1]);
+      return 1;
+    case 2:  // underfill below ceil((F-1)/2) records (keeps order and bounds)
+      if (t->min_records() < 2) return 0;
+      leaf->keys.resize(1);
+      leaf->vals.resize(1);
+      return 1;
+    case 3:
+      leaf->keys[0] = 0;  // below the separator that routes to this middle leaf
+      return leaf->keys[1] > 0 ? 1 : 0;
+    case 4: {  // relink leaves 0 -> 2 -> 1 -> 3: every record still reachable, order broken
+      Node* l0 = t->root;
+      while (!l0->leaf) l0 = l0->child[0];
+      Node* l1 = l0->next;
+      Node* l2 = l1 ? l1->next : nullptr;
+      if (!l2) return 0;
+      Node* l3 = l2->next;
+      l0->next = l2;
+      l2->next = l1;
+      l1->next = l3;
+      return 1;
+    }
+    case 5:
+      t->size += 1;
+      return 1;
+    case 6:
+      if (parent->child.size() < 2) return 0;
+      parent->child.pop_back();
+      return 1;
+  }
+  return 0;
+}
+
 extern "C" void orc_bpt_dump(void* tp, uint64_t* keys, uint64_t* vals) {
   const Node* n = ((Tree*)tp)->root;
   while (!n->leaf) n = n->child[0];

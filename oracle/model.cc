@@ -80,9 +80,12 @@ extern "C" uint32_t orc_ntg_steps(uint32_t r, uint32_t cnt, uint32_t gs, uint32_
 // the profiled levels; averaged over the warps of the sample.
 extern "C" double orc_ntg_warp_steps(const uint64_t* kr, const uint32_t* ps, uint32_t F,
                                      uint32_t h, const uint64_t* ls, const uint64_t* q,
-                                     uint64_t nq, uint32_t gs, uint32_t kpl, uint32_t lev0) {
+                                     uint64_t nq, uint32_t gs, uint32_t kpl, uint32_t lev0,
+                                     uint32_t warp) {
   (void)ls;
-  const uint32_t qpw = std::max<uint32_t>(1, 32 / gs);  // warpsize / GS queries per warp
+  // "the number of queries processed by one warp equals to warpsize/GS"; Fig 9 uses
+  // a warp of 8 threads, the B200 a warp of 32.
+  const uint32_t qpw = std::max<uint32_t>(1, warp / gs);
   std::vector<uint64_t> path;
   double total = 0;
   uint64_t warps = 0;
@@ -111,11 +114,11 @@ extern "C" double orc_ntg_warp_steps(const uint64_t* kr, const uint32_t* ps, uin
 extern "C" uint32_t orc_ntg_choose_gs(const uint64_t* kr, const uint32_t* ps, uint32_t F,
                                       uint32_t h, const uint64_t* ls, const uint64_t* q,
                                       uint64_t nq, uint32_t gs0, uint32_t kpl,
-                                      uint32_t lev0) {
+                                      uint32_t lev0, uint32_t warp) {
   uint32_t gs = gs0;
-  double sb = orc_ntg_warp_steps(kr, ps, F, h, ls, q, nq, gs, kpl, lev0);
+  double sb = orc_ntg_warp_steps(kr, ps, F, h, ls, q, nq, gs, kpl, lev0, warp);
   while (gs / 2 >= 2) {
-    double sa = orc_ntg_warp_steps(kr, ps, F, h, ls, q, nq, gs / 2, kpl, lev0);
+    double sa = orc_ntg_warp_steps(kr, ps, F, h, ls, q, nq, gs / 2, kpl, lev0, warp);
     double ratio = sa > 0 ? 2.0 * sb / sa : 0.0;
     if (!(ratio > 1.0)) break;
     gs /= 2;

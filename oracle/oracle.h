@@ -64,6 +64,8 @@ uint64_t orc_bpt_size(void* t);
 uint32_t orc_bpt_height(void* t);
 /* 0 = ok; otherwise a positive code naming the violated rule (see bptree.cc). */
 int      orc_bpt_check(void* t);
+/* Test hook pinning the checker: apply one targeted corruption (kinds 1-6, bptree.cc). */
+int      orc_bpt_debug_mutate(void* t, int kind);
 /* In-order dump via the leaf chain. */
 void     orc_bpt_dump(void* t, uint64_t* keys, uint64_t* vals);
 /* Level statistics: nodes[l], entries[l] (keys in leaves, children in internals). */
@@ -126,14 +128,15 @@ uint64_t orc_psa_bucket(uint64_t q, uint32_t nbits, uint64_t min_key, uint64_t m
  * per step. */
 uint32_t orc_ntg_steps(uint32_t r, uint32_t cnt, uint32_t gs, uint32_t kpl);
 /* Eq 3/4: average over warps of the per-warp maximum step count summed
- * over the profiled levels [lev0, h), for thread-group size gs (warp = 32 lanes). */
+ * over the profiled levels [lev0, h), for thread-group size gs; a warp of `warp` threads
+ * serves warp/gs consecutive queries (Fig 9 uses warp = 8, the B200 32). */
 double   orc_ntg_warp_steps(const uint64_t* key_region, const uint32_t* ps, uint32_t fanout,
                             uint32_t height, const uint64_t* level_start, const uint64_t* q,
-                            uint64_t nq, uint32_t gs, uint32_t kpl, uint32_t lev0);
+                            uint64_t nq, uint32_t gs, uint32_t kpl, uint32_t lev0, uint32_t warp);
 /* Static-profile choice: start at gs0, halve while Eq 4 ratio 2*S_b/S_a > 1. */
 uint32_t orc_ntg_choose_gs(const uint64_t* key_region, const uint32_t* ps, uint32_t fanout,
                            uint32_t height, const uint64_t* level_start, const uint64_t* q,
-                           uint64_t nq, uint32_t gs0, uint32_t kpl, uint32_t lev0);
+                           uint64_t nq, uint32_t gs0, uint32_t kpl, uint32_t lev0, uint32_t warp);
 /* Fig 2: memory transactions per warp per level = distinct nodes touched
  * by the warp's queries at that level, averaged over levels and warps. */
 double   orc_warp_transactions(const uint64_t* key_region, const uint32_t* ps,

@@ -115,3 +115,15 @@ def test_fig3_comparisons_weak(orc):
     assert np.all(avg > 1.5) and np.all(avg < 6.5)
     assert c.shape[1] == 4  # height 4 as in the paper's setting
     assert np.all(c.max(axis=0)[1:] - c.min(axis=0)[1:] >= 3)  # below the (small) root
+
+
+@pytest.mark.parametrize("kind,code", [(1, 1), (2, 3), (3, 4), (4, 5), (5, 6), (6, 3)])
+def test_checker_rejects_mutations(orc, kind, code):
+    """orc_bpt_check is not vacuous: each targeted corruption reports the rule it breaks
+    (1 key order, 3 occupancy, 4 separator bounds, 5 leaf chain, 6 size)."""
+    keys = gen.uniform_keys(2000)
+    t = orc.BPlusTree(8)
+    t.insert_many(keys[np.random.default_rng(5).permutation(keys.shape[0])], keys)
+    assert t.check() == 0 and t.height >= 3
+    assert t.debug_mutate(kind)
+    assert t.check() == code

@@ -144,3 +144,31 @@ def test_checker_rejects_mutations(orc):
     assert mutated(bad_val) == 7
     assert mutated(pad_val) == 6
     assert mutated(drop_key) in (3, 6, 7)  # value slot no longer padded, or record lost
+
+
+def test_hand_derived_layout_fill05(orc):
+    """A fill-0.5 build (C-A6) written out by hand: level sizes, PS, separators, slots."""
+    g = golden_kv("layout_n10_f4_fill05.txt")
+    F = int(g["fanout"])
+    keys = np.arange(10, 101, 10, dtype=np.uint64)
+    vals = keys + np.uint64(1)
+    lay = orc.layout_build(keys, vals, F, 0.5)
+    conv = lambda s: [PAD if t == "P" else int(t) for t in s.split()]
+    assert lay.h == int(g["height"])
+    assert lay.level_start.tolist() == conv(g["level_start"])
+    assert lay.ps.tolist() == conv(g["ps"])
+    for n in range(lay.n_nodes):
+        assert lay.key_region[n * F:(n + 1) * F].tolist() == conv(g[f"node{n}"]), n
+    assert lay.leaf_vals.tolist() == conv(g["leafvals"])
+    assert lay.check(keys, vals)[0] == 0
+
+
+def test_shape_fill_below_one():
+    """C-A6 at fill 0.69 / 0.5 against hand arithmetic (2^23 F64 -> h = 5)."""
+    import oracle
+
+    for ln in golden_lines("shape_fill.txt"):
+        f = ln.split()
+        n, F, fill, levels = 1 << int(f[0]), int(f[1]), float(f[2]), [int(x) for x in f[3:]]
+        h, ln_ = oracle.layout_shape(n, F, fill)
+        assert h == len(levels) and ln_.tolist() == levels, (n, F, fill)

@@ -100,3 +100,25 @@ def test_eq4_narrowing(orc):
     g_rand = lay.ntg_choose_gs(q, 32, kpl=2)
     assert 2 <= g_rand <= 32 and 2 <= g_sorted <= 32
     assert g_sorted <= g_rand  # sorted batches tolerate narrower groups
+
+
+def test_fig9b_warp_level_steps(orc):
+    """Fig 9(b): the warp's step count is the max over its thread groups -- target 2
+    takes two steps when target 6 shares its warp.  Pins the per-warp max and warp/GS queries
+    per warp of orc_ntg_warp_steps (warp size 8 as in the figure)."""
+    keys = np.arange(7, dtype=np.uint64)  # one fanout-8 node with keys 0..6
+    lay = orc.layout_build(keys, keys, 8, 1.0)
+    assert lay.h == 1
+    for ln in golden_lines("fig9b_warp.txt"):
+        lhs, rhs = ln.split("->")
+        f = [int(x) for x in lhs.split()]
+        warp, gs, targets = f[0], f[1], np.array(f[2:], dtype=np.uint64)
+        assert lay.ntg_warp_steps(targets, gs, kpl=1, warp=warp) == float(rhs), ln
+    # the same two targets in separate warps cost 1 and 2 steps (no divergence)
+    assert lay.ntg_warp_steps(np.array([2, 6], dtype=np.uint64), 4, kpl=1, warp=4) == 1.5
+    # Eq 4 on the figure's node: narrowing 8 -> 4 halves the comparisons per query but the
+    # warp still needs 2 steps for [2, 6]: ratio 2 * S_b / S_a = 2 * 1 / 2 = 1, not > 1
+    assert lay.ntg_choose_gs(np.array([2, 6], dtype=np.uint64), 8, kpl=1, warp=8) == 8
+    # [2, 2]: GS 8 -> 4 keeps 1 step per warp (ratio 2); GS 4 -> 2 needs 2 steps for
+    # target 2 (keys 0-1, then 2-3), ratio 2 * 1 / 2 = 1, so narrowing stops at 4
+    assert lay.ntg_choose_gs(np.array([2, 2], dtype=np.uint64), 8, kpl=1, warp=8) == 4
