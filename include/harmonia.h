@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define HARMONIA_ABI_VERSION 1
+#define HARMONIA_ABI_VERSION 2
 #define HARMONIA_NOT_FOUND UINT64_C(0xFFFFFFFFFFFFFFFF) /* result of an absent key (C-A4)     */
 #define HARMONIA_KEY_PAD   UINT64_C(0xFFFFFFFFFFFFFFFF) /* unused node slot; never a key (C-A2) */
 #define HARMONIA_MAX_LEVELS 64
@@ -64,8 +64,12 @@ typedef struct {
 
 /* Query options.  An all-zero struct (or a NULL pointer) selects every default. */
 typedef struct {
-  int32_t group_size;   /* NTG lanes per query G: 0 = auto (measured table for
-                           the tree's fanout); else a power of two in [2, 32] with 2G <= F.  */
+  int32_t group_size;   /* NTG lanes per query G: 0 = auto = 1 (the measured
+                           B200 choice for every fanout: the narrowing of
+                           Eq 4 continued to one lane per query); else a power of two in
+                           [1, 32] with 2G <= F.  G = 1 is a deviation from §8(b)'s 2..32:
+                           the paper's group narrowed to a single lane (lane-local binary
+                           rank instead of a ballot).                                        */
   int32_t psa_bits;     /* PSA sort bits Nb (Eq 2): 0 = auto = ceil(log2(T/K)), K=16;
                            < 0 = PSA off (queries searched in arrival order); else 1..28.   */
   int32_t smem_levels;  /* top tree levels staged in shared memory: 0 = auto plan (fits the
@@ -109,6 +113,11 @@ typedef struct {
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic
                                       per query) instead of the default two-level partition  */
+#define HARMONIA_QF_PSA_L16 8192u /* staged-return PSA: force two MSD levels (8 + 8 bits) and
+                                      bucket-aligned chunks, i.e. the whole window in Eq-2
+                                      order (default: chosen by the plan, see harmonia_plan) */
+#define HARMONIA_QF_PSA_L8 16384u /* staged-return PSA: force one MSD level (8 bits) + chunk
+                                      sort (the window is Eq-2 ordered inside each chunk)    */
 #define HARMONIA_QF_LINEAR     4u  /* in-node search = the paper's linear NTG walk (Fig 9:
                                       2G keys per step, early exit) instead of the default
                                       k-ary NTG (same G lanes, fixed log-depth steps)         */
@@ -153,11 +162,11 @@ harmonia_status harmonia_export_layout(const harmonia_tree* tree, uint64_t* h_ke
 /* ---------------------------------------------------------------------------------------
  * harmonia_search_batch — n point queries (§3.2.1; PSA §4.1; NTG §4.2).
  *   d_queries[n] -> d_values_out[n]: the value of each query's key, or HARMONIA_NOT_FOUND.
- *   Pipeline per PSA window (default: the whole batch up to 2^27 queries): PSA (Eq 2) as a
- *   two-level partition on the top Nb key bits -- 8-bit coarse rank + move passes, then a
- *   4096-query chunk counting sort on all Nb bits -- the descent with Eq 1 (child =
- *   PS[node] + i - 1) and leaf probe, then the results go back to the caller's order through
- *   a chunk-local shared-memory permutation and the inverse of the coarse move.  d_queries
+ *   Pipeline per PSA window (default: the whole batch up to 2^27 queries): PSA (Eq 2) on the
+ *   top Nb key bits -- one or two 8-bit MSD rank + move rounds (harmonia_plan.psa_levels),
+ *   then a counting sort of 4096/8192-query chunks on all Nb bits -- the descent with Eq 1
+ *   (child = PS[node] + i - 1) and leaf probe, then the results go back to the caller's
+ *   order through a chunk-local shared-memory permutation and the inverse moves.  d_queries
  *   and d_values_out may not overlap.  d_workspace must hold
  *   harmonia_search_workspace_bytes(tree, n, opts) bytes (about 36 bytes per window query),
  *   16-byte aligned.   Errors: INVALID_ARG, DEVICE_MISMATCH, CUDA.
@@ -205,9 +214,13 @@ harmonia_status harmonia_range_batch(const harmonia_tree* tree, const uint64_t* 
  *   1 = delete: remove if present), d_keys[n], d_values[n] (ignored for deletes).
  *   Sequential semantics in batch order: the last op on a key wins.  Keys equal to
  *   HARMONIA_KEY_PAD or upsert values equal to HARMONIA_NOT_FOUND are rejected
- *   (HARMONIA_ERR_RESERVED, tree unchanged).  The layout is rebuilt from the first affected
- *   leaf: merged leaf sequence, re-packed leaves, internal levels and PS recomputed
- *   (the paper's post-batch "movement", done as bulk-synchronous device passes).
+ *   (HARMONIA_ERR_RESERVED, tree unchanged).  The whole layout is rebuilt from the merged
+ *   record sequence: re-packed leaves, internal levels and PS recomputed (the paper's
+ *   post-batch "movement", as bulk-synchronous device passes; a rebuild from the
+ *   first affected leaf costs the same passes on the GPU, and the full rebuild keeps the
+ *   layout bit-identical to a fresh harmonia_build, invariant I8).  The batch sort and scans
+ *   use CUB (a library primitive, like cuBLAS for a GEMM; not on the query path).  A tree of
+ *   2^31 - 1 or more records after the batch is HARMONIA_ERR_TOO_LARGE (32-bit scan counts).
  *   May reallocate the tree's arrays; synchronises `stream`.
  *   d_workspace must hold harmonia_update_workspace_bytes(tree, n).
  * ------------------------------------------------------------------------------------- */
@@ -226,6 +239,12 @@ harmonia_status harmonia_update_batch(harmonia_tree* tree, const uint8_t* d_ops,
 harmonia_status harmonia_update_batch_seq(harmonia_tree* tree, const uint8_t* d_ops, const uint64_t* d_keys,
                                           const uint64_t* d_values, const uint64_t* d_seq, uint64_t n,
                                           void* d_workspace, size_t workspace_bytes, void* stream);
+/* harmonia_update_validate: *d_flags (uint32, device) = OR over the batch of 2 (a key equal to
+ * HARMONIA_KEY_PAD or an upsert value equal to HARMONIA_NOT_FOUND: the batch would be
+ * HARMONIA_ERR_RESERVED) and 4 (an op code other than 0/1).  Asynchronous.  The partitioned
+ * mode validates every rank's batch before routing so that all shards accept or all reject. */
+harmonia_status harmonia_update_validate(const uint8_t* d_ops, const uint64_t* d_keys, const uint64_t* d_values,
+                                         uint64_t n, uint32_t* d_flags, void* stream);
 harmonia_status harmonia_route_update_payload(const uint8_t* d_ops, const uint64_t* d_values,
                                               const uint32_t* d_pos, uint64_t n, uint32_t rank,
                                               uint8_t* d_ops_out, uint64_t* d_values_out,
@@ -332,9 +351,30 @@ typedef struct {
   uint32_t warp_shared;    /* 1: G = 1 warp-shared descent (see HARMONIA_QF_PER_LANE) */
   uint32_t sort_chunk;     /* staged return: level-2 chunk (queries); 0 when not staged */
   uint64_t l2_window_bytes; /* bytes of the internal key region pinned in L2 (0 = none) */
+  uint32_t psa_levels;     /* global MSD partition levels before the chunk sort: 1 = 8 bits
+                              (Eq-2 order inside each sort_chunk piece), 2 = 8 + 8 bits with
+                              chunks of whole 16-bit buckets (the whole window in Eq-2 order);
+                              0 = PSA off.  Auto: 2 when a level-1 chunk would hold fewer
+                              than 4 queries per leaf (large trees), else 1.                */
+  uint32_t chunk_group;    /* psa_levels 2: 16-bit buckets per chunk group (0 otherwise)     */
 } harmonia_plan;
 harmonia_status harmonia_query_plan(const harmonia_tree* tree, uint64_t n,
                                     const harmonia_query_opts* opts, harmonia_plan* out);
+
+/* ---------------------------------------------------------------------------------------
+ * harmonia_psa_inspect — run only the PSA stages (Eq 2) that
+ *   harmonia_search_batch would run for (n, opts) and write the queries to d_order_out[n] in
+ *   the order the search kernel visits them (window by window, chunk by chunk, no padding).
+ *   With the plan's psa_levels = 2 every window is non-decreasing in its Nb-bit bucket
+ *   (C-A11) except inside a chunk group larger than sort_chunk queries (skewed batches); with
+ *   psa_levels = 1 the top min(8, Nb) bucket bits are non-decreasing over each window and all
+ *   Nb bits inside each sort_chunk piece.  d_order_out is a permutation of d_queries.
+ *   Workspace as for harmonia_search_batch.  Asynchronous.  For tests and reports; it is not
+ *   part of the query path.  Errors: INVALID_ARG, DEVICE_MISMATCH, CUDA.
+ * ------------------------------------------------------------------------------------- */
+harmonia_status harmonia_psa_inspect(const harmonia_tree* tree, const uint64_t* d_queries, uint64_t n,
+                                     const harmonia_query_opts* opts, void* d_workspace,
+                                     size_t workspace_bytes, uint64_t* d_order_out, void* stream);
 
 /* ---------------------------------------------------------------------------------------
  * NTG static profiling (§4.2): the paper's model for the thread-group size.

@@ -82,6 +82,7 @@ def lib():
             "orc_eq1_child": (C.c_uint64, [u32p, C.c_uint64, C.c_uint64]),
             "orc_psa_bits": (C.c_uint32, [C.c_uint32, C.c_double, C.c_uint32]),
             "orc_psa_bucket": (C.c_uint64, [C.c_uint64, C.c_uint32, C.c_uint64, C.c_uint64]),
+            "orc_psa_buckets": (None, [u64p, C.c_uint64, C.c_uint32, C.c_uint64, C.c_uint64, u64p]),
             "orc_psa_order": (None, [u64p, C.c_uint64, C.c_uint32, C.c_uint64, C.c_uint64, u64p]),
             "orc_ntg_steps": (C.c_uint32, [C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32]),
             "orc_ntg_warp_steps": (C.c_double, [u64p, u32p, C.c_uint32, C.c_uint32, u64p, u64p, C.c_uint64,
@@ -323,6 +324,14 @@ def psa_bits(B: int, T: float, K: int) -> int:
 
 def psa_bucket(q: int, nbits: int, min_key: int, max_key: int) -> int:
     return int(lib().orc_psa_bucket(int(q), nbits, int(min_key), int(max_key)))
+
+
+def psa_buckets(q, nbits: int, min_key: int, max_key: int) -> np.ndarray:
+    """orc_psa_bucket of every query (C-A11)."""
+    q = _u64(q)
+    out = np.empty(q.shape[0], dtype=np.uint64)
+    lib().orc_psa_buckets(_p64(q), q.shape[0], nbits, min_key, max_key, _p64(out))
+    return out
 
 
 def psa_order(q, nbits: int, min_key: int, max_key: int) -> np.ndarray:

@@ -55,6 +55,12 @@ extern "C" uint64_t orc_psa_bucket(uint64_t q, uint32_t nbits, uint64_t min_key,
   return (c >> shift) & mask;
 }
 
+// orc_psa_bucket over an array (test convenience: one call instead of one per query)
+extern "C" void orc_psa_buckets(const uint64_t* q, uint64_t nq, uint32_t nbits, uint64_t min_key,
+                                uint64_t max_key, uint64_t* out) {
+  for (uint64_t i = 0; i < nq; ++i) out[i] = orc_psa_bucket(q[i], nbits, min_key, max_key);
+}
+
 // "the queries will be sorted based on their most significant N bits" (stable).
 extern "C" void orc_psa_order(const uint64_t* q, uint64_t nq, uint32_t nbits,
                               uint64_t min_key, uint64_t max_key, uint64_t* perm) {

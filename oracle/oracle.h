@@ -123,6 +123,8 @@ uint32_t orc_psa_bits(uint32_t B, double T, uint32_t K);
 void     orc_psa_order(const uint64_t* q, uint64_t nq, uint32_t nbits,
                        uint64_t min_key, uint64_t max_key, uint64_t* perm);
 uint64_t orc_psa_bucket(uint64_t q, uint32_t nbits, uint64_t min_key, uint64_t max_key);
+void     orc_psa_buckets(const uint64_t* q, uint64_t nq, uint32_t nbits, uint64_t min_key,
+                         uint64_t max_key, uint64_t* out);
 /* Fig 9, C-A13: comparison steps of one query whose target sits after r
  * keys (r = #keys <= q) in a node of cnt keys, with GS threads and kpl keys per thread
  * per step. */

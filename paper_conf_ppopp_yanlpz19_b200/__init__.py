@@ -32,6 +32,8 @@ QF_PSA_WIDE = 512
 QF_NO_L2_WINDOW = 4096
 QF_PER_LANE = 1024
 QF_RANGE_GROUP = 2048
+QF_PSA_L16 = 8192
+QF_PSA_L8 = 16384
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
            6: "DEVICE_MISMATCH", 7: "TOO_LARGE"}
 
@@ -61,7 +63,7 @@ class PlanInfo(C.Structure):
                 ("ps_in_smem", C.c_int32), ("window", C.c_uint64), ("smem_bytes", C.c_uint32),
                 ("smem_nodes", C.c_uint32), ("staged_return", C.c_uint32), ("lane_queries", C.c_uint32),
                 ("warp_shared", C.c_uint32), ("sort_chunk", C.c_uint32),
-                ("l2_window_bytes", C.c_uint64)]
+                ("l2_window_bytes", C.c_uint64), ("psa_levels", C.c_uint32), ("chunk_group", C.c_uint32)]
 
 
 class Info(C.Structure):
@@ -102,6 +104,7 @@ def lib():
             "harmonia_update_workspace_bytes": (_sz, [_vp, _u64]),
             "harmonia_update_batch": (C.c_int, [_vp, _vp, _vp, _vp, _u64, _vp, _sz, _vp]),
             "harmonia_update_batch_seq": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _u64, _vp, _sz, _vp]),
+            "harmonia_update_validate": (C.c_int, [_vp, _vp, _vp, _u64, _vp, _vp]),
             "harmonia_route_update_payload": (C.c_int, [_vp, _vp, _vp, _u64, C.c_uint32, _vp, _vp, _vp, _vp]),
             "harmonia_route_workspace_bytes": (_sz, [C.c_uint32, _u64]),
             "harmonia_route_partition": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _vp, _vp, _sz, _vp]),
@@ -127,6 +130,7 @@ def lib():
             "harmonia_tune_group_size": (C.c_int, [_vp, _vp, C.c_uint32, C.POINTER(QueryOpts),
                                                    C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
             "harmonia_query_plan": (C.c_int, [_vp, _u64, C.POINTER(QueryOpts), C.POINTER(PlanInfo)]),
+            "harmonia_psa_inspect": (C.c_int, [_vp, _vp, _u64, C.POINTER(QueryOpts), _vp, _sz, _vp, _vp]),
             "harmonia_profile_enable": (None, [C.c_int]),
             "harmonia_profile_read": (C.c_int, [C.POINTER(C.c_double), C.POINTER(_u64)]),
             "harmonia_status_string": (C.c_char_p, [C.c_int]),
@@ -292,14 +296,20 @@ class Tree:
                "harmonia_export_layout")
         return i, kr, ps, lv
 
-    def _workspace(self, nbytes: int):
+    def _workspace(self, nbytes: int, stream=None):
+        """Workspace for calls on `stream` (the C ABI needs one per stream).  Cached per stream
+        and allocated while that stream is current, so the caching allocator never hands the
+        block to another stream while a kernel may still use it."""
         torch = _torch()
         if nbytes == 0:
             return None
-        w = self._ws.get("buf")
+        s = stream if stream is not None else torch.cuda.current_stream(self.device)
+        key = int(s.cuda_stream)
+        w = self._ws.get(key)
         if w is None or w.numel() < nbytes:
-            w = torch.empty(nbytes, dtype=torch.uint8, device=self.device)
-            self._ws["buf"] = w
+            with torch.cuda.stream(s):
+                w = torch.empty(nbytes, dtype=torch.uint8, device=self.device)
+            self._ws[key] = w
         return w
 
     # ------------------------------------------------------------------ queries
@@ -312,7 +322,7 @@ class Tree:
             out = torch.empty(n, dtype=torch.uint64, device=self.device)
         o = opts if opts is not None else make_opts(**kw)
         ws_b = lib().harmonia_search_workspace_bytes(self._h, n, C.byref(o))
-        ws = self._workspace(ws_b)
+        ws = self._workspace(ws_b, stream)
         st = _stream_ptr(stream, self.device)
         _check(lib().harmonia_search_batch(self._h, q.data_ptr(), n, out.data_ptr(),
                                            ws.data_ptr() if ws is not None else None, ws_b, C.byref(o), st),
@@ -323,10 +333,24 @@ class Tree:
         """Point queries read from a raw device address (e.g. a peer-mapped receive buffer)."""
         o = opts if opts is not None else make_opts(**kw)
         ws_b = lib().harmonia_search_workspace_bytes(self._h, n, C.byref(o))
-        ws = self._workspace(ws_b)
+        ws = self._workspace(ws_b, stream)
         _check(lib().harmonia_search_batch(self._h, q_addr, n, out.data_ptr(),
                                            ws.data_ptr() if ws is not None else None, ws_b, C.byref(o),
                                            _stream_ptr(stream, self.device)), "harmonia_search_batch")
+        return out
+
+    def psa_inspect(self, q, *, opts: QueryOpts | None = None, stream=None, **kw):
+        """The queries in the order the search kernel visits them after PSA (harmonia_psa_inspect)."""
+        torch = _torch()
+        q = _as_u64_dev(q, self.device)
+        n = q.numel()
+        out = torch.empty(n, dtype=torch.uint64, device=self.device)
+        o = opts if opts is not None else make_opts(**kw)
+        ws_b = lib().harmonia_search_workspace_bytes(self._h, n, C.byref(o))
+        ws = self._workspace(ws_b, stream)
+        _check(lib().harmonia_psa_inspect(self._h, q.data_ptr(), n, C.byref(o),
+                                          ws.data_ptr() if ws is not None else None, ws_b, out.data_ptr(),
+                                          _stream_ptr(stream, self.device)), "harmonia_psa_inspect")
         return out
 
     def search_host(self, q_host, out_host=None, *, opts: QueryOpts | None = None, stream=None, **kw):
@@ -340,7 +364,7 @@ class Tree:
             out_host = torch.empty(n, dtype=torch.uint64, pin_memory=True)
         o = opts if opts is not None else make_opts(**kw)
         ws_b = lib().harmonia_search_host_workspace_bytes(self._h, n, C.byref(o))
-        ws = self._workspace(ws_b)
+        ws = self._workspace(ws_b, stream)
         st = _stream_ptr(stream, self.device)
         _check(lib().harmonia_search_batch_host(self._h, q_host.data_ptr(), n, out_host.data_ptr(),
                                                 ws.data_ptr(), ws_b, C.byref(o), st), "harmonia_search_batch_host")
@@ -362,7 +386,7 @@ class Tree:
             cnt = torch.empty(n, dtype=torch.uint32, device=self.device)
         o = opts if opts is not None else make_opts(**kw)
         ws_b = lib().harmonia_range_workspace_bytes(self._h, n, C.byref(o))
-        ws = self._workspace(ws_b)
+        ws = self._workspace(ws_b, stream)
         st = _stream_ptr(stream, self.device)
         _check(lib().harmonia_range_batch(self._h, lo.data_ptr(), hi.data_ptr(), n, cap,
                                           ko.data_ptr() if ko is not None else None,
@@ -391,6 +415,17 @@ class Tree:
             _check(lib().harmonia_update_batch_seq(self._h, ops.data_ptr(), keys.data_ptr(), values.data_ptr(),
                                                    seq.data_ptr(), n, ws.data_ptr(), ws_b, st),
                    "harmonia_update_batch_seq")
+
+
+def update_validate(ops, keys, values, stream=None):
+    """harmonia_update_validate: a device uint32[1] holding 0 for a valid update batch, else
+    2 (reserved key/value) | 4 (bad op code)."""
+    torch = _torch()
+    dev = keys.device
+    flags = torch.empty(1, dtype=torch.int32, device=dev)
+    _check(lib().harmonia_update_validate(ops.data_ptr(), keys.data_ptr(), values.data_ptr(), keys.numel(),
+                                          flags.data_ptr(), _stream_ptr(stream, dev)), "harmonia_update_validate")
+    return flags
 
 
 def route_partition(splitters, P: int, q, stream=None):

@@ -3,7 +3,9 @@
 // in the kernels of psa.cu / search.cu; this file only sequences launches on the caller's
 // stream.
 #include <algorithm>
+#include <cmath>
 #include <cstring>
+#include <mutex>
 
 #include "common.cuh"
 
@@ -18,6 +20,10 @@ namespace {
 #endif
 constexpr uint32_t kSmemBudget = 48 * 1024;  // auto plan: keeps >= 4 CTAs (32 warps) per SM
 constexpr uint64_t kAutoWindow = 1ull << 27;  // auto PSA window (queries): measured best, DESIGN.md §8
+#ifndef HM_L16_DENSITY
+#define HM_L16_DENSITY 0.5
+#endif
+constexpr double kL16MaxChunkDensity = HM_L16_DENSITY;  // two PSA levels below this density
 
 bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 }  // namespace
@@ -122,6 +128,23 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
       P.l2_hit = (float)std::min(1.0, (double)t->l2_persist_max / (double)bytes);
     }
   }
+  // two MSD levels (8 + 8 bits) before a bucket-aligned chunk sort puts the whole window in
+  // Eq-2 order.  It costs a second rank/move/unmove round (~0.9 ms per 2^26
+  // queries), which the search repays only when a level-1 chunk is very sparse in the tree:
+  // 4096 x 256 / leaves queries per leaf (c2 63, 2^26 keys 0.98 -> one level; 2^28 keys 0.25
+  // -> two levels: search 4.5 -> 2.1 ms, step 6.65 -> 6.19 ms).
+  P.psa_levels = 1;
+  if (P.ret && P.nb >= 16 && !(o->flags & HARMONIA_QF_PSA_WIDE) && !(o->flags & HARMONIA_QF_PSA_L8)) {
+    const double dens = t->L ? (double)kPsaChunk * 256.0 / (double)t->L : 1e9;
+    if ((o->flags & HARMONIA_QF_PSA_L16) || dens < kL16MaxChunkDensity) P.psa_levels = 2;
+  }
+  if (P.psa_levels == 2) {
+    if (o->sort_chunk == 0) P.chunk = kPsaChunkMax;  // measured: 8192 beats 4096 at every size
+    // buckets per chunk group: the group (mean + 4 sigma + padding) fits one chunk
+    const double mean = (double)std::min<uint64_t>(n, P.window) / (double)kL2Buckets;
+    const double fit = (double)P.chunk / (mean + 4.0 * std::sqrt(mean) + 8.0);
+    P.l2_group = (uint32_t)std::max(1.0, std::min(fit, (double)kL2Buckets));
+  }
   P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
   P.coop = P.ret && !(o->flags & HARMONIA_QF_PER_LANE);
   // ranges: the warp-per-range copy kernel unless a group size was requested explicitly or
@@ -150,22 +173,61 @@ static SearchArgs search_args(const harmonia_tree* t, const Plan& p) {
 }
 
 // The device's persisting-L2 set-aside must cover the window (cudaLimitPersistingL2CacheSize
-// is device-wide; raised once, never lowered by the library).  false: no window this call.
+// is device-wide).  The first tree that raises it records the device's previous limit; the
+// last such tree to be destroyed restores it (l2_persist_release), and a layout swap or a
+// destroy drops the persisting lines (cudaCtxResetPersistingL2Cache) so stale key regions do
+// not stay pinned.  false: no window this call.
+namespace {
+std::mutex g_l2_mu;
+struct L2Dev {
+  int users = 0;
+  size_t saved = 0;
+};
+L2Dev g_l2[64];
+}  // namespace
+
 static bool ensure_l2_persist(const harmonia_tree* tc, size_t bytes) {
   harmonia_tree* t = const_cast<harmonia_tree*>(tc);
   const size_t want = std::min(bytes, t->l2_persist_max);
   if (t->l2_persist_set >= want) return true;
+  std::lock_guard<std::mutex> lk(g_l2_mu);
   size_t cur = 0;
-  if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess && cur >= want) {
-    t->l2_persist_set = cur;
-    return true;
-  }
-  if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) != cudaSuccess) {
+  if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) != cudaSuccess) {
     cudaGetLastError();
     return false;
   }
-  t->l2_persist_set = want;
+  L2Dev& d = g_l2[t->device & 63];
+  const bool first_use = t->l2_persist_set == 0;
+  if (cur < want) {
+    if (d.users == 0) d.saved = cur;
+    if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    cur = want;
+  } else if (d.users == 0 && first_use) {
+    d.saved = cur;
+  }
+  if (first_use) ++d.users;
+  t->l2_persist_set = cur;
   return true;
+}
+
+void l2_persist_reset(const harmonia_tree* t) {
+  if (t->l2_persist_set) {
+    cudaCtxResetPersistingL2Cache();
+    cudaGetLastError();
+  }
+}
+
+void l2_persist_release(harmonia_tree* t) {
+  if (!t->l2_persist_set) return;
+  std::lock_guard<std::mutex> lk(g_l2_mu);
+  cudaCtxResetPersistingL2Cache();
+  L2Dev& d = g_l2[t->device & 63];
+  if (d.users > 0 && --d.users == 0) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, d.saved);
+  cudaGetLastError();
+  t->l2_persist_set = 0;
 }
 
 static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, uint64_t n, uint64_t* out,
@@ -203,6 +265,24 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       a.out = out + w0;
       a.bucket = p.bucket;
       if ((s = launch_sort_search(t, p, a, st)) != HARMONIA_OK) return s;
+      continue;
+    }
+    if (p.ret && p.psa_levels == 2) {  // two MSD levels + bucket-aligned chunks
+      if ((s = psa_partition2_l2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.l2_group, p.chunk)) != HARMONIA_OK)
+        return s;
+      a.q = w.sorted2;
+      a.idx = w.idx;
+      a.out = w.res2;
+      a.staged = 1;
+      a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
+      a.chunk = p.chunk;
+      a.ctab = w.chunks;
+      a.nctab = w.nchunks;
+      a.bucket = p.bucket;
+      if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+      if ((s = psa_unpartition2_l2(w, w.res2, nw, out + w0, t->sm_count, st)) != HARMONIA_OK) return s;
+      a.ctab = nullptr;
+      a.nctab = nullptr;
       continue;
     }
     if (p.ret) {  // staged return: level-1-order results, then the inverse move
@@ -258,6 +338,8 @@ extern "C" harmonia_status harmonia_search_batch(const harmonia_tree* t, const u
   if (!t) return HARMONIA_ERR_INVALID_ARG;
   if (n == 0) return HARMONIA_OK;
   if (!d_q || !d_out) return HARMONIA_ERR_INVALID_ARG;
+  DevGuard g(t->device, (cudaStream_t)stream);
+  if (g.status != HARMONIA_OK) return g.status;
   if (!on_device(d_q, t->device) || !on_device(d_out, t->device)) return HARMONIA_ERR_DEVICE_MISMATCH;
   Plan p;
   harmonia_status s = make_plan(t, n, o, &p);
@@ -293,6 +375,51 @@ extern "C" harmonia_status harmonia_query_plan(const harmonia_tree* t, uint64_t 
   out->warp_shared = p.coop ? 1u : 0u;
   out->sort_chunk = p.ret ? p.chunk : 0u;
   out->l2_window_bytes = p.l2_bytes;
+  out->psa_levels = p.psa ? (p.ret ? (uint32_t)p.psa_levels : 1u) : 0u;
+  out->chunk_group = p.psa_levels == 2 ? p.l2_group : 0u;
+  return HARMONIA_OK;
+}
+
+// ---- PSA order inspection (tests of the Eq-2 order) --------------------------------------
+extern "C" harmonia_status harmonia_psa_inspect(const harmonia_tree* t, const uint64_t* d_q, uint64_t n,
+                                                const harmonia_query_opts* o, void* ws, size_t ws_bytes,
+                                                uint64_t* d_order_out, void* stream) {
+  if (!t) return HARMONIA_ERR_INVALID_ARG;
+  if (n == 0) return HARMONIA_OK;
+  if (!d_q || !d_order_out) return HARMONIA_ERR_INVALID_ARG;
+  DevGuard g(t->device, (cudaStream_t)stream);
+  if (g.status != HARMONIA_OK) return g.status;
+  if (!on_device(d_q, t->device) || !on_device(d_order_out, t->device)) return HARMONIA_ERR_DEVICE_MISMATCH;
+  Plan p;
+  harmonia_status s = make_plan(t, n, o, &p);
+  if (s != HARMONIA_OK) return s;
+  cudaStream_t st = (cudaStream_t)stream;
+  if (!p.psa || t->n_keys == 0) {  // no partition: the search visits the caller's order
+    HM_CUDA(cudaMemcpyAsync(d_order_out, d_q, n * 8, cudaMemcpyDeviceToDevice, st));
+    return HARMONIA_OK;
+  }
+  const size_t need = psa_ws_bytes(p);
+  if (!ws || ws_bytes < need) return HARMONIA_ERR_INVALID_ARG;
+  if (((uintptr_t)ws & 255) != 0) {
+    const size_t adj = 256 - ((uintptr_t)ws & 255);
+    if (ws_bytes < need + adj) return HARMONIA_ERR_INVALID_ARG;
+    ws = (char*)ws + adj;
+  }
+  const PsaWs w = psa_ws_carve(p, ws);
+  for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
+    const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
+    if (p.ret && p.psa_levels == 2) {
+      if ((s = psa_partition2_l2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.l2_group, p.chunk)) != HARMONIA_OK)
+        return s;
+      if ((s = psa_compact_l2(w, d_order_out + w0, t->sm_count, st)) != HARMONIA_OK) return s;
+      continue;
+    }
+    if (p.psa_global) s = psa_partition(d_q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr);
+    else if (p.ret) s = psa_partition2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, 0, true, p.wide, p.chunk);
+    else s = psa_partition2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.fuse ? 2 : p.psa_level2);
+    if (s != HARMONIA_OK) return s;
+    HM_CUDA(cudaMemcpyAsync(d_order_out + w0, w.sorted_q, nw * 8, cudaMemcpyDeviceToDevice, st));
+  }
   return HARMONIA_OK;
 }
 
@@ -320,6 +447,8 @@ extern "C" harmonia_status harmonia_search_batch_host(const harmonia_tree* tc, c
   if (!t) return HARMONIA_ERR_INVALID_ARG;
   if (n == 0) return HARMONIA_OK;
   if (!h_q || !h_out || !ws) return HARMONIA_ERR_INVALID_ARG;
+  DevGuard g(t->device, (cudaStream_t)stream);
+  if (g.status != HARMONIA_OK) return g.status;
   Plan p;
   harmonia_status s = make_plan(t, std::min<uint64_t>(n, 1ull << 22), o, &p);
   if (s != HARMONIA_OK) return s;
@@ -380,6 +509,8 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   if (!t) return HARMONIA_ERR_INVALID_ARG;
   if (n == 0) return HARMONIA_OK;
   if (!d_lo || !d_hi || !d_counts || (cap > 0 && (!d_kout || !d_vout))) return HARMONIA_ERR_INVALID_ARG;
+  DevGuard g(t->device, (cudaStream_t)stream);
+  if (g.status != HARMONIA_OK) return g.status;
   if (!on_device(d_lo, t->device) || !on_device(d_counts, t->device)) return HARMONIA_ERR_DEVICE_MISMATCH;
   cudaStream_t st = (cudaStream_t)stream;
   Plan p;

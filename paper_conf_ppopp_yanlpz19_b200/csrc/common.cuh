@@ -41,6 +41,14 @@ void count_launch(uint64_t k = 1);
     if (e_ != cudaSuccess) return hm::cuda_fail(e_); \
   } while (0)
 
+// raise a kernel's dynamic shared-memory limit to >= bytes on the current device (once per
+// kernel and device; thread-safe)
+cudaError_t smem_attr(const void* kern, size_t bytes);
+template <class... A>
+inline cudaError_t smem_attr(void (*kern)(A...), size_t bytes) {
+  return smem_attr(reinterpret_cast<const void*>(kern), bytes);
+}
+
 __host__ __device__ inline uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 // whole warps iterate a grid-stride loop uniformly when its bound is a multiple of 32
 __host__ __device__ inline uint64_t round_up_dev(uint64_t n) { return (n + 31) & ~31ull; }
@@ -204,6 +212,10 @@ struct Plan {
   bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
   bool range_warp = true;    // ranges: one warp per range, resolve then stream-copy (k_range_warp)
   uint32_t chunk = 4096;     // staged return: level-2 chunk (4096 or kPsaChunkMax queries)
+  int psa_levels = 1;        // staged return: global MSD partition levels before the chunk sort:
+                             // 1 = 8 bits; 2 = 8 + 8 bits with bucket-aligned chunks (the whole
+                             // window in Eq-2 order)
+  uint32_t l2_group = 0;     // psa_levels 2: 16-bit buckets per chunk group
   const void* l2_base = nullptr;  // L2 access-policy window over the unstaged internal levels
   size_t l2_bytes = 0;
   float l2_hit = 0.f;
@@ -248,7 +260,20 @@ struct PsaWs {
   uint32_t* tile_counts;// ceil(window / 2048) x 256 per-tile coarse bin counts
   uint32_t* cta_counts; // kL1CtaRows: per level-1 CTA bin totals
   uint32_t* cta_base;   // kL1CtaRows: per level-1 CTA first global slot of each bin
+  // ---- second MSD level (Plan::psa_levels == 2), inside the level-1 segments
+  uint32_t* seg;        // [0..256] level-1 segment starts, [257..513] first level-2 tile per segment
+  uint32_t* packed2;    // window: level-2 digit | rank-in-tile << 8, at level-1 positions
+  uint32_t* tile_counts2;  // level-2 tiles x 256 digit counts
+  uint32_t* tile_base2;    // level-2 tiles x 256: level-2 position of each tile's digit run
+  uint32_t* comp_cnt;   // 65536 queries per 16-bit bucket
+  uint32_t* comp_start; // 65537 level-2 position of each 16-bit bucket (chunk groups padded to 8)
+  uint2* chunks;        // chunk table (start, queries): bucket-aligned chunks of <= Plan::chunk
+  uint32_t* chunk_pos;  // queries before each chunk (unpadded; harmonia_psa_inspect)
+  uint32_t* nchunks;    // [0] chunks, [1] padded level-2 length
+  uint64_t* sorted2;    // level-2 order (window + padding)
+  uint64_t* res2;       // results in level-2 order (window + padding)
 };
+constexpr uint32_t kL2Buckets = 65536;  // 16-bit composite buckets of the two MSD levels
 constexpr uint64_t kL1CtaRows = 2048 * 2048;  // >= (level-1 CTAs) x (bins) for every tiling
 constexpr uint32_t kPsaTile = 2048;   // level-1 tile (queries), 256-bin configuration
 // bytes of one per-(tile, bin) array: max over the level-1 tilings (256 bins / 2048-query
@@ -268,6 +293,21 @@ constexpr uint32_t kPsaChunkMax = 8192;  // staged-return chunk sizes: 4096 or 8
 #endif
 constexpr uint64_t kChunk8kMinQueriesPerLeaf = HM_CHUNK8K_QPL;  // auto 8192 chunks from this density
 constexpr uint32_t kScanTile = 4096;
+// second MSD level: level-2 tiles (segment-aligned 2048-query tiles), chunk-table entries and
+// the padded level-2 length (every chunk group is padded to a multiple of 8 queries, so chunk
+// starts stay 16-byte aligned for the TMA copies)
+struct L2Sizes {
+  uint64_t tiles, chunks, padded;
+};
+inline L2Sizes l2_sizes(uint64_t window, uint32_t chunk) {
+  return {(window + 2047) / 2048 + 256, window / chunk + kL2Buckets + 1, window + 8 * kL2Buckets};
+}
+inline uint64_t l2_ws_bytes(uint64_t window, uint32_t chunk) {
+  const L2Sizes z = l2_sizes(window, chunk);
+  auto r = [](uint64_t b) { return (b + 255) / 256 * 256; };
+  return r(2 * 257 * 4) + r(window * 4) + 2 * r(z.tiles * 256 * 4) + r(kL2Buckets * 4) + r((kL2Buckets + 1) * 4) +
+         r(z.chunks * 8) + r(z.chunks * 4) + 256 + 2 * r(z.padded * 8) + r(z.padded * 2);
+}
 size_t psa_ws_bytes(const Plan& p);
 PsaWs psa_ws_carve(const Plan& p, void* base);
 
@@ -296,6 +336,8 @@ struct SearchArgs {
                            // to out[] in level-1 order, chunk by chunk (kPsaChunk)
   uint32_t res_smem_off;
   uint32_t chunk;          // staged return: level-2 chunk (queries), 4096 or 8192
+  const uint2* ctab;       // chunk table (start, queries) instead of fixed chunks (psa_levels 2)
+  const uint32_t* nctab;   // device: chunks in ctab
   // warp-shared descent (G = 1 PSA path): clamp(q) -> (clamp(q) - kmin) >> cshift is a
   // monotone 32-bit image of the key, so two 32-bit warp reductions bound the warp's queries
   uint32_t coop;
@@ -310,6 +352,38 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
 // inverse of the level-1 move for the staged return: out[e] = res1[level-1 position of e]
 harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
                                  cudaStream_t st, bool wide);
+// two-level PSA (Plan::psa_levels == 2): partition into ws.sorted2 (chunk table ws.chunks),
+// and the inverse from level-2-order results; psa_compact_l2 = the chunks without padding
+harmonia_status psa_partition2_l2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
+                                  cudaStream_t st, uint32_t K, uint32_t cap);
+harmonia_status psa_unpartition2_l2(const PsaWs& ws, const uint64_t* res2, uint64_t n, uint64_t* out, int sm,
+                                    cudaStream_t st);
+harmonia_status psa_compact_l2(const PsaWs& ws, uint64_t* out, int sm, cudaStream_t st);
+
+// Entry points run on the tree's device: the current device is switched for the call and
+// restored; a stream of another device is HARMONIA_ERR_DEVICE_MISMATCH.
+struct DevGuard {
+  int prev = -1;
+  int dev = -1;
+  harmonia_status status = HARMONIA_OK;
+  DevGuard(int d, cudaStream_t s) : dev(d) {
+    if (cudaGetDevice(&prev) != cudaSuccess) {
+      status = cuda_fail(cudaGetLastError());
+      prev = -1;
+      return;
+    }
+    if (prev != dev && cudaSetDevice(dev) != cudaSuccess) {
+      status = cuda_fail(cudaGetLastError());
+      return;
+    }
+    int sd = dev;
+    if (s && cudaStreamGetDevice(s, &sd) == cudaSuccess && sd != dev) status = HARMONIA_ERR_DEVICE_MISMATCH;
+    cudaGetLastError();
+  }
+  ~DevGuard() {
+    if (prev >= 0 && prev != dev) cudaSetDevice(prev);
+  }
+};
 harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSplit& f, uint32_t P, const PsaWs& ws,
                                  int sm, cudaStream_t st, uint64_t* h_counts);
 // fused routing over peer memory (partitioned multi-GPU mode)
@@ -348,6 +422,11 @@ harmonia_status launch_gather(const uint64_t* sorted_out, const uint32_t* idx, u
                               uint64_t* out, int sm_count, cudaStream_t st);
 harmonia_status launch_scatter_back(const uint64_t* vals, const uint32_t* pos, uint64_t n,
                                     uint64_t* out, int sm_count, cudaStream_t st);
+
+// persisting-L2 bookkeeping of the access-policy window (capi.cu): drop the persisting lines
+// after a layout swap; on destroy also restore the device limit when the last tree goes
+void l2_persist_reset(const harmonia_tree* t);
+void l2_persist_release(harmonia_tree* t);
 
 // layout construction (tree.cu)
 harmonia_status build_layout(harmonia_tree* t, const uint64_t* d_keys, const uint64_t* d_vals,

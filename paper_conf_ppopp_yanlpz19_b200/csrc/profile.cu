@@ -1,6 +1,8 @@
 // harmonia_profile_*: CUDA-event timing of the library's kernels, per kernel class, on the
 // stream each kernel is launched on (used by bench.py for the roofline's kernel duration).
+#include <map>
 #include <mutex>
+#include <utility>
 #include <vector>
 
 #include "common.cuh"
@@ -8,6 +10,23 @@
 namespace hm {
 
 bool g_prof_on = false;
+
+// cudaFuncAttributeMaxDynamicSharedMemorySize is a per-device property of a kernel: remember
+// what was set per (kernel, device) so that a process driving trees on several devices sets
+// it on each (the per-process function-local caches skipped the second device).
+cudaError_t smem_attr(const void* kern, size_t bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, size_t> done;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(mu);
+  size_t& cur = done[{kern, dev}];
+  if (cur >= bytes) return cudaSuccess;
+  e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e == cudaSuccess) cur = bytes;
+  return e;
+}
 
 namespace {
 struct Rec {

@@ -168,6 +168,7 @@ size_t psa_ws_bytes(const Plan& p) {
   b += round_up(p.window * 4, 256);                        // packed digit/rank
   b += round_up(l1_rows_bytes(p.window), 256);        // per-tile counts
   b += 2 * kL1CtaRows * 4;                             // per-CTA counts and bases
+  if (p.psa_levels == 2) b += l2_ws_bytes(p.window, p.chunk);
   return b;
 }
 
@@ -191,6 +192,33 @@ PsaWs psa_ws_carve(const Plan& p, void* base) {
   w.cta_counts = (uint32_t*)c;
   c += kL1CtaRows * 4;
   w.cta_base = (uint32_t*)c;
+  c += kL1CtaRows * 4;
+  if (p.psa_levels == 2) {
+    const L2Sizes z = l2_sizes(p.window, p.chunk);
+    w.seg = (uint32_t*)c;
+    c += round_up(2 * 257 * 4, 256);
+    w.packed2 = (uint32_t*)c;
+    c += round_up(p.window * 4, 256);
+    w.tile_counts2 = (uint32_t*)c;
+    c += round_up(z.tiles * 256 * 4, 256);
+    w.tile_base2 = (uint32_t*)c;
+    c += round_up(z.tiles * 256 * 4, 256);
+    w.comp_cnt = (uint32_t*)c;
+    c += round_up(kL2Buckets * 4, 256);
+    w.comp_start = (uint32_t*)c;
+    c += round_up((kL2Buckets + 1) * 4, 256);
+    w.chunks = (uint2*)c;
+    c += round_up(z.chunks * 8, 256);
+    w.chunk_pos = (uint32_t*)c;
+    c += round_up(z.chunks * 4, 256);
+    w.nchunks = (uint32_t*)c;
+    c += 256;
+    w.sorted2 = (uint64_t*)c;
+    c += round_up(z.padded * 8, 256);
+    w.res2 = (uint64_t*)c;
+    c += round_up(z.padded * 8, 256);
+    w.idx = (uint32_t*)c;  // chunk-local offsets (uint16) at level-2 positions
+  }
   return w;
 }
 

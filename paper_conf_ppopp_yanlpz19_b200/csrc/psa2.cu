@@ -501,6 +501,272 @@ constexpr size_t unmove_smem() {
   return (size_t)C::TILE * 12 + 2 * C::BINS * 4 + (HM_L1_PREFETCH ? (size_t)C::TILE * 4 : 0);
 }
 
+// ---- second MSD level (Plan::psa_levels == 2) ----------------------------------------------
+// P:L418-L428 sorts the window by its top Nb bits.  Level 1 orders it by the top 8 bits; this
+// level orders every level-1 segment (one 8-bit bucket) by the next 8 bits with the same rank
+// + staged-move scheme on segment-aligned 2048-query tiles, so the level-2 order is sorted by
+// the top 16 bits.  The chunk sort then runs on chunks made of whole 16-bit buckets (groups of
+// Plan::l2_group consecutive buckets, each group padded to a multiple of 8 slots), which makes
+// the whole window sorted by all Nb bits.  Tile bases are computed by per-segment column scans
+// (deterministic; no global atomics).
+using L2C = L1Cfg<8, 2048, 256>;
+
+struct L2Digit {
+  BucketBits f;
+  uint32_t shift;  // nb - 16
+  __device__ __forceinline__ uint32_t operator()(uint64_t q) const { return (f(q) >> shift) & 255u; }
+};
+
+// segment starts from the level-1 bin counts, and the first level-2 tile of every segment
+__global__ void __launch_bounds__(256) k_l2_segs(const uint32_t* __restrict__ counts, uint32_t* __restrict__ seg) {
+  __shared__ uint32_t tmp[256 / 32 + 1];
+  const uint32_t c = counts[threadIdx.x];
+  uint32_t tot_n, tot_t;
+  const uint32_t s0 = block_scan<256>(c, tmp, &tot_n);
+  const uint32_t t0 = block_scan<256>((c + L2C::TILE - 1) / L2C::TILE, tmp, &tot_t);
+  seg[threadIdx.x] = s0;
+  seg[257 + threadIdx.x] = t0;
+  if (threadIdx.x == 0) {
+    seg[256] = tot_n;
+    seg[257 + 256] = tot_t;
+  }
+}
+
+// tile t of level 2 -> its segment, first level-1 position and length (s_seg: seg[] in smem)
+__device__ __forceinline__ void l2_tile(const uint32_t* s_seg, uint32_t t, uint32_t* s, uint32_t* t0, uint32_t* len) {
+  const uint32_t* tf = s_seg + 257;
+  uint32_t lo = 0, hi = 256;  // largest s with tf[s] <= t
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (tf[mid] <= t) lo = mid;
+    else hi = mid;
+  }
+  *s = lo;
+  *t0 = s_seg[lo] + (t - tf[lo]) * L2C::TILE;
+  const uint32_t end = s_seg[lo + 1];
+  *len = end - *t0 < (uint32_t)L2C::TILE ? end - *t0 : (uint32_t)L2C::TILE;
+}
+__device__ __forceinline__ void l2_tile_range(const uint32_t* s_seg, uint32_t* tb, uint32_t* te) {
+  const uint64_t T = s_seg[257 + 256];
+  *tb = (uint32_t)((uint64_t)blockIdx.x * T / gridDim.x);
+  *te = (uint32_t)((uint64_t)(blockIdx.x + 1) * T / gridDim.x);
+}
+__device__ __forceinline__ void l2_load_seg(uint32_t* s_seg, const uint32_t* __restrict__ seg) {
+  for (int i = threadIdx.x; i < 2 * 257; i += blockDim.x) s_seg[i] = seg[i];
+  __syncthreads();
+}
+
+// rank pass: each query's level-2 digit and its rank among the tile's queries with that digit
+__global__ void __launch_bounds__(L2C::NT, L2C::MINB) k_psa2_rank_s(const uint64_t* __restrict__ q1, L2Digit dg,
+                                                                   const uint32_t* __restrict__ seg,
+                                                                   uint32_t* __restrict__ packed2,
+                                                                   uint32_t* __restrict__ tile_counts2) {
+  __shared__ uint32_t s_seg[2 * 257];
+  __shared__ uint32_t cnt[L2C::BINS];
+  l2_load_seg(s_seg, seg);
+  uint32_t tb, te;
+  l2_tile_range(s_seg, &tb, &te);
+  for (uint32_t tile = tb; tile < te; ++tile) {
+    uint32_t s, t0, len;
+    l2_tile(s_seg, tile, &s, &t0, &len);
+    uint64_t v[L2C::PER];
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      v[k] = i < len ? __ldg(q1 + t0 + i) : 0;
+    }
+    cnt[threadIdx.x] = 0;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      if (i < len) {
+        const uint32_t d = dg(v[k]);
+        packed2[t0 + i] = d | (atomicAdd(&cnt[d], 1u) << 8);
+      }
+    }
+    __syncthreads();
+    tile_counts2[(uint64_t)tile * 256 + threadIdx.x] = cnt[threadIdx.x];
+    __syncthreads();
+  }
+}
+
+// per segment (one CTA) and digit (one thread): queries per 16-bit bucket
+__global__ void __launch_bounds__(256) k_l2_colsum(const uint32_t* __restrict__ seg,
+                                                   const uint32_t* __restrict__ tile_counts2,
+                                                   uint32_t* __restrict__ comp_cnt) {
+  const uint32_t s = blockIdx.x, t0 = seg[257 + s], t1 = seg[257 + s + 1];
+  uint32_t acc = 0;
+  for (uint32_t t = t0; t < t1; ++t) acc += __ldg(tile_counts2 + (uint64_t)t * 256 + threadIdx.x);
+  comp_cnt[s * 256 + threadIdx.x] = acc;
+}
+
+// level-2 layout (one CTA of 1024 threads): 16-bit buckets in groups of K, every group starts
+// at a multiple of 8; comp_start[b] = level-2 position of bucket b; the chunk table lists each
+// group (split into pieces of <= cap queries when larger); nch[0] = chunks, nch[1] = length.
+__global__ void __launch_bounds__(1024) k_l2_layout(const uint32_t* __restrict__ comp_cnt, uint32_t K, uint32_t cap,
+                                                    uint32_t* __restrict__ comp_start, uint2* __restrict__ chunks,
+                                                    uint32_t* __restrict__ chunk_pos, uint32_t* __restrict__ nch) {
+  __shared__ uint32_t tmp[1024 / 32 + 1];
+  const uint32_t ng = (kL2Buckets + K - 1) / K, gpt = (ng + 1023) / 1024;
+  const uint32_t g0 = min(ng, threadIdx.x * gpt), g1 = min(ng, g0 + gpt);
+  uint32_t padded = 0, pieces = 0, raw = 0;
+  for (uint32_t g = g0; g < g1; ++g) {
+    uint32_t sz = 0;
+    for (uint32_t b = g * K; b < min(kL2Buckets, (g + 1) * K); ++b) sz += comp_cnt[b];
+    padded += (sz + 7) & ~7u;
+    pieces += (sz + cap - 1) / cap;
+    raw += sz;
+  }
+  uint32_t tot_len, tot_ch, tot_raw;
+  uint32_t pos = block_scan<1024>(padded, tmp, &tot_len);
+  uint32_t ci = block_scan<1024>(pieces, tmp, &tot_ch);
+  uint32_t rpos = block_scan<1024>(raw, tmp, &tot_raw);
+  for (uint32_t g = g0; g < g1; ++g) {
+    uint32_t run = pos;
+    for (uint32_t b = g * K; b < min(kL2Buckets, (g + 1) * K); ++b) {
+      comp_start[b] = run;
+      run += comp_cnt[b];
+    }
+    const uint32_t sz = run - pos;
+    for (uint32_t o = 0; o < sz; o += cap) {
+      chunks[ci] = make_uint2(pos + o, min(cap, sz - o));
+      chunk_pos[ci++] = rpos + o;
+    }
+    pos += (sz + 7) & ~7u;
+    rpos += sz;
+  }
+  if (threadIdx.x == 0) {
+    comp_start[kL2Buckets] = tot_len;
+    nch[0] = tot_ch;
+    nch[1] = tot_len;
+  }
+}
+
+// per segment and digit: level-2 position of every tile's digit run (column scan)
+__global__ void __launch_bounds__(256) k_l2_tilebase(const uint32_t* __restrict__ seg,
+                                                     const uint32_t* __restrict__ tile_counts2,
+                                                     const uint32_t* __restrict__ comp_start,
+                                                     uint32_t* __restrict__ tile_base2) {
+  const uint32_t s = blockIdx.x, t0 = seg[257 + s], t1 = seg[257 + s + 1];
+  uint32_t run = comp_start[s * 256 + threadIdx.x];
+  for (uint32_t t = t0; t < t1; ++t) {
+    const uint64_t i = (uint64_t)t * 256 + threadIdx.x;
+    tile_base2[i] = run;
+    run += __ldg(tile_counts2 + i);
+  }
+}
+
+// staged move of every level-2 tile: level-1 order -> level-2 order (runs by consecutive lanes)
+__global__ void __launch_bounds__(L2C::NT, HM_MOVE_MINB) k_psa2_move_s(const uint64_t* __restrict__ q1, L2Digit dg,
+                                                                       const uint32_t* __restrict__ seg,
+                                                                       const uint32_t* __restrict__ packed2,
+                                                                       const uint32_t* __restrict__ tile_counts2,
+                                                                       const uint32_t* __restrict__ tile_base2,
+                                                                       uint64_t* __restrict__ q2) {
+  __shared__ uint32_t s_seg[2 * 257];
+  __shared__ __align__(16) uint64_t st_q[L2C::TILE];
+  __shared__ uint32_t bin_start[L2C::BINS], gbase[L2C::BINS], tmp[L2C::NT / 32 + 1];
+  l2_load_seg(s_seg, seg);
+  uint32_t tb, te;
+  l2_tile_range(s_seg, &tb, &te);
+  for (uint32_t tile = tb; tile < te; ++tile) {
+    uint32_t s, t0, len;
+    l2_tile(s_seg, tile, &s, &t0, &len);
+    uint64_t v[L2C::PER];
+    uint32_t pk[L2C::PER];
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      v[k] = i < len ? __ldg(q1 + t0 + i) : 0;
+      pk[k] = i < len ? __ldg(packed2 + t0 + i) : 0;
+    }
+    const uint64_t ti = (uint64_t)tile * 256 + threadIdx.x;
+    const uint32_t c = __ldg(tile_counts2 + ti);
+    gbase[threadIdx.x] = __ldg(tile_base2 + ti);
+    bin_start[threadIdx.x] = block_scan<L2C::NT>(c, tmp, nullptr);
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      if (i < len) st_q[bin_start[pk[k] & 255u] + (pk[k] >> 8)] = v[k];
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < len; i += L2C::NT) {
+      const uint64_t x = st_q[i];
+      const uint32_t d = dg(x);
+      q2[gbase[d] + (i - bin_start[d])] = x;
+    }
+    __syncthreads();
+  }
+}
+
+// inverse of k_psa2_move_s: res1[level-1 position] = res2[level-2 position]; reads res2 in
+// runs, writes res1 contiguously
+__global__ void __launch_bounds__(L2C::NT, HM_UNMOVE_MINB) k_psa2_unmove_s(const uint32_t* __restrict__ seg,
+                                                                           const uint32_t* __restrict__ packed2,
+                                                                           const uint32_t* __restrict__ tile_counts2,
+                                                                           const uint32_t* __restrict__ tile_base2,
+                                                                           const uint64_t* __restrict__ res2,
+                                                                           uint64_t* __restrict__ res1) {
+  __shared__ uint32_t s_seg[2 * 257];
+  __shared__ __align__(16) uint64_t st_r[L2C::TILE];
+  __shared__ uint32_t st_od[L2C::TILE];
+  __shared__ uint32_t bin_start[L2C::BINS], gbase[L2C::BINS], tmp[L2C::NT / 32 + 1];
+  l2_load_seg(s_seg, seg);
+  uint32_t tb, te;
+  l2_tile_range(s_seg, &tb, &te);
+  for (uint32_t tile = tb; tile < te; ++tile) {
+    uint32_t s, t0, len;
+    l2_tile(s_seg, tile, &s, &t0, &len);
+    uint32_t pk[L2C::PER];
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      pk[k] = i < len ? __ldg(packed2 + t0 + i) : 0;
+    }
+    const uint64_t ti = (uint64_t)tile * 256 + threadIdx.x;
+    const uint32_t c = __ldg(tile_counts2 + ti);
+    gbase[threadIdx.x] = __ldg(tile_base2 + ti);
+    bin_start[threadIdx.x] = block_scan<L2C::NT>(c, tmp, nullptr);
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      if (i < len) st_od[bin_start[pk[k] & 255u] + (pk[k] >> 8)] = i | ((pk[k] & 255u) << 11);
+    }
+    __syncthreads();
+    uint64_t rv[L2C::PER];
+    uint32_t oo[L2C::PER];
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k) {  // all loads in flight before the shared stores
+      const uint32_t i = k * L2C::NT + threadIdx.x;
+      if (i < len) {
+        const uint32_t od = st_od[i], d = od >> 11;
+        oo[k] = od & (L2C::TILE - 1);
+        rv[k] = __ldg(res2 + gbase[d] + (i - bin_start[d]));
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < L2C::PER; ++k)
+      if (k * L2C::NT + threadIdx.x < len) st_r[oo[k]] = rv[k];
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < len; i += L2C::NT) res1[t0 + i] = st_r[i];
+    __syncthreads();
+  }
+}
+
+// the queries of the level-2 chunks, pads skipped, in the order the search visits them
+// (harmonia_psa_inspect)
+__global__ void __launch_bounds__(256) k_l2_compact(const uint64_t* __restrict__ q2, const uint2* __restrict__ chunks,
+                                                    const uint32_t* __restrict__ nch, const uint32_t* __restrict__ cpos,
+                                                    uint64_t* __restrict__ out) {
+  for (uint32_t c = blockIdx.x; c < nch[0]; c += gridDim.x) {
+    const uint2 e = chunks[c];
+    for (uint32_t i = threadIdx.x; i < e.y; i += blockDim.x) out[cpos[c] + i] = q2[e.x + i];
+  }
+}
+
 // ---- level 2: chunk-local sort by the N-bit bucket (two stable LSD passes) ---------------
 template <int BITS, int SHIFT>
 __device__ __forceinline__ void lsd_pass(uint64_t (&v)[kSortBatches], uint32_t (&ix)[kSortBatches], uint32_t (&lk)[kSortBatches],
@@ -665,20 +931,12 @@ harmonia_status coarse_partition(const uint64_t* q, uint64_t n, const Digit& dg,
     ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
     if (idx) {
       constexpr size_t smb = move_smem<C, true, kRecompute>();
-      static bool cfg = false;
-      if (!cfg) {
-        HM_CUDA(cudaFuncSetAttribute(k_psa2_move<Digit, C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
-        cfg = true;
-      }
+      HM_CUDA(smem_attr(k_psa2_move<Digit, C, true>, smb));
       k_psa2_move<Digit, C, true><<<gm, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
                                                          ws.packed, ws.cta_counts, ws.cta_base, sorted_q, idx);
     } else {
       constexpr size_t smb = move_smem<C, false, kRecompute>();
-      static bool cfg = false;
-      if (!cfg) {
-        HM_CUDA(cudaFuncSetAttribute(k_psa2_move<Digit, C, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
-        cfg = true;
-      }
+      HM_CUDA(smem_attr(k_psa2_move<Digit, C, false>, smb));
       k_psa2_move<Digit, C, false><<<gm, C::NT, smb, st>>>(q, n, dg, ws.counts, ws.counts + C::BINS, ws.tile_counts,
                                                           ws.packed, ws.cta_counts, ws.cta_base, sorted_q, nullptr);
     }
@@ -691,11 +949,7 @@ template <class C>
 harmonia_status unpartition(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
                             cudaStream_t st) {
   constexpr size_t smb = unmove_smem<C>();
-  static bool cfg = false;
-  if (!cfg) {
-    HM_CUDA(cudaFuncSetAttribute(k_psa2_unmove<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb));
-    cfg = true;
-  }
+  HM_CUDA(smem_attr(k_psa2_unmove<C>, smb));
   ProfScope ps_(HARMONIA_PROF_RETURN, st);
   k_psa2_unmove<C><<<l1_grid_mv<C>(n, sm), C::NT, smb, st>>>(ws.tile_counts, ws.cta_base, ws.packed, res1, n, out);
   HM_LAUNCHED();
@@ -748,12 +1002,7 @@ harmonia_status route_push2(const uint64_t* q, uint64_t n, const BucketSplit& f,
   using C = Narrow;
   if (P > (uint32_t)C::BINS) return HARMONIA_ERR_INVALID_ARG;
   constexpr size_t smb = move_smem<C, false, false>();
-  static bool cfg = false;
-  if (!cfg) {
-    HM_CUDA(cudaFuncSetAttribute(k_psa2_move<BucketSplit, C, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)smb));
-    cfg = true;
-  }
+  HM_CUDA(smem_attr(k_psa2_move<BucketSplit, C, false, true>, smb));
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
     k_psa2_move<BucketSplit, C, false, true><<<l1_grid_mv<C>(n, sm), C::NT, smb, st>>>(
@@ -806,17 +1055,10 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
   if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation / fused chunk sort)
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);  // reported in the "scan" class: level-2 sort
-    static bool configured = false;
-    if (!configured) {
-      HM_CUDA(cudaFuncSetAttribute(k_psa2_local_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSortSmem));
-      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<false, kChunk>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)count_sort_smem<kChunk>()));
-      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<true, kChunk>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)count_sort_smem<kChunk>()));
-      HM_CUDA(cudaFuncSetAttribute(k_psa2_count_sort<true, (int)kPsaChunkMax>,
-                                   cudaFuncAttributeMaxDynamicSharedMemorySize, (int)count_sort_smem<kPsaChunkMax>()));
-      configured = true;
-    }
+    HM_CUDA(smem_attr(k_psa2_local_sort, kSortSmem));
+    HM_CUDA(smem_attr(k_psa2_count_sort<false, kChunk>, count_sort_smem<kChunk>()));
+    HM_CUDA(smem_attr(k_psa2_count_sort<true, kChunk>, count_sort_smem<kChunk>()));
+    HM_CUDA(smem_attr(k_psa2_count_sort<true, (int)kPsaChunkMax>, count_sort_smem<kPsaChunkMax>()));
 #ifndef HM_SORT_CTAS_PER_SM
 #define HM_SORT_CTAS_PER_SM 4
 #endif
@@ -836,6 +1078,77 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
     else
       k_psa2_count_sort<false, kChunk><<<std::max(g, 1), kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted_q, ws.idx, n, f);
   }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+
+// two-level PSA (Plan::psa_levels == 2) for the staged return: level 1 (rank + move on the top
+// 8 bits) into ws.sorted_q, level 2 (segmented rank + move on the next 8 bits) into
+// ws.sorted2, then the counting sort of the bucket-aligned chunks (K 16-bit buckets per
+// group, <= cap queries per chunk) in place; ws.idx receives the chunk-local offsets.
+harmonia_status psa_partition2_l2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
+                                  cudaStream_t st, uint32_t K, uint32_t cap) {
+  if (nb < 16 || (cap != kPsaChunk && cap != kPsaChunkMax)) return HARMONIA_ERR_INVALID_ARG;
+  harmonia_status s =
+      coarse_partition<Narrow>(q, n, CoarseDigit{f, (uint32_t)nb - 8}, ws, ws.sorted_q, nullptr, sm, st, nullptr, 0);
+  if (s != HARMONIA_OK) return s;
+  const L2Digit dg{f, (uint32_t)nb - 16};
+  const int g = l1_grid<L2C>(n + 256ull * L2C::TILE, sm), gm = l1_grid_mv<L2C>(n + 256ull * L2C::TILE, sm);
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_HIST, st);
+    k_l2_segs<<<1, 256, 0, st>>>(ws.counts, ws.seg);
+    k_psa2_rank_s<<<g, L2C::NT, 0, st>>>(ws.sorted_q, dg, ws.seg, ws.packed2, ws.tile_counts2);
+  }
+  HM_LAUNCHED();
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);
+    k_l2_colsum<<<256, 256, 0, st>>>(ws.seg, ws.tile_counts2, ws.comp_cnt);
+    k_l2_layout<<<1, 1024, 0, st>>>(ws.comp_cnt, K, cap, ws.comp_start, ws.chunks, ws.chunk_pos, ws.nchunks);
+    k_l2_tilebase<<<256, 256, 0, st>>>(ws.seg, ws.tile_counts2, ws.comp_start, ws.tile_base2);
+  }
+  HM_LAUNCHED();
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_SCATTER, st);
+    k_psa2_move_s<<<gm, L2C::NT, 0, st>>>(ws.sorted_q, dg, ws.seg, ws.packed2, ws.tile_counts2, ws.tile_base2,
+                                          ws.sorted2);
+  }
+  HM_LAUNCHED();
+  {
+    ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);
+    if (cap == kPsaChunkMax) {
+      auto kern = k_psa2_count_sort<true, (int)kPsaChunkMax, true>;
+      HM_CUDA(smem_attr(kern, count_sort_smem<kPsaChunkMax>()));
+      kern<<<sm * HM_SORT_CTAS_PER_SM_8K, kSortThreads, count_sort_smem<kPsaChunkMax>(), st>>>(ws.sorted2, ws.idx, n, f,
+                                                                                              ws.chunks, ws.nchunks);
+    } else {
+      auto kern = k_psa2_count_sort<true, kChunk, true>;
+      HM_CUDA(smem_attr(kern, count_sort_smem<kChunk>()));
+      kern<<<sm * HM_SORT_CTAS_PER_SM, kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted2, ws.idx, n, f,
+                                                                                      ws.chunks, ws.nchunks);
+    }
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
+// inverse of the two-level partition: res2 (level-2 order) -> ws.sorted_q as level-1-order
+// results (its queries are dead by now) -> out (caller order)
+harmonia_status psa_unpartition2_l2(const PsaWs& ws, const uint64_t* res2, uint64_t n, uint64_t* out, int sm,
+                                    cudaStream_t st) {
+  if (n == 0) return HARMONIA_OK;
+  {
+    ProfScope ps_(HARMONIA_PROF_RETURN, st);
+    k_psa2_unmove_s<<<l1_grid_mv<L2C>(n + 256ull * L2C::TILE, sm), L2C::NT, 0, st>>>(
+        ws.seg, ws.packed2, ws.tile_counts2, ws.tile_base2, res2, ws.sorted_q);
+  }
+  HM_LAUNCHED();
+  return unpartition<Narrow>(ws, ws.sorted_q, n, out, sm, st);
+}
+
+// harmonia_psa_inspect: the queries of the search's chunks in visiting order (two-level PSA)
+harmonia_status psa_compact_l2(const PsaWs& ws, uint64_t* out, int sm, cudaStream_t st) {
+  k_l2_compact<<<sm * 4, 256, 0, st>>>(ws.sorted2, ws.chunks, ws.nchunks, ws.chunk_pos, out);
   HM_LAUNCHED();
   return HARMONIA_OK;
 }

@@ -818,8 +818,20 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
   const bool ps_smem = a.ps_smem_bytes != 0;
   const bool leaf_smem = a.h - 1 < a.smem_levels;
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t c0 = (uint64_t)blockIdx.x * a.chunk; c0 < a.n; c0 += (uint64_t)gridDim.x * a.chunk) {
-    const uint32_t m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
+  // chunks: fixed a.chunk-query pieces of the level-1 order, or the bucket-aligned table of
+  // the two-level PSA (entries (start, queries), <= a.chunk queries each)
+  const uint64_t nch = a.ctab ? (uint64_t)*a.nctab : (a.n + a.chunk - 1) / a.chunk;
+  for (uint64_t c = blockIdx.x; c < nch; c += gridDim.x) {
+    uint64_t c0;
+    uint32_t m;
+    if (a.ctab) {
+      const uint2 e = a.ctab[c];
+      c0 = e.x;
+      m = e.y;
+    } else {
+      c0 = c * a.chunk;
+      m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
+    }
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
@@ -1218,11 +1230,7 @@ __global__ void __launch_bounds__(1024, 1) k_range_warp(const RangeArgs a) {
 template <int F>
 harmonia_status launch_range_warp_f(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
   auto kern = k_range_warp<F>;
-  static int configured_smem = -1;
-  if ((int)p.smem_bytes > configured_smem) {
-    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem = (int)p.smem_bytes;
-  }
+  HM_CUDA(smem_attr(kern, p.smem_bytes));
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, p.smem_bytes));
   per_sm = std::max(per_sm, 1);
@@ -1240,11 +1248,7 @@ template <int F>
 harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
   auto kern = a.staged ? k_sort_search<F, true> : k_sort_search<F, false>;
   const uint32_t smem = p.smem_bytes + kFuseSmem;
-  static int configured_smem[2] = {-1, -1};
-  if ((int)smem > configured_smem[a.staged ? 1 : 0]) {
-    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured_smem[a.staged ? 1 : 0] = (int)smem;
-  }
+  HM_CUDA(smem_attr(kern, smem));
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFuseThreads, smem));
   per_sm = std::max(per_sm, 1);
@@ -1264,16 +1268,11 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
                      : (U >= 4 ? k_lane_search_c<F, 4, false> : (U == 2 ? k_lane_search_c<F, 2, false> : k_lane_search_c<F, 1, false>));
   const uint32_t smem = a.res_smem_off + a.chunk * 8;
-  static int configured_smem[10] = {-1, -1, -1, -1, -1, -1, -1, -1, -1, -1};
-  const int ci = (U >= 4 ? 4 : U) + (a.coop ? 5 : 0);
-  if ((int)smem > configured_smem[ci]) {
-    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured_smem[ci] = (int)smem;
-  }
+  HM_CUDA(smem_attr(kern, smem));
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, HM_SEARCH_NT, smem));
   per_sm = std::max(per_sm, 1);
-  const uint64_t need = ceil_div(a.n, (uint64_t)a.chunk);
+  const uint64_t need = ceil_div(a.n, (uint64_t)a.chunk) + (a.ctab ? kL2Buckets : 0);
   const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
   {
     ProfScope ps_(HARMONIA_PROF_SEARCH, st);
@@ -1289,12 +1288,7 @@ harmonia_status launch_lane_search(const harmonia_tree* t, const Plan& p, const 
   const int U = p.lane_ilp;
   auto kern = U >= 4 ? k_lane_search_u<F, 4> : (U == 2 ? k_lane_search_u<F, 2> : k_lane_search<F>);
   const int bs = U >= 2 ? 1024 : kQueryBlock;
-  static int configured_smem[5] = {-1, -1, -1, -1, -1};
-  const int ci = U >= 4 ? 4 : U;
-  if ((int)p.smem_bytes > configured_smem[ci]) {
-    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem[ci] = (int)p.smem_bytes;
-  }
+  HM_CUDA(smem_attr(kern, p.smem_bytes));
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, bs, p.smem_bytes));
   per_sm = std::max(per_sm, 1);
@@ -1312,11 +1306,7 @@ template <int F, int G>
 harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
   const int mode = p.kary ? (p.ilp2 ? 2 : 1) : 0;
   auto kern = mode == 2 ? k_ntg_search2<F, G> : (mode == 1 ? k_ntg_search<F, G, 1> : k_ntg_search<F, G, 0>);
-  static int configured_smem[3] = {-1, -1, -1};  // per instantiation and mode
-  if ((int)p.smem_bytes > configured_smem[mode]) {
-    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem[mode] = (int)p.smem_bytes;
-  }
+  HM_CUDA(smem_attr(kern, p.smem_bytes));
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kQueryBlock, p.smem_bytes));
   per_sm = std::max(per_sm, 1);
@@ -1334,11 +1324,7 @@ harmonia_status launch_search_fg(const harmonia_tree* t, const Plan& p, const Se
 template <int F, int G>
 harmonia_status launch_range_fg(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
   auto kern = p.kary ? k_ntg_range<F, G, 1> : k_ntg_range<F, G, 0>;
-  static int configured_smem[2] = {-1, -1};
-  if ((int)p.smem_bytes > configured_smem[p.kary]) {
-    HM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes));
-    configured_smem[p.kary] = (int)p.smem_bytes;
-  }
+  HM_CUDA(smem_attr(kern, p.smem_bytes));
   int per_sm = 0;
   HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kQueryBlock, p.smem_bytes));
   per_sm = std::max(per_sm, 1);

@@ -232,6 +232,7 @@ static void free_tree(harmonia_tree* t) {
   cudaGetDevice(&cur);
   cudaSetDevice(t->device);
   cudaDeviceSynchronize();
+  l2_persist_release(t);
   cudaFree(t->d_keys);
   cudaFree(t->d_vals);
   cudaFree(t->d_ps);

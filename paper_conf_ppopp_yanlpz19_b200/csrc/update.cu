@@ -240,6 +240,11 @@ extern "C" harmonia_status harmonia_update_batch_seq(harmonia_tree* t, const uin
   if (n == 0) return HARMONIA_OK;
   if (!d_ops || !d_keys || !d_values || !ws) return HARMONIA_ERR_INVALID_ARG;
   if (n >= (1ull << 31)) return HARMONIA_ERR_INVALID_ARG;
+  // the CUB scans and the keep/position arrays count records in 32 bits: the
+  // merged sequence of at most n_keys + n records must stay below 2^31
+  if (t->n_keys + n >= (1ull << 31) - 1) return HARMONIA_ERR_TOO_LARGE;
+  DevGuard dg_(t->device, (cudaStream_t)stream);
+  if (dg_.status != HARMONIA_OK) return dg_.status;
   cudaStream_t st = (cudaStream_t)stream;
   const uint64_t nk = t->n_keys;
   const size_t cubb = cub_temp_bytes(n, nk);
@@ -359,6 +364,7 @@ extern "C" harmonia_status harmonia_update_batch_seq(harmonia_tree* t, const uin
     for (int l = 0; l <= HARMONIA_MAX_LEVELS; ++l) t->level_start[l] = old.level_start[l];
     return s;
   }
+  l2_persist_reset(t);  // the old key region (now the spare) must not stay pinned in L2
   if (nn > 0) {
     HM_CUDA(cudaMemcpyAsync(&t->min_key, NK, 8, cudaMemcpyDeviceToHost, st));
     HM_CUDA(cudaMemcpyAsync(&t->max_key, NK + nn - 1, 8, cudaMemcpyDeviceToHost, st));
@@ -367,6 +373,22 @@ extern "C" harmonia_status harmonia_update_batch_seq(harmonia_tree* t, const uin
     t->min_key = kPad;
     t->max_key = 0;
   }
+  return HARMONIA_OK;
+}
+
+extern "C" harmonia_status harmonia_update_validate(const uint8_t* d_ops, const uint64_t* d_keys,
+                                                    const uint64_t* d_values, uint64_t n, uint32_t* d_flags,
+                                                    void* stream) {
+  if (!d_flags) return HARMONIA_ERR_INVALID_ARG;
+  cudaStream_t st = (cudaStream_t)stream;
+  HM_CUDA(cudaMemsetAsync(d_flags, 0, 4, st));
+  if (n == 0) return HARMONIA_OK;
+  if (!d_ops || !d_keys || !d_values) return HARMONIA_ERR_INVALID_ARG;
+  int dev = 0, sm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sm, cudaDevAttrMultiProcessorCount, dev);
+  k_upd_validate<<<grid_of(n, sm), kBlock, 0, st>>>(d_ops, d_keys, d_values, n, (unsigned*)d_flags);
+  HM_LAUNCHED();
   return HARMONIA_OK;
 }
 

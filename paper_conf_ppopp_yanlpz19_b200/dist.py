@@ -27,7 +27,8 @@ from __future__ import annotations
 import torch
 import torch.distributed as dist
 
-from . import Tree, range_assemble, range_split, route_partition, route_update_payload, scatter_results
+from . import (HarmoniaError, Tree, range_assemble, range_split, route_partition, route_update_payload,
+               scatter_results, update_validate)
 
 __all__ = ["ReplicatedTree", "PartitionedTree", "PeerPartitionedTree", "CudaOps", "CudaPeerOps", "key_splitters",
            "peer_offsets"]
@@ -74,6 +75,9 @@ class CudaOps:
     def scatter(self, vals, pos):
         return scatter_results(vals, pos)
 
+    def validate_update(self, ops, keys, values):
+        return update_validate(ops, keys, values)
+
     def route_update(self, ops, keys, values, rank: int):
         rk, pos, counts = route_partition(self.split, self.P, keys)
         ro, rv, rs = route_update_payload(ops, values, pos, rank)
@@ -97,6 +101,13 @@ def _routed_update(tree_like, ops, keys, values):
     and the exchange deliver them in.  Collective: every rank calls it (possibly with 0 ops)."""
     ops_ = tree_like.ops
     group, P = tree_like.group, tree_like.world
+    # all shards accept the batch or all reject it: every rank's ops are validated before any
+    # is routed, the verdict is all-reduced, and every rank raises the same error (ADVICE r1)
+    flag = ops_.validate_update(ops, keys, values).to(torch.int32)
+    dist.all_reduce(flag, op=dist.ReduceOp.MAX, group=group)
+    bad = int(flag.item())
+    if bad:
+        raise HarmoniaError(3 if bad & 2 else 1, "partitioned update (some rank's batch)")
     rk, ro, rv, rs, counts = ops_.route_update(ops, keys, values, tree_like.rank)
     dev = keys.device
     send = torch.tensor(counts, dtype=torch.int64, device=dev)
@@ -121,11 +132,13 @@ def _routed_update(tree_like, ops, keys, values):
 class ReplicatedTree:
     """Same layout on every rank; each rank answers its own slice of the global batch."""
 
-    def __init__(self, keys, values, fanout: int = 64, fill: float = 1.0, group=None):
+    def __init__(self, keys, values, fanout: int = 64, fill: float = 1.0, group=None, tree=None):
         self.group = group
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
-        self.tree = Tree(keys, values, fanout=fanout, fill=fill)
+        # `tree`: any object with search/range (tests inject a CPU stand-in); default: the layout
+        # on this rank's device, built from the same seeded records on every rank
+        self.tree = tree if tree is not None else Tree(keys, values, fanout=fanout, fill=fill)
 
     def slice_of(self, n_global: int):
         """[begin, end) of this rank's share of an n_global-query batch."""
@@ -134,6 +147,20 @@ class ReplicatedTree:
 
     def search(self, q_local, **kw):
         return self.tree.search(q_local, **kw)
+
+    def search_global(self, q_global, gather: bool = False, **kw):
+        """This rank answers its slice of a batch every rank holds; no collective on the hot
+        path.  gather=True all-gathers the slices into the full result (outside any timed
+        region: it is the only collective of this mode)."""
+        b, e = self.slice_of(q_global.numel())
+        mine = self.search(q_global[b:e], **kw)
+        if not gather or self.world == 1:
+            return mine
+        n = q_global.numel()
+        parts = [torch.empty((n * (r + 1)) // self.world - (n * r) // self.world, dtype=torch.int64,
+                             device=mine.device) for r in range(self.world)]
+        dist.all_gather(parts, _i64(mine).contiguous(), group=self.group)
+        return _u64(torch.cat(parts))
 
     def range(self, lo, hi, cap, **kw):
         return self.tree.range(lo, hi, cap, **kw)

@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     assert len(names) >= 18
     for n in names:
         assert hasattr(L, n), n
-    assert L.harmonia_abi_version() == 1
+    assert L.harmonia_abi_version() == 2
 
 
 def test_sass_is_sm100a_and_uses_bulk_copy():

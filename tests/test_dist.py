@@ -113,6 +113,14 @@ class CpuOps:
                 f += take
         return torch.from_numpy(ko).view(torch.uint64), torch.from_numpy(vo).view(torch.uint64), torch.from_numpy(tot)
 
+    def validate_update(self, ops, keys, values):
+        kn = keys.view(torch.int64).numpy().view(np.uint64)
+        vn = values.view(torch.int64).numpy().view(np.uint64)
+        o = ops.numpy()
+        pad = np.uint64(0xFFFFFFFFFFFFFFFF)
+        bad = (2 if bool(np.any(kn == pad) or np.any((o == 0) & (vn == pad))) else 0) | (4 if bool(np.any(o > 1)) else 0)
+        return torch.tensor([bad], dtype=torch.int32)
+
     def route_update(self, ops, keys, values, rank):
         kn = keys.view(torch.int64).numpy().view(np.uint64)
         dest = np.searchsorted(self.split, kn, side="right")
@@ -356,3 +364,104 @@ def test_partitioned_update_gloo(world):
         assert p.exitcode == 0
     for rank, ok in res:
         assert ok, f"rank {rank}: routed updates differ from the global-order oracle"
+
+
+class CpuTree:
+    """Oracle stand-in for one rank's replicated layout (test only)."""
+
+    def __init__(self, keys, vals):
+        import oracle
+
+        self.orc, self.keys, self.vals = oracle, keys, vals
+
+    def search(self, q):
+        qn = q.view(torch.int64).numpy().view(np.uint64)
+        out = self.orc.sorted_search(self.keys, self.vals, qn, 1)
+        return torch.from_numpy(out.view(np.int64).copy()).view(torch.uint64)
+
+
+def _replicated_worker(rank, world, port, T, result_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_ppopp_yanlpz19_b200.dist import ReplicatedTree
+
+        keys = gen.uniform_keys(T)
+        vals = gen.values_for(keys)
+        rt = ReplicatedTree(keys, vals, tree=CpuTree(keys, vals))
+        q = np.concatenate([gen.uniform_queries(keys, 5001, miss_frac=0.3), gen.edge_queries(keys)])
+        qt = torch.from_numpy(q.view(np.int64).copy()).view(torch.uint64)
+        b, e = rt.slice_of(q.shape[0])
+        mine = rt.search_global(qt).view(torch.int64).numpy().view(np.uint64)
+        full = rt.search_global(qt, gather=True).view(torch.int64).numpy().view(np.uint64)
+        exp = oracle.sorted_search(keys, vals, q)
+        result_q.put((rank, bool(np.array_equal(mine, exp[b:e])), bool(np.array_equal(full, exp)), e - b))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_replicated_gloo(world):
+    """Replicated mode (SURVEY §8(e)): rank p answers [p*Q/P, (p+1)*Q/P) with no collective;
+    the slices tile the batch and the gathered result equals the oracle."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_replicated_worker, args=(r, world, port, 6000, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert sum(r[3] for r in res) == 5001 + len(gen.edge_queries(gen.uniform_keys(6000)))
+    for rank, ok_slice, ok_full, _ in res:
+        assert ok_slice and ok_full, rank
+
+
+def _reject_worker(rank, world, port, T, result_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_ppopp_yanlpz19_b200 import HarmoniaError
+        from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree, key_splitters
+
+        keys = gen.uniform_keys(T)
+        vals = gen.values_for(keys)
+        sp = key_splitters(keys, world)
+        bounds = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
+        lk, lv = keys[bounds[rank]:bounds[rank + 1]], vals[bounds[rank]:bounds[rank + 1]]
+        pt = PartitionedTree(lk, lv, sp, ops=CpuOps(lk, lv, sp, world))
+        o, k, v = gen.update_ops(keys, 500, insert_frac=0.1, seed=gen.SEED_OPS + rank)
+        if rank == 1:
+            k[7] = np.uint64(0xFFFFFFFFFFFFFFFF)  # a reserved key in one rank's batch only
+        t64 = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy()).view(torch.uint64)
+        status = None
+        try:
+            pt.update(torch.from_numpy(o.copy()), t64(k), t64(v))
+        except HarmoniaError as e:
+            status = e.status
+        got = pt.search(t64(keys)).view(torch.int64).numpy().view(np.uint64)
+        result_q.put((rank, status, bool(np.array_equal(got, oracle.sorted_search(keys, vals, keys)))))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_partitioned_update_rejects_everywhere(world):
+    """A reserved key in ONE rank's batch: every rank raises HARMONIA_ERR_RESERVED before any
+    shard applies an op, and every shard is unchanged."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_reject_worker, args=(r, world, port, 6000, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, status, unchanged in res:
+        assert status == 3 and unchanged, (rank, status, unchanged)

@@ -122,3 +122,11 @@ def test_fig9b_warp_level_steps(orc):
     # [2, 2]: GS 8 -> 4 keeps 1 step per warp (ratio 2); GS 4 -> 2 needs 2 steps for
     # target 2 (keys 0-1, then 2-3), ratio 2 * 1 / 2 = 1, so narrowing stops at 4
     assert lay.ntg_choose_gs(np.array([2, 2], dtype=np.uint64), 8, kpl=1, warp=8) == 4
+
+
+def test_psa_buckets_equals_scalar(orc):
+    keys = gen.uniform_keys(1 << 10)
+    q = gen.uniform_queries(keys, 500, miss_frac=0.5)
+    lo, hi = int(keys[0]), int(keys[-1])
+    b = orc.psa_buckets(q, 12, lo, hi)
+    assert b.tolist() == [orc.psa_bucket(int(x), 12, lo, hi) for x in q]
