@@ -278,11 +278,13 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       a.chunk = p.chunk;
       a.ctab = w.chunks;
       a.nctab = w.nchunks;
+      a.cbounds = w.cbounds;
       a.bucket = p.bucket;
       if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
       if ((s = psa_unpartition2_l2(w, w.res2, nw, out + w0, t->sm_count, st)) != HARMONIA_OK) return s;
       a.ctab = nullptr;
       a.nctab = nullptr;
+      a.cbounds = nullptr;
       continue;
     }
     if (p.ret) {  // staged return: level-1-order results, then the inverse move
@@ -294,7 +296,9 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
       a.chunk = p.chunk;
       a.bucket = p.bucket;
+      a.cbounds = fused ? nullptr : w.cbounds;
       if ((s = fused ? launch_sort_search(t, p, a, st) : launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+      a.cbounds = nullptr;
       if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, t->sm_count, st, p.wide)) != HARMONIA_OK) return s;
       continue;
     }

@@ -272,8 +272,12 @@ struct PsaWs {
   uint32_t* nchunks;    // [0] chunks, [1] padded level-2 length
   uint64_t* sorted2;    // level-2 order (window + padding)
   uint64_t* res2;       // results in level-2 order (window + padding)
+  uint2* cbounds;       // staged return: per chunk, its smallest and largest Nb-bit bucket (the
+                        // chunk sort writes them; the search starts every warp below the
+                        // chunk's shared path)
 };
 constexpr uint32_t kL2Buckets = 65536;  // 16-bit composite buckets of the two MSD levels
+inline uint64_t cbounds_entries(uint64_t window) { return window / 4096 + kL2Buckets + 4; }  // x 8 bytes
 constexpr uint64_t kL1CtaRows = 2048 * 2048;  // >= (level-1 CTAs) x (bins) for every tiling
 constexpr uint32_t kPsaTile = 2048;   // level-1 tile (queries), 256-bin configuration
 // bytes of one per-(tile, bin) array: max over the level-1 tilings (256 bins / 2048-query
@@ -337,6 +341,7 @@ struct SearchArgs {
   uint32_t res_smem_off;
   uint32_t chunk;          // staged return: level-2 chunk (queries), 4096 or 8192
   const uint2* ctab;       // chunk table (start, queries) instead of fixed chunks (psa_levels 2)
+  const uint2* cbounds;    // per chunk: min/max PSA bucket (nullptr = descend from the root)
   const uint32_t* nctab;   // device: chunks in ctab
   // warp-shared descent (G = 1 PSA path): clamp(q) -> (clamp(q) - kmin) >> cshift is a
   // monotone 32-bit image of the key, so two 32-bit warp reductions bound the warp's queries

@@ -169,6 +169,7 @@ size_t psa_ws_bytes(const Plan& p) {
   b += round_up(l1_rows_bytes(p.window), 256);        // per-tile counts
   b += 2 * kL1CtaRows * 4;                             // per-CTA counts and bases
   if (p.psa_levels == 2) b += l2_ws_bytes(p.window, p.chunk);
+  if (p.ret) b += round_up(cbounds_entries(p.window) * 8, 256);
   return b;
 }
 
@@ -193,6 +194,10 @@ PsaWs psa_ws_carve(const Plan& p, void* base) {
   c += kL1CtaRows * 4;
   w.cta_base = (uint32_t*)c;
   c += kL1CtaRows * 4;
+  if (p.ret) {
+    w.cbounds = (uint2*)c;
+    c += round_up(cbounds_entries(p.window) * 8, 256);
+  }
   if (p.psa_levels == 2) {
     const L2Sizes z = l2_sizes(p.window, p.chunk);
     w.seg = (uint32_t*)c;

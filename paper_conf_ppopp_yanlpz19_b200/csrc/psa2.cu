@@ -1072,9 +1072,11 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
       k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
     else if (local && ch == kPsaChunkMax)  // 8192-query chunks (denser key ranges per warp)
       k_psa2_count_sort<true, (int)kPsaChunkMax>
-          <<<std::max(g, 1), kSortThreads, count_sort_smem<kPsaChunkMax>(), st>>>(ws.sorted_q, ws.idx, n, f);
+          <<<std::max(g, 1), kSortThreads, count_sort_smem<kPsaChunkMax>(), st>>>(ws.sorted_q, ws.idx, n, f, nullptr,
+                                                                                 nullptr, ws.cbounds);
     else if (local)   // one counting pass with shared-memory atomics (default, measured faster)
-      k_psa2_count_sort<true, kChunk><<<std::max(g, 1), kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted_q, ws.idx, n, f);
+      k_psa2_count_sort<true, kChunk><<<std::max(g, 1), kSortThreads, count_sort_smem<kChunk>(), st>>>(
+          ws.sorted_q, ws.idx, n, f, nullptr, nullptr, ws.cbounds);
     else
       k_psa2_count_sort<false, kChunk><<<std::max(g, 1), kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted_q, ws.idx, n, f);
   }
@@ -1120,12 +1122,13 @@ harmonia_status psa_partition2_l2(const uint64_t* q, uint64_t n, const BucketBit
       auto kern = k_psa2_count_sort<true, (int)kPsaChunkMax, true>;
       HM_CUDA(smem_attr(kern, count_sort_smem<kPsaChunkMax>()));
       kern<<<sm * HM_SORT_CTAS_PER_SM_8K, kSortThreads, count_sort_smem<kPsaChunkMax>(), st>>>(ws.sorted2, ws.idx, n, f,
-                                                                                              ws.chunks, ws.nchunks);
+                                                                                              ws.chunks, ws.nchunks,
+                                                                                              ws.cbounds);
     } else {
       auto kern = k_psa2_count_sort<true, kChunk, true>;
       HM_CUDA(smem_attr(kern, count_sort_smem<kChunk>()));
       kern<<<sm * HM_SORT_CTAS_PER_SM, kSortThreads, count_sort_smem<kChunk>(), st>>>(ws.sorted2, ws.idx, n, f,
-                                                                                      ws.chunks, ws.nchunks);
+                                                                                      ws.chunks, ws.nchunks, ws.cbounds);
     }
   }
   HM_LAUNCHED();

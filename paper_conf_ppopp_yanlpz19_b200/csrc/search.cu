@@ -698,10 +698,30 @@ __device__ __forceinline__ void window_rank(const uint64_t* base, const uint64_t
   }
 }
 
+// The chunk's own shared path: the chunk sort recorded the chunk's smallest and largest
+// query, so every warp of the chunk shares the Eq-1 path of that interval.  One cooperative
+// descent per warp and chunk (instead of one per 64 queries) finds the node where the
+// chunk's interval splits; the warps start their own shared descent there.
+template <int F>
+__device__ __forceinline__ void chunk_path(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
+                                           bool ps_smem, uint64_t lo, uint64_t hi, uint32_t& node, uint32_t& lev) {
+  node = 0;
+  lev = 0;
+  if (lo > hi) return;
+  for (; lev + 1 < a.h; ++lev) {
+    uint32_t rlo, rhi;
+    if (lev < a.smem_levels) coop_rank<F, true, false>(s_keys + (uint64_t)node * F, lo, hi, rlo, rhi);
+    else coop_rank<F, false, false>(a.keys + (uint64_t)node * F, lo, hi, rlo, rhi);
+    if (rlo != rhi) return;
+    node = (ps_smem ? s_ps[node] : __ldg(a.ps + node)) + rlo;  // Eq 1
+  }
+}
+
 template <int F, int U>
 __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                           bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
-                                          const bool (&act)[U], uint64_t (&res)[U]) {
+                                          const bool (&act)[U], uint64_t (&res)[U], uint32_t node0 = 0,
+                                          uint32_t lev0 = 0) {
   uint64_t q[U];
   bool live[U];
   uint32_t tmin = 0xFFFFFFFFu, tmax = 0;
@@ -724,7 +744,7 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
   const uint64_t qlo = a.kmin + ((uint64_t)tmin << a.cshift);
   const uint64_t d = (uint64_t)tmax << a.cshift, m = (1ull << a.cshift) - 1;
   const uint64_t qhi = (a.kmax - a.kmin - d <= m) ? a.kmax : a.kmin + d + m;
-  uint32_t node = 0, l = 0;
+  uint32_t node = node0, l = lev0;
   for (; l + 1 < a.h; ++l) {
     const uint32_t first = ps_smem ? s_ps[node] : __ldg(a.ps + node);  // PS[node_idx]
     uint32_t rlo, rhi;
@@ -832,6 +852,18 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
       c0 = c * a.chunk;
       m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
     }
+    uint32_t node0 = 0, lev0 = 0;
+    if (COOP && a.cbounds) {
+      // bucket b holds the keys whose bits [shift, span) equal b under the common prefix of
+      // [kmin, kmax] (C-A11); queries outside [kmin, kmax] sit in the end buckets
+      const uint2 cb = a.cbounds[c];
+      const BucketBits& f = a.bucket;
+      const uint32_t span = f.shift + (uint32_t)__popc(f.mask);
+      const uint64_t pre = span >= 64 ? 0ull : f.kmin & ~((1ull << span) - 1);
+      const uint64_t lo = cb.x <= f(f.kmin) ? 0ull : pre | ((uint64_t)cb.x << f.shift);
+      const uint64_t hi = cb.y >= f(f.kmax) ? kPad - 1 : (pre | ((uint64_t)cb.y << f.shift)) + ((1ull << f.shift) - 1);
+      chunk_path<F>(a, s_keys, s_ps, ps_smem, lo, hi, node0, lev0);
+    }
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
@@ -848,7 +880,7 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
 #endif
       }
       uint64_t res[U];
-      if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res, node0, lev0);
       else lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
 #pragma unroll
       for (int u = 0; u < U; ++u)
