@@ -33,6 +33,11 @@ CONFIGS = {
     2: dict(name="c2_T2^23_F64_Q2^26_uniform", T=1 << 23, F=64, Q=1 << 26, dist="uniform"),
     3: dict(name="c3_T2^26_F64_Q2^26_zipf", T=1 << 26, F=64, Q=1 << 26, dist="zipf"),
     4: dict(name="c4_T2^28_F64_Q2^27_uniform_replicated", T=1 << 28, F=64, Q=1 << 27, dist="uniform"),
+    # config 5: 2^32 keys range-partitioned over 8 shards of 2^29 (rank p holds shard p), queries
+    # uniform over the running ranks' keys and routed, update batches of 2^22 ops (5 % insert,
+    # 5 % delete, 90 % update) interleaved 1:1 with the query batches
+    5: dict(name="c5_T2^32_8shards_F64_Q2^27_uniform_partitioned_updates", T=1 << 32, F=64, Q=1 << 27,
+            dist="uniform", shards=8, ops=1 << 22),
 }
 METRIC = "point queries/sec (G q/s) at 1/2/4/8 B200; % of L2/HBM roofline"
 UNIT = "G q/s"
@@ -62,6 +67,8 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--mode", default="replicated", choices=["replicated", "partitioned", "peer"])
     ap.add_argument("--sweep", default="", help="comma list of k=v option sets separated by ';' (diagnostics)")
+    ap.add_argument("--no-extra", action="store_true", help="skip the c4 / c3-fanout extra lines (default run)")
+    ap.add_argument("--extra-steps", type=int, default=10)
     return ap.parse_args()
 
 
@@ -154,27 +161,74 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------ CPU legs
-def cpu_oracle_rate(keys, vals, q, seconds):
-    """Time the oracle (std::lower_bound, all host threads) on a bounded sample of q."""
+def cpu_model() -> str:
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def _best_rate(fn, n, runs=5):
+    """queries/s of fn(n): one warm-up, then the best of `runs`."""
+    fn(n)
+    best = 1e30
+    for _ in range(runs):
+        t0 = time.perf_counter()
+        fn(n)
+        best = min(best, time.perf_counter() - t0)
+    return n / best, best
+
+
+def _size_for(fn, seconds, cap):
+    """A sample size whose run takes about `seconds` (calibrated on 2^16 queries)."""
+    n0 = min(cap, 1 << 16)
+    t0 = time.perf_counter()
+    fn(n0)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    return int(max(n0, min(cap, n0 * seconds / dt)))
+
+
+def cpu_baselines(keys, vals, q, seconds, fanout):
+    """The CPU oracle as it stands, on the host cores of this box: O1
+    std::lower_bound + value fetch and the O2 pointer B+tree (the paper's regular B+tree,
+    P:L120/L218; built by sorted-order insertion, fanout F), each with 1 thread and with
+    every host thread, best of 5 after 1 warm-up on a bounded sample of the batch."""
     import oracle
 
     nth = host_threads()
-    n = min(q.shape[0], 1 << 18)
+    per = max(0.2, seconds / 24.0)  # 4 legs x 6 runs
+    out = {"cores": nth, "cpu_model": cpu_model(), "method": "best of 5 after 1 warm-up"}
+    f1 = lambda n: oracle.sorted_search(keys, vals, q[:n], 1)
+    fN = lambda n: oracle.sorted_search(keys, vals, q[:n], nth)
+    n1 = _size_for(f1, per, q.shape[0])
+    nN = _size_for(fN, per, q.shape[0])
+    out["o1_1thread"], _ = _best_rate(f1, n1)
+    out["o1_all"], _ = _best_rate(fN, nN)
+    out["o1_samples"] = [n1, nN]
     t0 = time.perf_counter()
-    oracle.sorted_search(keys, vals, q[:n], nth)
-    dt = max(time.perf_counter() - t0, 1e-6)
-    n2 = int(min(q.shape[0], max(n, n * seconds / dt)))
-    t0 = time.perf_counter()
-    oracle.sorted_search(keys, vals, q[:n2], nth)
-    dt2 = time.perf_counter() - t0
-    return n2, dt2, nth
+    bpt = oracle.BPlusTree(fanout)
+    bpt.insert_many(keys, vals)
+    out["o2_build_s"] = time.perf_counter() - t0
+    out["o2_height"] = bpt.height
+    g1 = lambda n: bpt.search(q[:n], 1)
+    gN = lambda n: bpt.search(q[:n], nth)
+    m1 = _size_for(g1, per, q.shape[0])
+    mN = _size_for(gN, per, q.shape[0])
+    out["o2_1thread"], _ = _best_rate(g1, m1)
+    out["o2_all"], _ = _best_rate(gN, mN)
+    out["o2_samples"] = [m1, mN]
+    return out
 
 
 def run_reference(a, c, rank, world):
     """--impl reference: the CPU oracle (the only reference this paper-tier run has)."""
     if rank != 0:
         return
-    keys = gen.uniform_keys(c["T"])
+    T_ref = c["T"] // c.get("shards", 1)  # config 5: one shard (the CPU holds one shard's keys)
+    keys = gen.uniform_keys(c["T"], count=T_ref) if T_ref != c["T"] else gen.uniform_keys(c["T"])
     vals = gen.values_for(keys)
     q = make_queries(keys, c["Q"], c["dist"], 0)
     import oracle
@@ -200,7 +254,8 @@ def run_reference(a, c, rank, world):
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": dt / a.steps * 1e3,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
         "data": "synthetic", "config": {"workload": c["name"], "T": c["T"], "fanout": c["F"], "Q": c["Q"],
-                                        "queries": c["dist"], "sample_per_step": step_n},
+                                        "queries": c["dist"], "sample_per_step": step_n,
+                                        "oracle_keys": int(T_ref)},
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": nth, "kind": "oracle",
                          "sample": f"{step_n} of the {c['Q']} {c['dist']} queries per step; std::lower_bound "
                                    f"over {c['T']} sorted keys + value fetch, {nth} threads"},
@@ -234,6 +289,257 @@ def roofline_model(info, plan, nq_window, l2_bytes):
     return nq_window * io + tree, noreuse
 
 
+def step_model(info, plan, nq, l2_cap, hbm_gbs, l2_gbs, psa=True):
+    """Step-level roofline of SURVEY §8(d): bytes per query by tier and the bound
+    min(BW_HBM / B_HBM, BW_L2 / B_L2) in G q/s.
+
+    B_io = 16 (query in, result out), B_psa = 72 with PSA (histogram read 8, scatter 8 + 8 + 4,
+    search 8 + 8, gather 4 + 32 + 8, minus B_io); every level below the shared-memory stage
+    costs S + 32 (node + a PS or value sector).  Unstaged levels are in the L2 tier while their
+    cumulative bytes (the leaf level with its values) stay within the L2 capacity (+5 %: the c2
+    leaves + values are 131 MB against 126 MB, which SURVEY §8(d) counts as L2), the rest HBM.
+    B_HBM = B_io + B_psa + HBM-tier levels; B_L2 = B_HBM + L2-tier levels (HBM bytes also pass
+    L2).  The reuse-aware variant charges each tier min(no-reuse bytes, unique tier bytes / Q)."""
+    F, h, ls = info["fanout"], info["height"], info["level_start"]
+    S = F * 8
+    b_io, b_psa = 16, (72 if psa else 0)
+    cum, l2_lv, hbm_lv, l2_unique, hbm_unique = 0, 0, 0, 0, 0
+    for lev in range(plan["smem_levels"], h):
+        nodes = ls[lev + 1] - ls[lev]
+        lbytes = nodes * S * (2 if lev == h - 1 else 1)
+        cum += lbytes
+        if cum <= 1.05 * l2_cap:
+            l2_lv += S + 32
+            l2_unique += lbytes
+        else:
+            hbm_lv += S + 32
+            hbm_unique += lbytes
+    b_hbm = b_io + b_psa + hbm_lv
+    b_l2 = b_hbm + l2_lv
+    bound = min(hbm_gbs / b_hbm, l2_gbs / b_l2)
+    r_hbm = b_io + b_psa + min(hbm_lv, hbm_unique / nq)
+    r_l2 = r_hbm + min(l2_lv, l2_unique / nq)
+    rbound = min(hbm_gbs / r_hbm, l2_gbs / r_l2)
+    return {"B_hbm": b_hbm, "B_l2": b_l2, "bound_gqs": bound, "l2_tier_levels": l2_lv // (S + 32),
+            "hbm_tier_levels": hbm_lv // (S + 32),
+            "reuse_aware": {"B_hbm": r_hbm, "B_l2": r_l2, "bound_gqs": rbound}}
+
+
+def ncu_stats(workload, kernel):
+    """Per-launch ncu figures of `kernel` for `workload` from the committed capture summary
+    (profiles/ncu_r2.json, tools/ncu_summary.py): DRAM and L2 bytes, sectors per request
+    (the paper's memory divergence), warp coherence = active threads per
+    executed instruction / 32 (P:L654 fn 4), branch uniformity."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_r2.json")))
+        return d.get(workload, {}).get(kernel)
+    except Exception:
+        return None
+
+
+def load_peaks():
+    hbm, src = 6650.0, "fallback (B200_PROFILING.md)"
+    try:
+        p = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        hbm, src = float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        pass
+    l2, l2src = None, None
+    try:
+        p = json.load(open(os.path.join(ROOT, "profiles", "r2_peaks.json")))
+        l2, l2src = float(p["l2_read_gbs"]), "measured (profiles/r2_peaks.json, tools/peaks.cu)"
+    except Exception:
+        pass
+    return hbm, src, l2, l2src
+
+
+def timed(step, steps, stream):
+    """K steps bracketed by CUDA events on the launch stream (one event pair per step):
+    (total ms, per-step ms list)."""
+    import torch
+
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+    ev[0].record(stream)
+    for i in range(steps):
+        step()
+        ev[i + 1].record(stream)
+    torch.cuda.synchronize()
+    per = [ev[i].elapsed_time(ev[i + 1]) for i in range(steps)]
+    return ev[0].elapsed_time(ev[steps]), per
+
+
+def run_extras(hm, dev, a):
+    """Extra bench points measured in the default run: config 4 at N = 1 (the first point of
+    the metric's 1/2/4/8-GPU curve) and config 3's fanout sweep (Zipf, theta 0.99).  Device-
+    generated inputs; each point is warmed up and timed like the headline."""
+    import torch
+
+    out = {}
+    stream = torch.cuda.current_stream(dev)
+
+    def measure(t, q, steps):
+        res = torch.empty_like(q)
+        for _ in range(3):
+            t.search(q, res)
+        torch.cuda.synchronize()
+        hm.profile_enable(True)
+        hm.profile_read()
+        ms, per = timed(lambda: t.search(q, res), steps, stream)
+        hm.profile_enable(False)
+        pr = hm.profile_read()
+        ok = bool(torch.equal(res[:1 << 16].view(torch.int64), gen.values_for_t(q[:1 << 16].view(torch.int64))))
+        return {"value": q.numel() / (ms / steps) / 1e6, "unit": UNIT, "ms_per_step": ms / steps,
+                "ms_per_step_median": float(np.median(per)), "parity_sample_ok": ok,
+                "kernels_ms_per_step": {k: v[0] / steps for k, v in pr.items()}}
+
+    c4 = CONFIGS[4]
+    keys = gen.uniform_keys_t(c4["T"], dev)
+    t = hm.Tree(keys.view(torch.uint64), gen.values_for_t(keys).view(torch.uint64), fanout=c4["F"])
+    q = gen.uniform_queries_t(keys, c4["Q"]).view(torch.uint64)
+    r = measure(t, q, a.extra_steps)
+    r.update({"workload": c4["name"] + "_n1", "plan": t.plan(c4["Q"])})
+    out["c4_n1"] = r
+    del t, q, keys
+    torch.cuda.empty_cache()
+    c3 = CONFIGS[3]
+    keys = gen.uniform_keys_t(c3["T"], dev)
+    qz = gen.zipf_queries_t(keys, c3["Q"]).view(torch.uint64)
+    sweep = []
+    for F in (8, 16, 32, 64, 128):
+        t = hm.Tree(keys.view(torch.uint64), gen.values_for_t(keys).view(torch.uint64), fanout=F)
+        r = measure(t, qz, max(3, a.extra_steps // 2))
+        p = t.plan(c3["Q"])
+        sweep.append({"fanout": F, "value": r["value"], "ms_per_step": r["ms_per_step"],
+                      "parity_sample_ok": r["parity_sample_ok"], "psa_levels": p["psa_levels"],
+                      "height": t.info()["height"]})
+        del t
+        torch.cuda.empty_cache()
+    out["c3_fanout_sweep_zipf"] = {"workload": "c3_T2^26_Q2^26_zipf0.99", "unit": UNIT, "points": sweep}
+    return out
+
+
+def run_config5(a, c, hm, dev, world, rank, local, pg):
+    """Config 5: key-range partitioned tree, one 2^29-key shard of the
+    2^32-key set per rank (the 8-way partition; ranks 0..N-1 hold shards 0..N-1), queries
+    uniform over the running ranks' keys routed by NCCL all-to-all (bypassed at N = 1), and
+    one 2^22-op update batch (5 % insert, 5 % delete, 90 % update, routed) after every query
+    batch.  value = queries of all ranks / max-over-ranks time of query + update
+    batches; the update rate is reported beside it."""
+    import torch
+
+    from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree
+
+    T, P, S, F = c["T"], world, c["T"] // c["shards"], c["F"]
+    if P > c["shards"]:
+        raise SystemExit("config 5: at most %d ranks" % c["shards"])
+    lk = gen.uniform_keys_t(T, dev, start=rank * S, count=S)
+    sp = [int(x) & ((1 << 64) - 1) for x in gen.keys_at_t(T, torch.tensor([p * S for p in range(1, P)],
+                                                                            dtype=torch.int64)).tolist()]
+    t_build = time.perf_counter()
+    pt = PartitionedTree(lk.view(torch.uint64), gen.values_for_t(lk).view(torch.uint64), sp, fanout=F, device=dev)
+    torch.cuda.synchronize()
+    t_build = time.perf_counter() - t_build
+    del lk
+    t = pt.ops.tree
+    info = t.info()
+    nidx = gen._t_umod(gen._t_stream(gen.SEED_QUERY, rank * c["Q"], c["Q"], dev), P * S)
+    q = gen.keys_at_t(T, nidx).view(torch.uint64)
+    del nidx
+    nb = 8  # distinct update batches, cycled (each step applies a fresh batch of the cycle)
+    batches = [gen.update_ops_t(T, c["ops"], 0.05, 0.05, dev, seed=gen.SEED_OPS + 1000 * b + rank, hi=P * S)
+               for b in range(nb)]
+    batches = [(o, k.view(torch.uint64), v.view(torch.uint64)) for o, k, v in batches]
+    out = torch.empty_like(q)
+    first = pt.search(q)
+    torch.cuda.synchronize()
+    sel = torch.from_numpy(np.asarray(gen._stream(99, 0, 1 << 16) % np.uint64(c["Q"]), dtype=np.int64)).to(dev)
+    parity_ok = bool(torch.equal(first.view(torch.int64)[sel], gen.values_for_t(q.view(torch.int64)[sel])))
+    it = [0]
+
+    def step():
+        out.copy_(pt.search(q))
+        o, k, v = batches[it[0] % nb]
+        it[0] += 1
+        pt.update(o, k, v)
+
+    for _ in range(max(3, a.warmup)):
+        step()
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream(dev)
+    if pg:
+        pg.barrier()
+    torch.cuda.synchronize()
+    l0 = hm.kernel_launches()
+    hm.profile_enable(True)
+    hm.profile_read()
+    with ClockSampler(local) as clk:
+        ms, per_step = timed(step, a.steps, stream)
+    hm.profile_enable(False)
+    launches = hm.kernel_launches() - l0
+    prof = hm.profile_read()
+    ms_max = ms
+    if pg:
+        tt = torch.tensor([ms], device=dev, dtype=torch.float64)
+        pg.all_reduce(tt, op=pg.ReduceOp.MAX)
+        ms_max = float(tt.item())
+    value = c["Q"] * world * a.steps / (ms_max / 1e3) / 1e9
+    ups = c["ops"] * world * a.steps / (ms_max / 1e3) / 1e9
+    e2e = None
+    if not a.no_e2e:
+        q_host = q.cpu().pin_memory()
+        out_host = torch.empty(c["Q"], dtype=torch.uint64, pin_memory=True)
+
+        def e2e_step():
+            q.copy_(q_host, non_blocking=True)
+            out_host.copy_(pt.search(q), non_blocking=True)
+            o, k, v = batches[it[0] % nb]
+            it[0] += 1
+            pt.update(o, k, v)
+
+        e2e_step()
+        torch.cuda.synchronize()
+        k2 = max(1, a.e2e_steps)
+        hms, _ = timed(e2e_step, k2, stream)
+        if pg:
+            tt = torch.tensor([hms], device=dev, dtype=torch.float64)
+            pg.all_reduce(tt, op=pg.ReduceOp.MAX)
+            hms = float(tt.item())
+        e2e = {"value": c["Q"] * world * k2 / (hms / 1e3) / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": int(c["Q"] * 8), "d2h_bytes_per_step": int(c["Q"] * 8), "steps": k2,
+               "ms_per_step": hms / k2, "api": "PartitionedTree.search + update, pinned query/result copies",
+               "note": "update batches are device-resident (generated on the device) in both measurements"}
+    if rank != 0:
+        return
+    hbm_peak, peak_src, _, _ = load_peaks()
+    breakdown = {k: {"ms_per_step": v[0] / a.steps, "launches_per_step": v[1] / a.steps,
+                     "share": v[0] / max(1e-9, sum(x[0] for x in prof.values()))} for k, v in prof.items()}
+    roof = None
+    if "update" in prof:  # the rebuild: read records (16 B), write merged records (16 B),
+        # write the key region + leaf values (16 B x F/(F-1)) per record of the shard
+        n_rec = info["n_keys"]
+        byt = n_rec * (16 + 16 + 16 * F / (F - 1))
+        avg = prof["update"][0] / prof["update"][1]
+        roof = {"bound": "hbm", "kernel": "harmonia_update_batch (sort, merge, layout rebuild)",
+                "achieved": byt / (avg / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
+                "frac": byt / (avg / 1e3) / 1e9 / hbm_peak, "traffic": None, "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": byt, "avg_launch_ms": avg}
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
+        "warmup": max(3, a.warmup), "ms_per_step": ms_max / a.steps,
+        "ms_per_step_median": float(np.median(per_step)), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": c["name"], "T": T, "shard_keys": S, "fanout": F, "Q_per_gpu": c["Q"],
+                   "update_ops_per_step_per_gpu": c["ops"], "update_mix": "5% insert, 5% delete, 90% update",
+                   "queries": "uniform over the running shards' keys", "mode": "partitioned",
+                   "l2_flush": "inputs_larger_than_L2 (2^27 queries + a 2^29-key shard per GPU)",
+                   "plan": t.plan(c["Q"]), "height": info["height"], "build_s": t_build},
+        "updates_per_s": {"value": ups, "unit": "G ops/s"},
+        "roofline": roof, "cpu_baseline": None, "e2e": e2e, "gpu_launches": int(launches),
+        "clocks": clk.summary(), "kernel_breakdown": breakdown, "parity_sample_ok": parity_ok,
+    }
+    print(json.dumps(line), flush=True)
+
+
 def main():
     a = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -260,7 +566,7 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     pg = None
-    if world > 1 or a.mode in ("partitioned", "peer"):
+    if world > 1 or a.mode in ("partitioned", "peer") or a.config == 5:
         import torch.distributed as dist
 
         if world == 1:  # a one-rank group without torchrun (--mode partitioned/peer at N = 1)
@@ -274,6 +580,12 @@ def main():
     def barrier():
         if pg:
             pg.barrier()
+
+    if a.config == 5:
+        run_config5(a, c, hm, dev, world, rank, local, pg)
+        if pg:
+            pg.destroy_process_group()
+        return
 
     # ---- inputs (synthetic, seeded).  replicated: identical tree on every rank, each rank its
     # own slice of the global query stream (weak scaling, no collective).  partitioned: rank p
@@ -344,23 +656,17 @@ def main():
 
     # ---- timed region: K steps, events on the launch stream, max over ranks
     stream = torch.cuda.current_stream(dev)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
     torch.cuda.synchronize()
     l0 = hm.kernel_launches()
     hm.profile_enable(True)
     hm.profile_read()
     with ClockSampler(local) as clk:
-        e0.record(stream)
-        for _ in range(a.steps):
-            step()
-        e1.record(stream)
-        torch.cuda.synchronize()
+        ms, per_step = timed(step, a.steps, stream)
     hm.profile_enable(False)
     launches = hm.kernel_launches() - l0
     prof = hm.profile_read()
     barrier()
-    ms = e0.elapsed_time(e1)
     ms_max = ms
     if pg:
         tt = torch.tensor([ms], device=dev, dtype=torch.float64)
@@ -411,12 +717,7 @@ def main():
         return
 
     # ---- roofline of the dominant kernel (events around each launch, same stream)
-    peaks = {}
-    try:
-        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-        hbm_peak, peak_src = float(peaks["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
-    except Exception:
-        hbm_peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
+    hbm_peak, peak_src, l2_peak, l2_src = load_peaks()
     dom = max(prof.items(), key=lambda kv: kv[1][0]) if prof else ("search", (ms, 1))
     dom_kind, (dom_ms, dom_n) = dom
     l2_bytes = torch.cuda.get_device_properties(dev).L2_cache_size
@@ -453,35 +754,54 @@ def main():
         roof = {"bound": "hbm", "kernel": dom_kind, "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
                 "frac": achieved / hbm_peak, "traffic": None, "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": nw * per_q, "avg_launch_ms": avg_ms}
-    # ncu DRAM traffic per launch, if a capture summary was committed for this workload
-    try:
-        prof_sum = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        ent = prof_sum.get(c["name"], {}).get(roof["kernel"])
-        if ent:
-            roof["traffic"] = ent["dram_bytes_per_launch"]
-            roof["traffic_source"] = ent.get("source")
-            if "l1_wavefront_pct" in ent:  # the on-chip limiter of the search
-                roof["limiter"] = {"resource": "L1 data-pipe (LSU) wavefronts", "frac": ent["l1_wavefront_pct"] / 100,
-                                   "source": ent.get("source")}
-            if ent.get("sol_pct"):  # ncu speed-of-light of every tier: none saturated -> latency-bound
-                roof["ncu_sol"] = {k: v / 100 for k, v in ent["sol_pct"].items()}
-                if ent.get("ncu_time_s"):  # DRAM GB/s of the captured launch vs the measured peak
-                    roof["ncu_sol"]["dram"] = ent["dram_bytes_per_launch"] / ent["ncu_time_s"] / 1e9 / hbm_peak
-                if "long_scoreboard_stall_share" in ent:
-                    roof["ncu_sol"]["long_scoreboard_stall_share"] = ent["long_scoreboard_stall_share"]
-    except Exception:
-        pass
+    # L2 tier of the same kernel: its L2 traffic per launch (ncu lts__t_bytes of the committed
+    # capture) over the live launch time, against the measured L2 read peak; and the step-level
+    # model of SURVEY §8(d) (no-reuse and reuse-aware) against the measured step rate
+    st = ncu_stats(c["name"], roof["kernel"]) if roof else None
+    if roof is not None and st:
+        roof["traffic"] = st.get("dram_bytes")
+        roof["traffic_source"] = st.get("source")
+        if l2_peak and st.get("lts_bytes"):
+            ach = st["lts_bytes"] / (roof["avg_launch_ms"] / 1e3) / 1e9
+            roof["l2"] = {"achieved": ach, "peak": l2_peak, "unit": "GB/s", "frac": ach / l2_peak,
+                          "bytes_per_launch": st["lts_bytes"], "peak_source": l2_src,
+                          "bytes_source": st.get("source")}
+        roof["ncu"] = {k: st[k] for k in ("sectors_per_request", "warp_coherence", "branch_uniform_pct",
+                                          "dram_bytes_per_query", "lts_bytes_per_query", "l1_hit_pct",
+                                          "lts_hit_pct", "issue_active_pct", "l1_wavefront_pct", "lts_pct",
+                                          "long_scoreboard_stall_share") if k in st}
+        if "l1_wavefront_pct" in st:  # the on-chip limiter of the search
+            roof["limiter"] = {"resource": "L1 data-pipe (LSU) wavefronts", "frac": st["l1_wavefront_pct"] / 100,
+                               "source": st.get("source")}
+    if roof is not None and l2_peak:
+        sm_ = step_model(info, plan, c["Q"] * 1, l2_bytes, hbm_peak, l2_peak, psa=plan["psa_bits"] > 0)
+        sm_["frac"] = value / world / sm_["bound_gqs"]
+        sm_["reuse_aware"]["frac"] = value / world / sm_["reuse_aware"]["bound_gqs"]
+        sm_["note"] = "per GPU; no-reuse frac > 1 means PSA neighbours share nodes (SURVEY §8(d) caveat)"
+        roof["step_model"] = sm_
 
     cpu = None
     if not a.no_cpu and world == 1:
-        n2, dt2, nth = cpu_oracle_rate(keys, vals, q_np, a.cpu_seconds)
-        cpu = {"value": n2 / dt2 / 1e9, "unit": UNIT, "cores": nth, "kind": "oracle",
-               "sample": f"first {n2} of the {c['Q']} {c['dist']} queries; std::lower_bound over {c['T']} "
-                         f"sorted keys + value fetch; {dt2:.1f} s"}
+        cb = cpu_baselines(keys, vals, q_np, a.cpu_seconds, c["F"])
+        cpu = {"value": cb["o1_all"] / 1e9, "unit": UNIT, "cores": cb["cores"], "kind": "oracle",
+               "sample": f"prefixes of the {c['Q']} {c['dist']} queries ({cb['o1_samples'][1]} for all threads, "
+                         f"{cb['o1_samples'][0]} for 1 thread); std::lower_bound over {c['T']} sorted keys + value "
+                         f"fetch; best of 5 after 1 warm-up", "cpu_model": cb["cpu_model"],
+               "one_thread": cb["o1_1thread"] / 1e9,
+               "bptree": {"value": cb["o2_all"] / 1e9, "one_thread": cb["o2_1thread"] / 1e9,
+                          "what": f"O2 pointer B+tree (P:L120/L218), fanout {c['F']}, built by sorted insertion "
+                                  f"in {cb['o2_build_s']:.1f} s, height {cb['o2_height']}",
+                          "samples": cb["o2_samples"]}}
+    extra = None
+    if a.config == 2 and world == 1 and not a.no_extra and not (a.keys or a.queries or a.fanout or a.dist):
+        del q, out
+        torch.cuda.empty_cache()
+        extra = run_extras(hm, dev, a)
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
-        "warmup": max(3, a.warmup), "ms_per_step": ms_max / a.steps, "higher_is_better": True,
+        "warmup": max(3, a.warmup), "ms_per_step": ms_max / a.steps,
+        "ms_per_step_median": float(np.median(per_step)), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": c["name"], "T": c["T"], "fanout": c["F"], "fill": a.fill, "Q_per_gpu": c["Q"],
                    "queries": c["dist"], "mode": a.mode if (world > 1 or a.mode in ("partitioned", "peer")) else "single",
@@ -492,6 +812,8 @@ def main():
         "clocks": clk.summary(), "kernel_breakdown": breakdown, "parity_sample_ok": parity_ok,
         "context": {"paper_titan_v_gqs": PAPER_TITANV_GQS, "note": "P:L40/L592, TITAN V — other hardware"},
     }
+    if extra:
+        line["extra"] = extra
     print(json.dumps(line), flush=True)
     if pg:
         pg.destroy_process_group()

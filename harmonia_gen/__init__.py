@@ -256,6 +256,59 @@ def uniform_queries_t(keys, Q: int, seed: int = SEED_QUERY, start: int = 0):
     return keys[_t_umod(_t_stream(seed, start, Q, keys.device), T)]
 
 
+def keys_at_t(T: int, idx, seed: int = SEED_KEY):
+    """uniform_keys(T)[idx] for an int64 index tensor (the closed form per index)."""
+    D = ((1 << 64) - 2) // T
+    return idx * _t_const(D, idx.device) + _t_umod(splitmix64_t(_t_const(seed & _M64, idx.device) ^ idx), D)
+
+
+def _t_unit(seed: int, start: int, n: int, device):
+    import torch
+
+    return _t_lsr(_t_stream(seed, start, n, device), 11).to(torch.float64) * (1.0 / (1 << 53))
+
+
+def zipf_queries_t(keys, Q: int, theta: float = 0.99, seed: int = SEED_QUERY, start: int = 0):
+    """zipf_queries on the device (same streams and formulas in float64; equal to the numpy
+    version up to the last-ulp rounding of pow, tests/test_gen.py)."""
+    import torch
+
+    T = keys.shape[0]
+    zetan = _zeta(T, theta)
+    zeta2 = 1.0 + 0.5 ** theta
+    alpha = 1.0 / (1.0 - theta)
+    eta = (1.0 - (2.0 / T) ** (1.0 - theta)) / (1.0 - zeta2 / zetan)
+    u = _t_unit(seed ^ 0x3333, start, Q, keys.device)
+    uz = u * zetan
+    r = torch.floor(T * torch.pow(eta * u - eta + 1.0, alpha))
+    r = torch.where(uz < 1.0, torch.zeros_like(r), torch.where(uz < 1.0 + 0.5 ** theta, torch.ones_like(r), r))
+    r = torch.clamp(r, max=T - 1).to(torch.int64)
+    return keys[_t_umod(splitmix64_t(r), T)]
+
+
+def update_ops_t(T: int, n: int, insert_frac: float, delete_frac: float, device, seed: int = SEED_OPS,
+                 lo: int = 0, hi: int | None = None):
+    """update_ops over the keys uniform_keys(T)[lo:hi], generated on the device from indices
+    (no key array needed: the partitioned config holds 2^29 keys per shard).  Inserts are the
+    midpoints of random gaps, updates/deletes hit existing keys.  Returns (ops uint8, keys
+    int64, values int64) tensors."""
+    import torch
+
+    hi = T if hi is None else hi
+    u = _t_unit(seed, 0, n, device)
+    span = max(1, hi - lo - 1)
+    g = _t_umod(_t_stream(seed ^ 0x99, 0, n, device), span) + lo
+    a, b = keys_at_t(T, g), keys_at_t(T, g + 1)
+    mid = a + _t_lsr(b - a, 1)
+    exist = keys_at_t(T, _t_umod(_t_stream(seed ^ 0x98, 0, n, device), hi - lo) + lo)
+    is_ins = u < insert_frac
+    is_del = (u >= insert_frac) & (u < insert_frac + delete_frac)
+    k = torch.where(is_ins, mid, exist)
+    ops = is_del.to(torch.uint8)
+    v = values_for_t(_t_stream(seed ^ 0xAA, 0, n, device), seed ^ 0xBB)
+    return ops, k, v
+
+
 # ------------------------------------------------------------------------------ updates
 def update_ops(keys: np.ndarray, n: int, insert_frac: float = 0.05, delete_frac: float = 0.0,
                seed: int = SEED_OPS):

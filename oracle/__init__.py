@@ -63,6 +63,8 @@ def lib():
             "orc_bpt_insert": (C.c_int, [C.c_void_p, C.c_uint64, C.c_uint64]),
             "orc_bpt_erase": (C.c_int, [C.c_void_p, C.c_uint64]),
             "orc_bpt_search": (None, [C.c_void_p, u64p, C.c_uint64, u64p]),
+            "orc_bpt_search_mt": (None, [C.c_void_p, u64p, C.c_uint64, u64p, C.c_int]),
+            "orc_bpt_insert_array": (C.c_uint64, [C.c_void_p, u64p, u64p, C.c_uint64]),
             "orc_bpt_range": (None, [C.c_void_p, u64p, u64p, C.c_uint64, C.c_uint32, u64p, u64p, u32p]),
             "orc_bpt_size": (C.c_uint64, [C.c_void_p]),
             "orc_bpt_height": (C.c_uint32, [C.c_void_p]),
@@ -171,16 +173,19 @@ class BPlusTree:
         return lib().orc_bpt_insert(self._h, int(k), int(v))
 
     def insert_many(self, keys, vals):
-        for k, v in zip(np.asarray(keys, dtype=np.uint64).tolist(), np.asarray(vals, dtype=np.uint64).tolist()):
-            lib().orc_bpt_insert(self._h, k, v)
+        k, v = _u64(keys), _u64(vals)
+        return int(lib().orc_bpt_insert_array(self._h, _p64(k), _p64(v), k.shape[0]))
 
     def erase(self, k) -> int:
         return lib().orc_bpt_erase(self._h, int(k))
 
-    def search(self, q) -> np.ndarray:
+    def search(self, q, nthreads: int = 1) -> np.ndarray:
         q = _u64(q)
         out = np.empty(q.shape[0], dtype=np.uint64)
-        lib().orc_bpt_search(self._h, _p64(q), q.shape[0], _p64(out))
+        if nthreads == 1:
+            lib().orc_bpt_search(self._h, _p64(q), q.shape[0], _p64(out))
+        else:
+            lib().orc_bpt_search_mt(self._h, _p64(q), q.shape[0], _p64(out), nthreads)
         return out
 
     def range(self, lo, hi, cap: int):

@@ -13,6 +13,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <thread>
 #include <vector>
 
 namespace {
@@ -269,6 +270,30 @@ extern "C" void orc_bpt_search(void* tp, const uint64_t* q, uint64_t nq, uint64_
     out[j] = (it != n->keys.end() && *it == q[j]) ? n->vals[it - n->keys.begin()]
                                                     : ORC_NOT_FOUND;
   }
+}
+
+// The same search split over nthreads host threads (static chunks; the tree is read-only
+// here), for the CPU baseline timing of the paper's pointer B+tree.
+extern "C" void orc_bpt_search_mt(void* tp, const uint64_t* q, uint64_t nq, uint64_t* out, int nthreads) {
+  if (nthreads <= 0) nthreads = (int)std::max(1u, std::thread::hardware_concurrency());
+  if (nthreads == 1 || nq < 4096) {
+    orc_bpt_search(tp, q, nq, out);
+    return;
+  }
+  std::vector<std::thread> th;
+  const uint64_t chunk = (nq + nthreads - 1) / nthreads;
+  for (int i = 0; i < nthreads; ++i) {
+    const uint64_t b = std::min<uint64_t>(nq, i * chunk), e = std::min<uint64_t>(nq, b + chunk);
+    if (b < e) th.emplace_back([=] { orc_bpt_search(tp, q + b, e - b, out + b); });
+  }
+  for (auto& x : th) x.join();
+}
+
+// n inserts in array order (one orc_bpt_insert each); returns the number of new keys
+extern "C" uint64_t orc_bpt_insert_array(void* tp, const uint64_t* keys, const uint64_t* vals, uint64_t n) {
+  uint64_t fresh = 0;
+  for (uint64_t i = 0; i < n; ++i) fresh += (uint64_t)orc_bpt_insert(tp, keys[i], vals[i]);
+  return fresh;
 }
 
 extern "C" void orc_bpt_range(void* tp, const uint64_t* lo, const uint64_t* hi, uint64_t nq,

@@ -58,6 +58,8 @@ void     orc_bpt_destroy(void* t);
 int      orc_bpt_insert(void* t, uint64_t key, uint64_t value); /* 1 new, 0 replaced */
 int      orc_bpt_erase(void* t, uint64_t key);                  /* 1 erased, 0 absent */
 void     orc_bpt_search(void* t, const uint64_t* q, uint64_t nq, uint64_t* out);
+void     orc_bpt_search_mt(void* t, const uint64_t* q, uint64_t nq, uint64_t* out, int nthreads);
+uint64_t orc_bpt_insert_array(void* t, const uint64_t* keys, const uint64_t* vals, uint64_t n);
 void     orc_bpt_range(void* t, const uint64_t* lo, const uint64_t* hi, uint64_t nq,
                        uint32_t cap, uint64_t* kout, uint64_t* vout, uint32_t* counts);
 uint64_t orc_bpt_size(void* t);

@@ -24,6 +24,7 @@ constexpr uint64_t kAutoWindow = 1ull << 27;  // auto PSA window (queries): meas
 #define HM_L16_DENSITY 0.5
 #endif
 constexpr double kL16MaxChunkDensity = HM_L16_DENSITY;  // two PSA levels below this density
+constexpr uint64_t kL16MinKeys = 1ull << 27;
 
 bool pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
 }  // namespace
@@ -136,7 +137,10 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.psa_levels = 1;
   if (P.ret && P.nb >= 16 && !(o->flags & HARMONIA_QF_PSA_WIDE) && !(o->flags & HARMONIA_QF_PSA_L8)) {
     const double dens = t->L ? (double)kPsaChunk * 256.0 / (double)t->L : 1e9;
-    if ((o->flags & HARMONIA_QF_PSA_L16) || dens < kL16MaxChunkDensity) P.psa_levels = 2;
+    // and only for trees far beyond L2 (>= 2^27 keys): with 2^26 keys a Zipf batch (c3) lost
+    // 30 % with two levels, uniform ones broke even
+    if ((o->flags & HARMONIA_QF_PSA_L16) || (dens < kL16MaxChunkDensity && t->n_keys >= kL16MinKeys))
+      P.psa_levels = 2;
   }
   if (P.psa_levels == 2) {
     if (o->sort_chunk == 0) P.chunk = kPsaChunkMax;  // measured: 8192 beats 4096 at every size

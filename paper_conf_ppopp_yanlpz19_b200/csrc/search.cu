@@ -827,7 +827,11 @@ __global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const 
 #ifndef HM_SEARCH_NT
 #define HM_SEARCH_NT 1024  // threads per staged-search CTA (2 CTAs per SM)
 #endif
-template <int F, int U, bool COOP>
+// TAB (two-level PSA): the chunks come from the bucket-aligned chunk table, and with the
+// warp-shared descent every warp starts below its chunk's shared path.  A separate
+// instantiation: the variable start node costs registers at the 32-register cap (8 bytes of
+// spills), which the narrow bucket-aligned chunks repay and the one-level chunks do not.
+template <int F, int U, bool COOP, bool TAB = false>
 __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
@@ -838,32 +842,9 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
   const bool ps_smem = a.ps_smem_bytes != 0;
   const bool leaf_smem = a.h - 1 < a.smem_levels;
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  // chunks: fixed a.chunk-query pieces of the level-1 order, or the bucket-aligned table of
-  // the two-level PSA (entries (start, queries), <= a.chunk queries each)
-  const uint64_t nch = a.ctab ? (uint64_t)*a.nctab : (a.n + a.chunk - 1) / a.chunk;
-  for (uint64_t c = blockIdx.x; c < nch; c += gridDim.x) {
-    uint64_t c0;
-    uint32_t m;
-    if (a.ctab) {
-      const uint2 e = a.ctab[c];
-      c0 = e.x;
-      m = e.y;
-    } else {
-      c0 = c * a.chunk;
-      m = (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk);
-    }
-    uint32_t node0 = 0, lev0 = 0;
-    if (COOP && a.cbounds) {
-      // bucket b holds the keys whose bits [shift, span) equal b under the common prefix of
-      // [kmin, kmax] (C-A11); queries outside [kmin, kmax] sit in the end buckets
-      const uint2 cb = a.cbounds[c];
-      const BucketBits& f = a.bucket;
-      const uint32_t span = f.shift + (uint32_t)__popc(f.mask);
-      const uint64_t pre = span >= 64 ? 0ull : f.kmin & ~((1ull << span) - 1);
-      const uint64_t lo = cb.x <= f(f.kmin) ? 0ull : pre | ((uint64_t)cb.x << f.shift);
-      const uint64_t hi = cb.y >= f(f.kmax) ? kPad - 1 : (pre | ((uint64_t)cb.y << f.shift)) + ((1ull << f.shift) - 1);
-      chunk_path<F>(a, s_keys, s_ps, ps_smem, lo, hi, node0, lev0);
-    }
+  // one chunk: its queries in warp batches, results permuted back to level-1 order in shared
+  // memory, written contiguously
+  auto chunk = [&](uint64_t c0, uint32_t m, uint32_t node0, uint32_t lev0) {
     for (uint32_t b0 = warp * 32 * U; b0 < m; b0 += blockDim.x * U) {
       uint64_t q0[U];
       uint32_t o[U];
@@ -880,8 +861,13 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
 #endif
       }
       uint64_t res[U];
-      if constexpr (COOP) warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res, node0, lev0);
-      else lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      if constexpr (COOP && TAB) {
+        warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res, node0, lev0);
+      } else if constexpr (COOP) {
+        warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      } else {
+        lane_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
+      }
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (act[u]) s_res[o[u]] = res[u];
@@ -889,6 +875,31 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
     __syncthreads();
     for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) a.out[c0 + i] = s_res[i];
     __syncthreads();
+  };
+  if constexpr (TAB) {
+    // the bucket-aligned chunk table of the two-level PSA (entries (start, queries))
+    const uint32_t nch = *a.nctab;
+    for (uint32_t c = blockIdx.x; c < nch; c += gridDim.x) {
+      const uint2 e = a.ctab[c];
+      if constexpr (!COOP) {
+        chunk(e.x, e.y, 0, 0);
+        continue;
+      }
+      // bucket b holds the keys whose bits [shift, span) equal b under the common prefix of
+      // [kmin, kmax] (C-A11); queries outside [kmin, kmax] sit in the end buckets
+      const uint2 cb = a.cbounds[c];
+      const BucketBits& f = a.bucket;
+      const uint32_t span = f.shift + (uint32_t)__popc(f.mask);
+      const uint64_t pre = span >= 64 ? 0ull : f.kmin & ~((1ull << span) - 1);
+      const uint64_t lo = cb.x <= f(f.kmin) ? 0ull : pre | ((uint64_t)cb.x << f.shift);
+      const uint64_t hi = cb.y >= f(f.kmax) ? kPad - 1 : (pre | ((uint64_t)cb.y << f.shift)) + ((1ull << f.shift) - 1);
+      uint32_t node0, lev0;
+      chunk_path<F>(a, s_keys, s_ps, ps_smem, lo, hi, node0, lev0);
+      chunk(e.x, e.y, node0, lev0);
+    }
+  } else {  // fixed a.chunk-query chunks of the level-1 order
+    for (uint64_t c0 = (uint64_t)blockIdx.x * a.chunk; c0 < a.n; c0 += (uint64_t)gridDim.x * a.chunk)
+      chunk(c0, (uint32_t)(a.n - c0 < a.chunk ? a.n - c0 : a.chunk), 0, 0);
   }
 }
 
@@ -1299,6 +1310,9 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
   const int U = p.lane_ilp;
   auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
                      : (U >= 4 ? k_lane_search_c<F, 4, false> : (U == 2 ? k_lane_search_c<F, 2, false> : k_lane_search_c<F, 1, false>));
+  if (a.ctab)
+    kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true, true> : (U == 2 ? k_lane_search_c<F, 2, true, true> : k_lane_search_c<F, 1, true, true>))
+                  : (U >= 4 ? k_lane_search_c<F, 4, false, true> : (U == 2 ? k_lane_search_c<F, 2, false, true> : k_lane_search_c<F, 1, false, true>));
   const uint32_t smem = a.res_smem_off + a.chunk * 8;
   HM_CUDA(smem_attr(kern, smem));
   int per_sm = 0;

@@ -101,6 +101,9 @@ def _routed_update(tree_like, ops, keys, values):
     and the exchange deliver them in.  Collective: every rank calls it (possibly with 0 ops)."""
     ops_ = tree_like.ops
     group, P = tree_like.group, tree_like.world
+    if P == 1:  # one shard: the batch applies in place, in batch order (C-A18)
+        ops_.update(ops, keys, values, None)
+        return
     # all shards accept the batch or all reject it: every rank's ops are validated before any
     # is routed, the verdict is all-reduced, and every rank raises the same error (ADVICE r1)
     flag = ops_.validate_update(ops, keys, values).to(torch.int32)
@@ -185,6 +188,8 @@ class PartitionedTree:
     # ------------------------------------------------------------------ point queries
     def search(self, q: torch.Tensor) -> torch.Tensor:
         P = self.world
+        if P == 1:  # one shard: nothing to route (no partition pass, no exchange, no scatter)
+            return self.ops.search(q)
         routed, pos, counts = self.ops.route(q)              # destination-major grouping
         dev = q.device
         send = torch.tensor(counts, dtype=torch.int64, device=dev)
@@ -213,6 +218,8 @@ class PartitionedTree:
         values [n, cap] uint64, counts [n] = true totals); slab entries past the count hold
         PAD / NOT_FOUND."""
         n, dev = lo.numel(), lo.device
+        if self.world == 1:
+            return self.ops.range(lo, hi, cap)
         plo, phi, pid, send_n, pbase = self.ops.range_split(lo, hi)   # kernels: cut + dest-major
         recv_counts = torch.empty(self.world, dtype=torch.int64, device=dev)
         dist.all_to_all_single(recv_counts, torch.tensor(send_n, dtype=torch.int64, device=dev), group=self.group)

@@ -25,3 +25,25 @@ def test_no_psa_and_unstaged_levels():
         min(1000 * 544, 2081 * 512) + min(1000 * 544, 133153 * 1024)
     assert got == expect
     assert noreuse == 16 + 4 * 544
+
+
+def test_c2_step_model_by_hand():
+    """SURVEY §8(d) step model on c2: levels 0-1 in shared memory; level 2 (2081 x 512 B) and
+    the leaves with their values (133153 x 1024 B) fit the 126.5 MiB L2 (+5 %): L2 tier."""
+    plan = {"smem_levels": 2}
+    m = bench.step_model(INFO, plan, NW, 132644864, 6538.0, 17775.2, psa=True)
+    assert m["B_hbm"] == 16 + 72
+    assert m["B_l2"] == 88 + 2 * (512 + 32)
+    assert m["l2_tier_levels"] == 2 and m["hbm_tier_levels"] == 0
+    assert abs(m["bound_gqs"] - min(6538.0 / 88, 17775.2 / 1176)) < 1e-9
+    unique = (2081 * 512 + 133153 * 1024) / NW
+    assert abs(m["reuse_aware"]["B_l2"] - (88 + unique)) < 1e-9
+    assert abs(m["reuse_aware"]["bound_gqs"] - 6538.0 / 88) < 1e-9
+
+
+def test_step_model_hbm_tier():
+    """c4 geometry (2^28 keys, F64): levels 2-3 (33 MiB) in L2, the 2 GiB leaves in HBM."""
+    info = {"fanout": 64, "height": 5, "level_start": [0, 1, 18, 1059, 67636, 4328517]}
+    m = bench.step_model(info, {"smem_levels": 2}, 1 << 27, 132644864, 6538.0, 17775.2)
+    assert m["l2_tier_levels"] == 2 and m["hbm_tier_levels"] == 1
+    assert m["B_hbm"] == 88 + 544 and m["B_l2"] == 88 + 3 * 544

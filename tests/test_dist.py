@@ -133,7 +133,8 @@ class CpuOps:
                 np.bincount(dest, minlength=self.P).tolist())
 
     def update(self, ops, keys, values, seq):
-        order = np.argsort(seq.view(torch.int64).numpy().view(np.uint64), kind="stable")
+        order = (np.arange(keys.numel()) if seq is None
+                 else np.argsort(seq.view(torch.int64).numpy().view(np.uint64), kind="stable"))
         m = self.orc.UpdateMap(self.keys, self.vals)
         m.apply(ops.numpy()[order], keys.view(torch.int64).numpy().view(np.uint64)[order],
                 values.view(torch.int64).numpy().view(np.uint64)[order])
@@ -185,7 +186,7 @@ def _worker(rank, world, port, T, cap, result_q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,cap", [(2, 16), (3, 0), (3, 64)])
+@pytest.mark.parametrize("world,cap", [(1, 16), (2, 16), (3, 0), (3, 64)])
 def test_partitioned_exchange_gloo(world, cap):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -350,7 +351,7 @@ def _update_worker(rank, world, port, T, result_q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("world", [1, 2, 3])
 def test_partitioned_update_gloo(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()

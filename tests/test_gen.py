@@ -77,3 +77,32 @@ def test_update_ops_mix():
     assert 0.04 < (ops == 1).mean() < 0.06
     ins = (ops == 0) & ~np.isin(ks, k)
     assert 0.04 < ins.mean() < 0.06
+
+
+def test_device_zipf_and_key_index_generators():
+    import torch
+
+    k = gen.uniform_keys(100003)
+    kt = torch.from_numpy(k.view(np.int64))
+    idx = torch.tensor([0, 1, 5, 100002, 77777], dtype=torch.int64)
+    assert np.array_equal(gen.keys_at_t(100003, idx).numpy().view(np.uint64), k[idx.numpy()])
+    zn = gen.zipf_queries(k, 50000, start=3)
+    zt = gen.zipf_queries_t(kt, 50000, start=3).numpy().view(np.uint64)
+    assert (zn == zt).mean() > 0.999  # equal up to last-ulp pow rounding at rank boundaries
+
+
+def test_device_update_ops():
+    import torch
+
+    T = 1 << 14
+    k = gen.uniform_keys(T)
+    ops, ks, vs = gen.update_ops_t(T, 100000, 0.05, 0.05, "cpu")
+    ops, ks = ops.numpy(), ks.numpy().view(np.uint64)
+    assert 0.04 < (ops == 1).mean() < 0.06
+    ins = (ops == 0) & ~np.isin(ks, k)
+    assert 0.04 < ins.mean() < 0.06
+    assert np.isin(ks[ops == 1], k).all()
+    # a shard: keys of [lo, hi) only
+    ops2, ks2, _ = gen.update_ops_t(T, 20000, 0.05, 0.05, "cpu", lo=4096, hi=8192)
+    kk = ks2.numpy().view(np.uint64)
+    assert (kk >= k[4096]).all() and (kk <= k[8191]).all()

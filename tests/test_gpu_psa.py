@@ -82,7 +82,7 @@ def test_auto_plan_levels(hm):
     big = gen.uniform_keys_t(1 << 27, "cuda")
     t2 = hm.Tree(big.view(torch.uint64), gen.values_for_t(big).view(torch.uint64), fanout=64)
     p = t2.plan(1 << 24)
-    assert p["psa_levels"] == 2 and p["sort_chunk"] == 8192    # 2.1M leaves: 0.49 queries per leaf
+    assert p["psa_levels"] == 2 and p["sort_chunk"] == 8192    # 2^27 keys, 2.1M leaves: 0.49 queries per leaf
 
 
 def test_two_level_skewed_batch(hm, orc):

@@ -127,3 +127,14 @@ def test_checker_rejects_mutations(orc, kind, code):
     assert t.check() == 0 and t.height >= 3
     assert t.debug_mutate(kind)
     assert t.check() == code
+
+
+def test_threaded_search_and_bulk_insert(orc):
+    """The CPU-baseline helpers: bulk insert = one insert per key; threaded search = serial."""
+    keys = gen.uniform_keys(50000)
+    vals = gen.values_for(keys)
+    t = orc.BPlusTree(16)
+    assert t.insert_many(keys, vals) == 50000 and t.check() == 0
+    q = gen.uniform_queries(keys, 20000, miss_frac=0.3)
+    assert np.array_equal(t.search(q, nthreads=4), t.search(q)) and np.array_equal(
+        t.search(q), orc.sorted_search(keys, vals, q))

@@ -25,6 +25,7 @@ METRICS = [
     "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
     "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed",
     "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+    "lts__t_sectors.sum", "lts__t_sectors_srcunit_tex.sum", "lts__t_sectors_srcunit_ltcfabric.sum",
 ]
 
 
@@ -99,26 +100,42 @@ if __name__ == "__main__":
     if a.rep:
         res["full_capture"] = full(a.rep)
     json.dump(res, open(a.out + ".json", "w"), indent=1)
-    # traffic per launch for bench.py's roofline.traffic (first capture of each kernel)
-    tr_path = os.path.join(os.path.dirname(a.out), "ncu_traffic.json")
+    # per-launch figures for bench.py's roofline (profiles/ncu_r2.json): traffic, L2 bytes,
+    # sectors per request (memory divergence), warp coherence (P:L654 fn 4)
+    tr_path = os.path.join(os.path.dirname(a.out), "ncu_r2.json")
     tr = json.load(open(tr_path)) if os.path.exists(tr_path) else {}
     for d in res.get("full_capture", []):
         k = d["kernel"].split("<")[0]
         rd = to_bytes(d.get("dram__bytes_read.sum", 0), d.get("dram__bytes_read.sum.unit", "byte"))
         wr = to_bytes(d.get("dram__bytes_write.sum", 0), d.get("dram__bytes_write.sum.unit", "byte"))
-        ent = {"dram_bytes_per_launch": rd + wr,
-               "source": os.path.basename(a.out) + ".json (ncu --set full, cold L2)"}
-        l1 = d.get("l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed")
-        if isinstance(l1, float):
-            ent["l1_wavefront_pct"] = l1
-        # speed-of-light fractions of each tier / pipe (which one binds the kernel)
-        sol = {"l2": d.get("lts__throughput.avg.pct_of_peak_sustained_elapsed"),
-               "dram": d.get("dram__throughput.avg.pct_of_peak_sustained_elapsed"),
-               "l1_lsu": l1, "issue": d.get("smsp__issue_active.avg.pct_of_peak_sustained_active")}
-        ent["sol_pct"] = {k: v for k, v in sol.items() if isinstance(v, float)}
+        # L2 traffic of the kernel = sectors its SMs (L1/TEX units) moved through L2 x 32 B
+        # (lts__t_bytes is not in this ncu's full set; cross-die fabric sectors excluded)
+        lts = float(d.get("lts__t_sectors_srcunit_tex.sum", 0) or 0) * 32.0
+        ent = {"dram_bytes": rd + wr, "lts_bytes": lts,
+               "source": os.path.basename(a.out) + ".json (ncu --set full --clock-control none, cold L2)"}
+        if a.queries_per_launch:
+            ent["dram_bytes_per_query"] = (rd + wr) / a.queries_per_launch
+            ent["lts_bytes_per_query"] = lts / a.queries_per_launch
+        sec = d.get("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum")
+        req = d.get("l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum")
+        if isinstance(sec, float) and isinstance(req, float) and req:
+            ent["sectors_per_request"] = sec / req
+        r = d.get("smsp__thread_inst_executed_per_inst_executed.ratio")
+        if isinstance(r, float):
+            ent["warp_coherence"] = r / 32.0
+        for key, m in (("branch_uniform_pct", "smsp__sass_average_branch_targets_threads_uniform.pct"),
+                       ("l1_hit_pct", "l1tex__t_sector_hit_rate.pct"), ("lts_hit_pct", "lts__t_sector_hit_rate.pct"),
+                       ("issue_active_pct", "smsp__issue_active.avg.pct_of_peak_sustained_active"),
+                       ("l1_wavefront_pct", "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed"),
+                       ("lts_pct", "lts__throughput.avg.pct_of_peak_sustained_elapsed"),
+                       ("dram_pct", "dram__throughput.avg.pct_of_peak_sustained_elapsed")):
+            v = d.get(m)
+            if isinstance(v, float):
+                ent[key] = v
         tv, tu = d.get("gpu__time_duration.sum"), d.get("gpu__time_duration.sum.unit", "nsecond")
-        if isinstance(tv, float):  # capture duration: DRAM GB/s of this launch = bytes / time
-            ent["ncu_time_s"] = tv * {"ns": 1e-9, "nsecond": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3, "msecond": 1e-3, "s": 1.0, "second": 1.0}.get(tu, 1e-9)
+        if isinstance(tv, float):
+            ent["ncu_time_s"] = tv * {"ns": 1e-9, "nsecond": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3,
+                                      "msecond": 1e-3, "s": 1.0, "second": 1.0}.get(tu, 1e-9)
         st = d.get("stall_share")
         if isinstance(st, dict) and "long_scoreboard" in st:
             ent["long_scoreboard_stall_share"] = st["long_scoreboard"]
