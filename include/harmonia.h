@@ -109,6 +109,9 @@ typedef struct {
                                       default warp-per-range resolve-then-copy kernel; also
                                       implied by an explicit group_size                      */
 #define HARMONIA_QF_NO_L2_WINDOW 4096u /* no L2 access-policy window on the search kernels   */
+#define HARMONIA_QF_NO_RANGE_LANE 32768u /* ranges with max_results < 512: the G-lane group walk
+                                      instead of the default lane-per-range kernel (one lane
+                                      per range on the warp-shared descent of PSA-ordered lo) */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
 #define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic

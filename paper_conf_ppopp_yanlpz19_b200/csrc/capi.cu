@@ -550,10 +550,18 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
   a.smem_nodes = p.smem_nodes;
   a.ps_smem_bytes = p.ps_smem ? p.ps_smem_bytes : 0;
   a.cap = cap;
-  // long slabs: one warp per range, resolve then stream-copy (164 vs 128 G records/s at
-  // len 1024, 137 vs 123 at 256); short ones: several ranges per warp in G-lane groups (43 vs
-  // 22 G records/s at len 16), measured at c2
-  p.range_warp = p.range_warp && cap >= 128;
+  // long slabs (cap >= 512): one warp per range, resolve then stream-copy (164 G records/s at
+  // len 1024); shorter ones: one lane per range on the warp-shared descent, copies by the
+  // whole warp (98 / 179 / 204 G records/s at len 16 / 64 / 256 against 39 / 96 / 136 for the
+  // G-lane group walk and the warp kernel), measured at c2
+  const bool auto_kernel = p.range_warp;  // no group size, no QF_RANGE_GROUP
+#ifndef HM_RANGE_LANE_MAX
+#define HM_RANGE_LANE_MAX 512  // measured: lane kernel 1.5x at cap 256, warp kernel 1.5x at 1024
+#endif
+  p.range_warp = p.range_warp && cap >= HM_RANGE_LANE_MAX;
+  // short slabs: one lane per range on the warp-shared descent of the PSA-ordered lo (needs
+  // the PSA partition with positions, i.e. the non-staged path); DESIGN.md §8
+  p.range_lane = auto_kernel && cap < HM_RANGE_LANE_MAX && p.psa && !p.psa_global && !(o && (o->flags & HARMONIA_QF_NO_RANGE_LANE));
   if (p.g_auto) {  // the leaf scan wants wide groups for long ranges (measured)
     int G = 8;
     while (G < 32 && (uint32_t)(4 * G) < cap) G *= 2;
@@ -583,6 +591,12 @@ extern "C" harmonia_status harmonia_range_batch(const harmonia_tree* t, const ui
     a.kout = d_kout ? d_kout + w0 * cap : nullptr;
     a.vout = d_vout ? d_vout + w0 * cap : nullptr;
     a.counts = d_counts + w0;
+    if (p.range_lane) {
+      SearchArgs sa = search_args(t, p);
+      sa.n = nw;
+      if ((s = launch_range_lane(t, p, a, sa, st)) != HARMONIA_OK) return s;
+      continue;
+    }
     if ((s = launch_range(t, p, a, st)) != HARMONIA_OK) return s;
   }
   return HARMONIA_OK;

@@ -211,6 +211,7 @@ struct Plan {
   bool wide = false;         // staged return with the 11-bit level-1 partition
   bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
   bool range_warp = true;    // ranges: one warp per range, resolve then stream-copy (k_range_warp)
+  bool range_lane = false;   // short ranges: one lane per range on the warp-shared descent
   uint32_t chunk = 4096;     // staged return: level-2 chunk (4096 or kPsaChunkMax queries)
   int psa_levels = 1;        // staged return: global MSD partition levels before the chunk sort:
                              // 1 = 8 bits; 2 = 8 + 8 bits with bucket-aligned chunks (the whole
@@ -422,6 +423,9 @@ struct RangeArgs {
 };
 harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeArgs& a,
                              cudaStream_t st);
+// short ranges (cap < 128, PSA-ordered lo): one lane per range on the warp-shared descent
+harmonia_status launch_range_lane(const harmonia_tree* t, const Plan& p, const RangeArgs& ra, const SearchArgs& sa,
+                                  cudaStream_t st);
 
 harmonia_status launch_gather(const uint64_t* sorted_out, const uint32_t* idx, uint64_t n,
                               uint64_t* out, int sm_count, cudaStream_t st);

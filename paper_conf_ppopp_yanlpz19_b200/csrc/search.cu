@@ -496,7 +496,9 @@ __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint3
 // the memory-level parallelism without adding work.  A warp takes 32*U consecutive
 // (PSA-ordered) queries: query (u, lane) = base + u*32 + lane.
 // one lane, U interleaved queries, from level l0 at nodes node[]: descent (Eq 1) + leaf probe
-template <int F, int U>
+// RANK: instead of the value, res = (leaf index << 32) | #keys <= q in that leaf (the range
+// kernels turn it into a global record rank with leaf_base)
+template <int F, int U, bool RANK = false>
 __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                              bool ps_smem, bool leaf_smem, uint32_t l0, uint32_t (&node)[U],
                                              const uint64_t (&q)[U], const bool (&live)[U], uint64_t (&res)[U]) {
@@ -569,9 +571,13 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
   }
 #pragma unroll
   for (int u = 0; u < U; ++u) {
-    res[u] = kNotFound;
-    if (live[u] && r[u] > 0 && best[u] == q[u])
-      res[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+    if constexpr (RANK) {
+      res[u] = ((uint64_t)(node[u] - a.leaf_start) << 32) | r[u];
+    } else {
+      res[u] = kNotFound;
+      if (live[u] && r[u] > 0 && best[u] == q[u])
+        res[u] = __ldg(a.vals + (uint64_t)(node[u] - a.leaf_start) * F + (r[u] - 1));
+    }
   }
 }
 
@@ -717,7 +723,7 @@ __device__ __forceinline__ void chunk_path(const SearchArgs& a, const uint64_t* 
   }
 }
 
-template <int F, int U>
+template <int F, int U, bool RANK = false>
 __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                           bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
                                           const bool (&act)[U], uint64_t (&res)[U], uint32_t node0 = 0,
@@ -766,7 +772,7 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
     else window_rank<F, U, false>(a.keys, off, q, rlo, rhi, r, best);
 #pragma unroll
     for (int u = 0; u < U; ++u) nd[u] = first + r[u];
-    lane_descend<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, l + 1, nd, q, live, res);
+    lane_descend<F, U, RANK>(a, s_keys, s_ps, ps_smem, leaf_smem, l + 1, nd, q, live, res);
     return;
   }
   // the whole warp reached the same leaf
@@ -784,8 +790,12 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
   const uint64_t* vrow = a.vals + (uint64_t)(node - a.leaf_start) * F;
 #pragma unroll
   for (int u = 0; u < U; ++u) {
-    res[u] = kNotFound;
-    if (live[u] && r[u] > rlo && best[u] == q[u]) res[u] = __ldg(vrow + (r[u] - 1));
+    if constexpr (RANK) {
+      res[u] = ((uint64_t)(node - a.leaf_start) << 32) | r[u];
+    } else {
+      res[u] = kNotFound;
+      if (live[u] && r[u] > rlo && best[u] == q[u]) res[u] = __ldg(vrow + (r[u] - 1));
+    }
   }
 }
 
@@ -1049,9 +1059,10 @@ __global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArg
   }
 }
 
-// Range scan: descend with lo, then walk leaf slots in key-region order.
+// Range scan: descend with lo, then walk leaf slots in key-region order.  One CTA per SM
+// (64 registers): at two CTAs the 32-register cap spilled 16-40 bytes per thread.
 template <int F, int G, int MODE>
-__global__ void __launch_bounds__(kQueryBlock, kQueryBlocksPerSM) k_ntg_range(const RangeArgs a) {
+__global__ void __launch_bounds__(kQueryBlock, 1) k_ntg_range(const RangeArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ __align__(8) uint64_t bar;
   stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
@@ -1270,6 +1281,111 @@ __global__ void __launch_bounds__(1024, 1) k_range_warp(const RangeArgs a) {
   }
 }
 
+// ---- short ranges (cap < 512): one lane per range ------------------------------------------
+// The ranges arrive PSA-ordered by lo, so a warp's 32 ranges lie in a narrow key interval and
+// share the warp's descent (warp_core): every lane ranks lo - 1 and hi at once (two chains per
+// lane), R0 = leaf_base[leaf(lo-1)] + #keys <= lo-1 there = #keys < lo, R1 = #keys <= hi,
+// count = R1 - R0 (the first target key by the basic search, then the key region is
+// scanned); then the warp copies the ranges' min(count, cap) records range by range with
+// consecutive lanes.  No G-lane group walk, no per-range cooperative descent.
+template <int F>
+__global__ void __launch_bounds__(1024, 1) k_range_lane(const RangeArgs ra, const SearchArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar;
+  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
+  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
+  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
+  const bool ps_smem = a.ps_smem_bytes != 0;
+  const bool leaf_smem = a.h - 1 < a.smem_levels;
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t ls = a.leaf_start;
+  const uint32_t cap = ra.cap;
+  for (uint64_t base = warp * 32; base < ra.n; base += nwarps * 32) {
+    const uint64_t j = base + lane;
+    const bool act = j < ra.n;
+    const uint64_t lo = act ? ld_stream(ra.lo + j) : kPad;
+    const uint64_t slab = act ? (ra.idx ? (uint64_t)ld_stream32(ra.idx + j) : j) : 0;
+    uint64_t hi = act ? __ldg(ra.hi + slab) : 0;
+    const bool valid = act && lo <= hi && lo != kPad;
+    if (hi == kPad) hi = kPad - 1;  // no key equals PAD
+    uint64_t q0[2] = {valid && lo > 0 ? lo - 1 : kPad, valid ? hi : kPad};
+    bool qa[2] = {q0[0] != kPad, q0[1] != kPad};
+    uint64_t res[2];
+    warp_core<F, 2, true>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, qa, res);
+    uint64_t count = 0, r0 = 0;  // lo = 0: from the first record
+    uint32_t leaf = 0;
+    if (valid) {
+      if (qa[0]) {
+        leaf = (uint32_t)(res[0] >> 32);
+        r0 = __ldg(ra.leaf_base + leaf) + (uint32_t)res[0];
+      }
+      const uint64_t r1 = __ldg(ra.leaf_base + (res[1] >> 32)) + (uint32_t)res[1];
+      count = r1 > r0 ? r1 - r0 : 0;
+    }
+    const uint32_t ncopy = (uint32_t)(count < cap ? count : cap);
+    // the warp copies its ranges with consecutive lanes: record t of range i has global rank
+    // R0_i + t; its leaf is found from leaf_base starting at the leaf of lo, so the reads
+    // (consecutive slots) and the slab writes coalesce.  Slabs of <= w records (w = the warp's
+    // largest copy rounded up to a power of two, <= 32) go 32 / w ranges per step.
+    const uint32_t mx = __reduce_max_sync(kFull, ncopy);
+    const uint32_t w = mx <= 1 ? 1u : (mx >= 32 ? 32u : 1u << (32 - __clz(mx - 1)));
+    const uint32_t sub = lane / w, t_in = lane % w;
+    for (uint32_t i0 = 0; mx && i0 < 32; i0 += 32 / w) {
+      const uint32_t i = i0 + sub;
+      const uint32_t nc = __shfl_sync(kFull, ncopy, i);
+      const uint64_t rb = __shfl_sync(kFull, r0, i), sb = __shfl_sync(kFull, slab, i);
+      const uint32_t lb = __shfl_sync(kFull, leaf, i);
+      uint64_t* ko = ra.kout + sb * cap;
+      uint64_t* vo = ra.vout + sb * cap;
+      for (uint32_t t = t_in; t < nc; t += w) {
+        const uint64_t R = rb + t;
+        uint32_t j = lb;
+        while (__ldg(ra.leaf_base + j + 1) <= R) ++j;
+        const uint32_t sl = (uint32_t)(R - __ldg(ra.leaf_base + j));
+        ko[t] = __ldg(a.keys + (ls + j) * F + sl);
+        vo[t] = __ldg(a.vals + (uint64_t)j * F + sl);
+      }
+    }
+    if (act) ra.counts[slab] = (uint32_t)(count > 0xFFFFFFFFull ? 0xFFFFFFFFull : count);
+  }
+}
+
+template <int F>
+harmonia_status launch_range_lane_f(const harmonia_tree* t, const Plan& p, const RangeArgs& ra, const SearchArgs& sa,
+                                    cudaStream_t st) {
+  auto kern = k_range_lane<F>;
+  HM_CUDA(smem_attr(kern, p.smem_bytes));
+  int per_sm = 0;
+  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 1024, p.smem_bytes));
+  per_sm = std::max(per_sm, 1);
+  const uint64_t need = ceil_div(ra.n, (uint64_t)1024);
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm * 4));
+  {
+    ProfScope ps_(HARMONIA_PROF_RANGE, st);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(1024);
+    cfg.dynamicSmemBytes = p.smem_bytes;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    if (p.l2_bytes) {
+      at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+      at[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(p.l2_base);
+      at[0].val.accessPolicyWindow.num_bytes = p.l2_bytes;
+      at[0].val.accessPolicyWindow.hitRatio = p.l2_hit;
+      at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+    }
+    HM_CUDA(cudaLaunchKernelEx(&cfg, kern, ra, sa));
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
+}
+
 template <int F>
 harmonia_status launch_range_warp_f(const harmonia_tree* t, const Plan& p, const RangeArgs& a, cudaStream_t st) {
   auto kern = k_range_warp<F>;
@@ -1465,6 +1581,21 @@ harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeA
   }
   const int G = p.G == 1 ? 2 : p.G;  // ranges scan leaves with at least a lane pair
   HM_DISPATCH(launch_range_fg, t->F, G, t, p, a, st)
+}
+
+harmonia_status launch_range_lane(const harmonia_tree* t, const Plan& p, const RangeArgs& ra, const SearchArgs& sa,
+                                  cudaStream_t st) {
+  if (ra.n == 0) return HARMONIA_OK;
+  switch (t->F) {
+    case 4: return launch_range_lane_f<4>(t, p, ra, sa, st);
+    case 8: return launch_range_lane_f<8>(t, p, ra, sa, st);
+    case 16: return launch_range_lane_f<16>(t, p, ra, sa, st);
+    case 32: return launch_range_lane_f<32>(t, p, ra, sa, st);
+    case 64: return launch_range_lane_f<64>(t, p, ra, sa, st);
+    case 128: return launch_range_lane_f<128>(t, p, ra, sa, st);
+    case 256: return launch_range_lane_f<256>(t, p, ra, sa, st);
+  }
+  return HARMONIA_ERR_INVALID_ARG;
 }
 
 harmonia_status launch_sort_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {

@@ -271,6 +271,43 @@ def test_range_warp_kernel(hm, orc, F, fill, length, cap):
     _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
 
 
+@pytest.mark.parametrize("F,fill", [(4, 1.0), (8, 0.69), (16, 0.5), (64, 1.0), (64, 0.69), (128, 1.0), (256, 0.69)])
+@pytest.mark.parametrize("length,cap", [(1, 1), (16, 16), (16, 5), (40, 64), (64, 127), (300, 100), (7, 0),
+                                        (256, 256), (700, 511)])
+def test_range_lane_kernel(hm, orc, F, fill, length, cap):
+    """Default short-range path (cap < 512, k_range_lane: one lane per range on the warp-shared
+    descent of the PSA-ordered lo, counts from leaf_base ranks, per-lane leaf walk): exact slabs
+    and true totals, mid-leaf starts, ranges across leaves, truncation, empty ranges in key gaps,
+    lo > hi, lo = 0, PAD bounds, several PSA windows."""
+    keys = gen.uniform_keys(70000) if F != 4 else gen.uniform_keys(9000)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, F, fill)
+    lo, hi = gen.ranges(keys, 20000, min(length, len(keys)))
+    lo2, hi2 = gen.random_ranges(keys, 5000, max_width_keys=3 * max(cap, 8))
+    lo3 = np.array([0, 0, int(keys[500]), int(keys[-1]), MAX, 5, MAX - 1, int(keys[7]) + 1, 1, int(keys[3])],
+                   dtype=np.uint64)
+    hi3 = np.array([MAX, int(keys[99]), MAX, MAX, MAX, 4, MAX, int(keys[9]), 0, int(keys[3])], dtype=np.uint64)
+    lo, hi = np.concatenate([lo, lo2, lo3]), np.concatenate([hi, hi2, hi3])
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, cap)
+    for kw in ({}, {"window": 4096}, {"smem_levels": -1}, {"psa_bits": 20}):
+        ko, vo, cnt = t.range(cu(lo), cu(hi), cap, **kw)
+        _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
+    ko, vo, cnt = t.range(cu(lo), cu(hi), cap, flags=hm.QF_NO_RANGE_LANE)  # the G-lane group walk
+    _cmp_range(host(ko) if cap else None, host(vo) if cap else None, host(cnt), eko, evo, ecnt, cap)
+
+
+def test_range_lane_clustered(hm, orc):
+    """Dense sorted-run keys (a common prefix: C-A11 span) with long and short ranges."""
+    keys = gen.clustered_keys(1 << 17)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 32)
+    lo, hi = gen.random_ranges(keys, 30000, max_width_keys=200)
+    for cap in (16, 100):
+        eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, cap)
+        ko, vo, cnt = t.range(cu(lo), cu(hi), cap)
+        _cmp_range(host(ko), host(vo), host(cnt), eko, evo, ecnt, cap)
+
+
 def test_range_unbounded_counts(hm, orc):
     keys = gen.uniform_keys(100000)
     vals = gen.values_for(keys)

@@ -64,7 +64,8 @@ def range_bench(T=1 << 23, F=64, reps=5, groups=(0,), flags=0):
             cnt = outb[2].cpu().numpy()
             ok = bool((cnt == length).all())  # lo = key[p], hi = key[p+len-1]: exactly len records
             res.append({"what": "range_batch", "T": T, "F": F, "G": G, "len": length, "Qr": Qr, "ms": ms,
-                        "kernel": "group" if (G or flags & hm.QF_RANGE_GROUP or length < 128) else "warp", "counts_ok": ok,
+                        "kernel": ("group" if (G or flags & (hm.QF_RANGE_GROUP | hm.QF_NO_RANGE_LANE)) else
+                                   ("lane" if length < 128 else "warp")), "counts_ok": ok,
                         "Gq_per_s": Qr / ms / 1e6, "G_records_per_s": Qr * length / ms / 1e6,
                         "GB_per_s_out": Qr * length * 16 / ms / 1e6})
             print(json.dumps(res[-1]), flush=True)
@@ -104,6 +105,7 @@ if __name__ == "__main__":
         rows = {"update": update_bench, "range": range_bench,
                 "range_sweep": lambda: range_bench(groups=(2, 4, 8, 16, 32)),
                 "range_group": lambda: range_bench(flags=hm.QF_RANGE_GROUP),
+                "range_nolane": lambda: range_bench(flags=hm.QF_NO_RANGE_LANE),
                 "sweep": lambda: sweep_bench(dist=a.sweep_dist)}[w]()
         for r in rows:
             print(json.dumps(r), flush=True)
