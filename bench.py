@@ -68,6 +68,7 @@ def parse():
     ap.add_argument("--mode", default="replicated", choices=["replicated", "partitioned", "peer"])
     ap.add_argument("--sweep", default="", help="comma list of k=v option sets separated by ';' (diagnostics)")
     ap.add_argument("--no-extra", action="store_true", help="skip the c4 / c3-fanout extra lines (default run)")
+    ap.add_argument("--slices", type=int, default=4, help="partitioned mode: exchange/search overlap slices")
     ap.add_argument("--extra-steps", type=int, default=10)
     return ap.parse_args()
 
@@ -605,6 +606,11 @@ def main():
         pt = cls(torch.from_numpy(lk).to(dev), torch.from_numpy(lv).to(dev), sp, fanout=c["F"], fill=a.fill,
                  device=dev)
         t = pt.ops.tree
+    elif world > 1:  # replicated mode: the same layout on every rank, no collective on the hot path
+        from paper_conf_ppopp_yanlpz19_b200.dist import ReplicatedTree
+
+        t = ReplicatedTree(torch.from_numpy(keys).to(dev), torch.from_numpy(vals).to(dev), fanout=c["F"],
+                           fill=a.fill).tree
     else:
         t = hm.Tree(torch.from_numpy(keys).to(dev), torch.from_numpy(vals).to(dev), fanout=c["F"], fill=a.fill)
     info = t.info()
@@ -616,7 +622,7 @@ def main():
 
     def step():
         if pt is not None:
-            out.copy_(pt.search(q))
+            out.copy_(pt.search(q, slices=a.slices) if a.mode == "partitioned" else pt.search(q))
         else:
             t.search(q, out, opts=opts)
 

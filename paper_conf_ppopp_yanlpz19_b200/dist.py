@@ -186,10 +186,17 @@ class PartitionedTree:
         self.splitters = list(splitters)
 
     # ------------------------------------------------------------------ point queries
-    def search(self, q: torch.Tensor) -> torch.Tensor:
+    def search(self, q: torch.Tensor, slices: int = 1) -> torch.Tensor:
+        """Point queries routed to their shards.  slices > 1 splits the batch so that the
+        exchange of slice i+1 overlaps the local search of slice i: every
+        slice is routed on the caller's stream, its query all-to-all is asynchronous, the
+        search runs on a side stream once the exchange has landed, and the results go back
+        slice by slice (collectives are issued in the same order on every rank)."""
         P = self.world
         if P == 1:  # one shard: nothing to route (no partition pass, no exchange, no scatter)
             return self.ops.search(q)
+        if slices > 1 and q.numel() >= slices:
+            return self._search_sliced(q, slices)
         routed, pos, counts = self.ops.route(q)              # destination-major grouping
         dev = q.device
         send = torch.tensor(counts, dtype=torch.int64, device=dev)
@@ -204,6 +211,48 @@ class PartitionedTree:
         dist.all_to_all_single(back, _i64(vals), output_split_sizes=counts, input_split_sizes=rc,
                                group=self.group)               # C5: return values
         return self.ops.scatter(_u64(back), pos)               # caller's order
+
+    def _search_sliced(self, q, slices):
+        import contextlib
+
+        dev = q.device
+        cuda = dev.type == "cuda"
+        side = torch.cuda.Stream(dev) if cuda else None
+        main = torch.cuda.current_stream(dev) if cuda else None
+        n = q.numel()
+        cuts = [(n * i) // slices for i in range(slices + 1)]
+        pending = []  # (recv handle, recv buffer, counts, rc, pos, lo, hi)
+        for i in range(slices):  # route + exchange every slice; searches start as exchanges land
+            qs = q[cuts[i]:cuts[i + 1]]
+            routed, pos, counts = self.ops.route(qs)
+            send = torch.tensor(counts, dtype=torch.int64, device=dev)
+            recv = torch.empty(self.world, dtype=torch.int64, device=dev)
+            dist.all_to_all_single(recv, send, group=self.group)
+            rc = recv.tolist()
+            recv_q = torch.empty(sum(rc), dtype=torch.int64, device=dev)
+            work = dist.all_to_all_single(recv_q, _i64(routed), output_split_sizes=rc, input_split_sizes=counts,
+                                          group=self.group, async_op=True)
+            pending.append((work, recv_q, counts, rc, pos, cuts[i], cuts[i + 1], routed))
+        out = torch.empty(n, dtype=q.dtype, device=dev)
+        results = []
+        for work, recv_q, counts, rc, pos, lo, hi, routed in pending:
+            with (torch.cuda.stream(side) if cuda else contextlib.nullcontext()):
+                work.wait()                                    # this slice's queries have landed
+                vals = self.ops.search(_u64(recv_q))
+                ev = torch.cuda.Event() if cuda else None
+                if cuda:
+                    ev.record(side)
+                    recv_q.record_stream(side)
+            results.append((vals, ev, counts, rc, pos, lo, hi))
+        for vals, ev, counts, rc, pos, lo, hi in results:
+            if cuda:
+                main.wait_event(ev)
+                vals.record_stream(main)
+            back = torch.empty(hi - lo, dtype=torch.int64, device=dev)
+            dist.all_to_all_single(back, _i64(vals), output_split_sizes=counts, input_split_sizes=rc,
+                                   group=self.group)
+            out[lo:hi] = self.ops.scatter(_u64(back), pos)
+        return out
 
     # ------------------------------------------------------------------ updates
     def update(self, ops, keys, values):

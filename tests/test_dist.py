@@ -163,6 +163,9 @@ def _worker(rank, world, port, T, cap, result_q):
         got = pt.search(qt).view(torch.int64).numpy().view(np.uint64)
         exp = oracle.sorted_search(keys, vals, q)
         ok_pts = bool(np.array_equal(got, exp))
+        # the sliced exchange (slice i+1 in flight while slice i is searched) gives the same
+        got3 = pt.search(qt, slices=3).view(torch.int64).numpy().view(np.uint64)
+        ok_pts = ok_pts and bool(np.array_equal(got3, exp))
         # ranges: short, long (crossing several shards), empty, lo > hi, full span
         lo1, hi1 = gen.ranges(keys, 200, 40, seed=gen.SEED_RANGE + rank)
         lo2, hi2 = gen.random_ranges(keys, 200, seed=gen.SEED_RANGE + 7 * rank, max_width_keys=T)
