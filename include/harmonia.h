@@ -92,28 +92,28 @@ typedef struct {
 #define HARMONIA_QF_GATHER     2u  /* PSA return via a separate gather pass instead of the
                                       search kernel scattering results in place             */
 #define HARMONIA_QF_ILP1       16u /* k-ary search with one query per lane group instead of two */
-#define HARMONIA_QF_FUSE_SORT 128u /* G = 1: PSA chunk sort fused into the search kernel
-                                      (ablation; measured slower than two kernels)          */
+/* 64, 128, 512: ablations of ABI 1 removed in ABI 2 (LSD chunk sort, fused chunk sort + search,
+ * 11-bit level-1 partition; all measured slower).  Set, they are INVALID_ARG. */
+#define HARMONIA_QF_REMOVED_PSA_LSD   64u
+#define HARMONIA_QF_REMOVED_FUSE_SORT 128u
+#define HARMONIA_QF_REMOVED_PSA_WIDE  512u
 #define HARMONIA_QF_SCATTER_RETURN 256u /* G = 1 PSA path: the search scatters results to
                                       out[original position] instead of the default staged
                                       return (chunk-local smem permutation + k_psa2_unmove) */
-#define HARMONIA_QF_PSA_WIDE 512u /* staged return with an 11-bit (2048-bin) level-1 partition
-                                      instead of the default 8-bit one (ablation: denser
-                                      chunks for the search, but 2-query runs in the moves)  */
 #define HARMONIA_QF_PER_LANE 1024u /* G = 1 PSA path: every lane descends on its own instead of
                                       the default warp-shared descent (the warp's PSA-ordered
                                       queries share the path down to the level where their
                                       key interval splits)                           */
 #define HARMONIA_QF_RANGE_GROUP 2048u /* ranges: the G-lane group walk of the leaves (one
                                       load-ballot-store step per 2G slots) instead of the
-                                      default warp-per-range resolve-then-copy kernel; also
-                                      implied by an explicit group_size                      */
+                                      default lane-per-range (max_results < 512) or
+                                      warp-per-range kernel; also implied by an explicit
+                                      group_size                                             */
 #define HARMONIA_QF_NO_L2_WINDOW 4096u /* no L2 access-policy window on the search kernels   */
 #define HARMONIA_QF_NO_RANGE_LANE 32768u /* ranges with max_results < 512: the G-lane group walk
                                       instead of the default lane-per-range kernel (one lane
                                       per range on the warp-shared descent of PSA-ordered lo) */
 #define HARMONIA_QF_PSA_COARSE 32u /* PSA level 1 only (8-bit coarse partition, no chunk sort) */
-#define HARMONIA_QF_PSA_LSD    64u /* chunk sort by two ballot-multisplit LSD passes        */
 #define HARMONIA_QF_PSA_GLOBAL 8u  /* PSA as one global pass over all 2^Nb buckets (one atomic
                                       per query) instead of the default two-level partition  */
 #define HARMONIA_QF_PSA_L16 8192u /* staged-return PSA: force two MSD levels (8 + 8 bits) and

@@ -25,10 +25,7 @@ QF_LINEAR = 4
 QF_PSA_GLOBAL = 8
 QF_ILP1 = 16
 QF_PSA_COARSE = 32
-QF_PSA_LSD = 64
-QF_FUSE_SORT = 128
 QF_SCATTER_RETURN = 256
-QF_PSA_WIDE = 512
 QF_NO_L2_WINDOW = 4096
 QF_PER_LANE = 1024
 QF_RANGE_GROUP = 2048

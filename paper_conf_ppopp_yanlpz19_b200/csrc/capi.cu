@@ -74,8 +74,11 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
 #define HM_LANE_ILP 2
 #endif
   P.lane_ilp = o->lane_queries ? (int)o->lane_queries : HM_LANE_ILP;
-  P.psa_level2 = (o->flags & HARMONIA_QF_PSA_COARSE) ? 2 : ((o->flags & HARMONIA_QF_PSA_LSD) ? 1 : 0);
-  P.fuse = (o->flags & HARMONIA_QF_FUSE_SORT) != 0;  // measured slower
+  // flag bits of removed ablations (ABI 1: fused chunk sort, LSD chunk sort, 11-bit level 1;
+  // all measured slower) are rejected
+  if (o->flags & (HARMONIA_QF_REMOVED_FUSE_SORT | HARMONIA_QF_REMOVED_PSA_LSD | HARMONIA_QF_REMOVED_PSA_WIDE))
+    return HARMONIA_ERR_INVALID_ARG;
+  P.psa_level2 = (o->flags & HARMONIA_QF_PSA_COARSE) ? 2 : 0;
   P.psa_global = (o->flags & HARMONIA_QF_PSA_GLOBAL) != 0;
   // ---- shared-memory staging plan: PS first (P:L272 keeps the PS top on chip), then the
   // top levels in BFS order while they fit
@@ -110,7 +113,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   P.ret = P.psa && P.G == 1 && !P.psa_global && P.psa_level2 == 0 && !P.gather &&
           !(o->flags & HARMONIA_QF_SCATTER_RETURN) &&
           2 * (round_up(P.smem_bytes, 16) + P.chunk * 8 + 1024) <= t->smem_per_sm;
-  if (!P.ret || P.fuse) P.chunk = kPsaChunk;
+  if (!P.ret) P.chunk = kPsaChunk;
   // L2 access-policy window over the internal levels below the staged top (north_star (c):
   // the upper levels are pinned in L2 while leaves, values and query streams pass through)
   if (HM_L2_WINDOW && !(o->flags & HARMONIA_QF_NO_L2_WINDOW) && t->l2_window_max && t->l2_persist_max && t->h > 1 &&
@@ -135,7 +138,7 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
   // 4096 x 256 / leaves queries per leaf (c2 63, 2^26 keys 0.98 -> one level; 2^28 keys 0.25
   // -> two levels: search 4.5 -> 2.1 ms, step 6.65 -> 6.19 ms).
   P.psa_levels = 1;
-  if (P.ret && P.nb >= 16 && !(o->flags & HARMONIA_QF_PSA_WIDE) && !(o->flags & HARMONIA_QF_PSA_L8)) {
+  if (P.ret && P.nb >= 16 && !(o->flags & HARMONIA_QF_PSA_L8)) {
     const double dens = t->L ? (double)kPsaChunk * 256.0 / (double)t->L : 1e9;
     // and only for trees far beyond L2 (>= 2^27 keys): with 2^26 keys a Zipf batch (c3) lost
     // 30 % with two levels, uniform ones broke even
@@ -149,7 +152,6 @@ harmonia_status make_plan(const harmonia_tree* t, uint64_t n, const harmonia_que
     const double fit = (double)P.chunk / (mean + 4.0 * std::sqrt(mean) + 8.0);
     P.l2_group = (uint32_t)std::max(1.0, std::min(fit, (double)kL2Buckets));
   }
-  P.wide = P.ret && P.nb > 8 && (o->flags & HARMONIA_QF_PSA_WIDE);
   P.coop = P.ret && !(o->flags & HARMONIA_QF_PER_LANE);
   // ranges: the warp-per-range copy kernel unless a group size was requested explicitly or
   // the G-lane group walk is asked for (HARMONIA_QF_RANGE_GROUP)
@@ -254,23 +256,14 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
   const PsaWs w = psa_ws_carve(p, ws);
   for (uint64_t w0 = 0; w0 < n; w0 += p.window) {
     const uint64_t nw = std::min<uint64_t>(p.window, n - w0);
-    const bool fused = p.fuse && p.G == 1 && !p.psa_global && p.psa_level2 == 0 && !p.gather &&
-                       p.smem_bytes + (8u << 10) + (48u << 10) <= t->smem_optin;
     harmonia_status s = HARMONIA_OK;
     if (!p.ret) {
       s = p.psa_global ? psa_partition(q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr)
-                       : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : p.psa_level2);
+                       : psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.psa_level2);
       if (s != HARMONIA_OK) return s;
     }
     a.q = w.sorted_q;
     a.n = nw;
-    if (fused && !p.ret) {  // level-2 chunk sort inside the search kernel
-      a.idx = w.idx;
-      a.out = out + w0;
-      a.bucket = p.bucket;
-      if ((s = launch_sort_search(t, p, a, st)) != HARMONIA_OK) return s;
-      continue;
-    }
     if (p.ret && p.psa_levels == 2) {  // two MSD levels + bucket-aligned chunks
       if ((s = psa_partition2_l2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.l2_group, p.chunk)) != HARMONIA_OK)
         return s;
@@ -292,7 +285,7 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       continue;
     }
     if (p.ret) {  // staged return: level-1-order results, then the inverse move
-      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, fused ? 2 : 0, true, p.wide, p.chunk);
+      s = psa_partition2(q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, 0, true, p.chunk);
       if (s != HARMONIA_OK) return s;
       a.idx = w.idx;
       a.out = w.sorted_out;
@@ -300,10 +293,10 @@ static harmonia_status search_device(const harmonia_tree* t, const uint64_t* q, 
       a.res_smem_off = (uint32_t)round_up(p.smem_bytes, 16);
       a.chunk = p.chunk;
       a.bucket = p.bucket;
-      a.cbounds = fused ? nullptr : w.cbounds;
-      if ((s = fused ? launch_sort_search(t, p, a, st) : launch_search(t, p, a, st)) != HARMONIA_OK) return s;
+      a.cbounds = w.cbounds;
+      if ((s = launch_search(t, p, a, st)) != HARMONIA_OK) return s;
       a.cbounds = nullptr;
-      if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, t->sm_count, st, p.wide)) != HARMONIA_OK) return s;
+      if ((s = psa_unpartition2(w, w.sorted_out, nw, out + w0, t->sm_count, st)) != HARMONIA_OK) return s;
       continue;
     }
     if (p.gather) {
@@ -423,8 +416,8 @@ extern "C" harmonia_status harmonia_psa_inspect(const harmonia_tree* t, const ui
       continue;
     }
     if (p.psa_global) s = psa_partition(d_q + w0, nw, p.bucket, p.nbins, w, t->sm_count, st, nullptr);
-    else if (p.ret) s = psa_partition2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, 0, true, p.wide, p.chunk);
-    else s = psa_partition2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.fuse ? 2 : p.psa_level2);
+    else if (p.ret) s = psa_partition2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, 0, true, p.chunk);
+    else s = psa_partition2(d_q + w0, nw, p.bucket, p.nb, w, t->sm_count, st, p.psa_level2);
     if (s != HARMONIA_OK) return s;
     HM_CUDA(cudaMemcpyAsync(d_order_out + w0, w.sorted_q, nw * 8, cudaMemcpyDeviceToDevice, st));
   }

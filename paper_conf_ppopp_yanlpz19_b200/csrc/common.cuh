@@ -204,11 +204,9 @@ struct Plan {
   int kary = 1;              // in-node search: 1 = k-ary NTG, 0 = linear NTG (Fig 9)
   bool ilp2 = true;          // k-ary: two queries per lane group (k_ntg_search2)
   int lane_ilp = 2;          // G = 1: queries interleaved per lane (k_lane_search_u)
-  int psa_level2 = 0;        // chunk sort: 0 counting, 1 ballot LSD, 2 none (coarse only)
-  bool fuse = false;         // G = 1 + counting chunk sort fused into the search (k_sort_search)
+  int psa_level2 = 0;        // chunk sort: 0 counting, 2 none (coarse only, ablation)
   bool psa_global = false;   // one-pass Eq-2 partition with global atomics (ablation)
   bool ret = false;          // staged inverse return (chunk-local result staging + unmove)
-  bool wide = false;         // staged return with the 11-bit level-1 partition
   bool coop = false;         // G = 1 PSA path: warp-shared descent (k_lane_search_c<.., true>)
   bool range_warp = true;    // ranges: one warp per range, resolve then stream-copy (k_range_warp)
   bool range_lane = false;   // short ranges: one lane per range on the warp-shared descent
@@ -335,7 +333,7 @@ struct SearchArgs {
   const uint32_t* idx;     // original position within the window (nullptr = identity)
   uint64_t n;
   uint64_t* out;           // results: out[idx ? idx[j] : j]
-  BucketBits bucket;       // PSA bucket (fused level-2 sort only)
+  BucketBits bucket;       // PSA bucket (two-level PSA: the chunks' key intervals)
   uint32_t staged;         // staged return: idx holds chunk-local level-1 offsets and results
                            // go through shared memory (at dynamic-smem offset res_smem_off)
                            // to out[] in level-1 order, chunk by chunk (kPsaChunk)
@@ -350,14 +348,12 @@ struct SearchArgs {
   uint32_t cshift;
   uint64_t kmin, kmax;
 };
-harmonia_status launch_sort_search(const harmonia_tree* t, const struct Plan& p, const SearchArgs& a,
-                                   cudaStream_t st);
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws,
                                int sm_count, cudaStream_t st, int level2 = 0, bool local = false,
-                               bool wide = false, uint32_t chunk = kPsaChunk);
+                               uint32_t chunk = kPsaChunk);
 // inverse of the level-1 move for the staged return: out[e] = res1[level-1 position of e]
 harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
-                                 cudaStream_t st, bool wide);
+                                 cudaStream_t st);
 // two-level PSA (Plan::psa_levels == 2): partition into ws.sorted2 (chunk table ws.chunks),
 // and the inverse from level-2-order results; psa_compact_l2 = the chunks without padding
 harmonia_status psa_partition2_l2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,

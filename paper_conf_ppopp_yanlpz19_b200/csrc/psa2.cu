@@ -1,18 +1,19 @@
-// Two-level partially-sorted aggregation (default PSA path).
+// Partially-sorted aggregation (PSA, §4.1) as MSD partition passes.
 //
 // "the queries will be sorted based on their most significant N bits", N from
 // Eq 2.  On sm_100a a one-pass partition over 2^N buckets costs one global atomic per query
-// and shared-memory atomics cost ~2 cycles per lane, so the N-bit order is built in two
-// atomic-free levels:
-//   level 1  coarse MSB partition of the PSA window on the top kCoarseBits bits of the
-//            N-bit bucket: warp multisplit by ballots (rank = popc(peers & lanemask_lt)),
-//            per-warp counters, one global atomic per (tile, bin), tile staged in shared
-//            memory so that every bin's run is written with consecutive lanes;
-//   level 2  every kChunk-sized chunk of that order is sorted by its full N-bit bucket
-//            (offset by the chunk minimum, capped at kLocalBits bits) with two stable LSD
-//            passes of the same ballot multisplit, entirely in shared memory.
-// The result orders each chunk by the top-N bits and the chunks by the top-8 bits, which is
-// the paper's partial sort at chunk granularity; order inside a bucket is free (C-A12).
+// (the one-pass form is kept in psa.cu as the literal ablation), so the N-bit order is built
+// from shared-memory passes:
+//   level 1  MSB partition of the PSA window on the top 8 bits of the N-bit bucket: a rank
+//            pass (digit + rank in the 2048-query tile by one shared-memory atomic), then a
+//            move pass that stages each tile in digit order so that every bin's run is
+//            written by consecutive lanes; persistent CTAs reserve bin space once per bin;
+//   level 2  (psa_levels = 2, large trees) the same rank + move on the next 8 bits inside
+//            every level-1 segment, tile bases from per-segment column scans;
+//   chunk    every 4096/8192-query chunk of that order (bucket-aligned chunks after level 2)
+//            is counting-sorted by its full N-bit bucket in shared memory.
+// One level orders each chunk by all N bits and the chunks by the top 8 bits; two levels
+// order the whole window.  Order inside a bucket is free (C-A12).
 #include <algorithm>
 
 #include <type_traits>
@@ -45,33 +46,13 @@ constexpr int kCoarseTile = kBlock * kBatches;           // 2048 queries per sca
 #define HM_SORT_THREADS 512
 #endif
 constexpr int kSortThreads = HM_SORT_THREADS, kSortWarps = kSortThreads / 32;
-constexpr int kChunk = (int)kPsaChunk;                   // queries per LSD local-sort chunk (4096)
-constexpr int kSortBatches = kChunk / kSortThreads;      // 32-query batches per warp per chunk
-static_assert(kChunk == kSortThreads * kSortBatches, "chunk = threads x batches");
-constexpr int kLocalBits = 11, kLoBits = 6, kHiBits = kLocalBits - kLoBits;
-constexpr size_t kSortSmem = (size_t)kChunk * (8 + 4 + 2);  // keys, positions, local digits
+constexpr int kChunk = (int)kPsaChunk;                   // queries per chunk-sort chunk (4096)
+constexpr int kLocalBits = 11;                           // chunk sort: 2048 local buckets
 
 __device__ __forceinline__ unsigned lane_lt() {
   unsigned m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
   return m;
-}
-
-// lanes of the warp whose digit equals mine (BITS-bit digits), restricted to `valid`
-template <int BITS>
-__device__ __forceinline__ unsigned peers_of(uint32_t d, unsigned valid) {
-#ifndef HARMONIA_MATCH_ANY  // measured: BITS ballots beat one MATCH.ANY on sm_100a
-  unsigned m = valid;
-#pragma unroll
-  for (int b = 0; b < BITS; ++b) {
-    const bool bit = (d >> b) & 1u;
-    const unsigned bb = __ballot_sync(kFull, bit);
-    m &= bit ? bb : ~bb;
-  }
-  return m;
-#else
-  return __match_any_sync(kFull, d) & valid;  // one MATCH.ANY instead of BITS ballots
-#endif
 }
 
 // exclusive scan of one value per thread (NT threads); `tmp` needs NT/32 + 1 words
@@ -113,9 +94,9 @@ struct CoarseDigit {
 
 // ---- level-1 configurations -------------------------------------------------------------
 // BITS-bit coarse digit, TILE queries per tile, NT threads per CTA (PER = TILE / NT queries
-// per thread).  Narrow: 256 bins -- the multi-GPU router and the non-staged PSA modes.  Wide:
-// 2048 bins -- the default staged-return PSA: a 4096-query level-2 chunk then spans ~2
-// coarse bins instead of 1/8 of one, so the search sees ~8x denser key ranges per warp.
+// per thread).  Narrow: 256 bins, 2048-query tiles (runs of ~8 queries per bin): the PSA levels
+// and the multi-GPU router.  (An 11-bit level with 4096-query tiles was measured slower: its
+// 2-query runs made the moves 3x slower.)
 template <int BITS_, int TILE_, int NT_>
 struct L1Cfg {
   static constexpr int BITS = BITS_, BINS = 1 << BITS_, TILE = TILE_, NT = NT_, PER = TILE_ / NT_;
@@ -132,10 +113,6 @@ struct L1Cfg {
 #define HM_NARROW_NT 256
 #endif
 using Narrow = L1Cfg<8, HM_NARROW_TILE, HM_NARROW_NT>;
-#ifndef HM_WIDE_TILE
-#define HM_WIDE_TILE 4096
-#endif
-using Wide = L1Cfg<11, HM_WIDE_TILE, 512>;
 
 // exclusive scan over C::BINS values held BPT per thread (thread t owns [t*BPT, t*BPT+BPT))
 template <class C>
@@ -767,122 +744,6 @@ __global__ void __launch_bounds__(256) k_l2_compact(const uint64_t* __restrict__
   }
 }
 
-// ---- level 2: chunk-local sort by the N-bit bucket (two stable LSD passes) ---------------
-template <int BITS, int SHIFT>
-__device__ __forceinline__ void lsd_pass(uint64_t (&v)[kSortBatches], uint32_t (&ix)[kSortBatches], uint32_t (&lk)[kSortBatches],
-                                         uint32_t m, uint32_t (*wcnt)[1 << kLoBits], uint32_t* bin_start, uint32_t* tmp,
-                                         uint64_t* s_q, uint32_t* s_i, uint16_t* s_k) {
-  constexpr int NB = 1 << BITS;
-  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (int i = threadIdx.x; i < kSortWarps * NB; i += kSortThreads) wcnt[i / NB][i % NB] = 0;
-  __syncthreads();
-  uint32_t pos[kSortBatches], dg[kSortBatches];
-#pragma unroll
-  for (int k = 0; k < kSortBatches; ++k) {  // element order = (warp, batch, lane): stable ranks
-    const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
-    const bool valid = e < m;
-    dg[k] = (lk[k] >> SHIFT) & (NB - 1);
-    const unsigned peers = peers_of<BITS>(dg[k], __ballot_sync(kFull, valid));
-    const uint32_t run = valid ? wcnt[warp][dg[k]] : 0u;
-    __syncwarp();
-    if (valid && lane == (unsigned)(__ffs(peers) - 1)) wcnt[warp][dg[k]] = run + __popc(peers);
-    __syncwarp();
-    pos[k] = run + __popc(peers & lane_lt());
-  }
-  __syncthreads();
-  uint32_t acc = 0;
-  if (threadIdx.x < NB) {
-#pragma unroll
-    for (int w = 0; w < kSortWarps; ++w) {
-      const uint32_t c = wcnt[w][threadIdx.x];
-      wcnt[w][threadIdx.x] = acc;
-      acc += c;
-    }
-  }
-  const uint32_t bs = block_scan<kSortThreads>(threadIdx.x < NB ? acc : 0u, tmp, nullptr);
-  if (threadIdx.x < NB) bin_start[threadIdx.x] = bs;
-  __syncthreads();
-#pragma unroll
-  for (int k = 0; k < kSortBatches; ++k) {
-    const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
-    if (e < m) {
-      const uint32_t dst = bin_start[dg[k]] + wcnt[warp][dg[k]] + pos[k];
-      s_q[dst] = v[k];
-      s_i[dst] = ix[k];
-      s_k[dst] = (uint16_t)lk[k];
-    }
-  }
-  __syncthreads();
-#pragma unroll
-  for (int k = 0; k < kSortBatches; ++k) {  // reload in the new order for the next pass
-    const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
-    if (e < m) {
-      v[k] = s_q[e];
-      ix[k] = s_i[e];
-      lk[k] = s_k[e];
-    }
-  }
-  __syncthreads();
-}
-
-__global__ void __launch_bounds__(kSortThreads, 2) k_psa2_local_sort(uint64_t* __restrict__ sorted_q,
-                                                                  uint32_t* __restrict__ idx, uint64_t n, BucketBits f) {
-  extern __shared__ __align__(16) unsigned char sm[];
-  uint64_t* s_q = reinterpret_cast<uint64_t*>(sm);
-  uint32_t* s_i = reinterpret_cast<uint32_t*>(sm + kChunk * 8);
-  uint16_t* s_k = reinterpret_cast<uint16_t*>(sm + kChunk * 12);
-  __shared__ uint32_t wcnt[kSortWarps][1 << kLoBits];
-  __shared__ uint32_t bin_start[1 << kLoBits], tmp[kSortWarps + 1], s_mm[2][kSortWarps];
-  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t c0 = (uint64_t)blockIdx.x * kChunk; c0 < n; c0 += (uint64_t)gridDim.x * kChunk) {
-    const uint32_t m = (uint32_t)std::min<uint64_t>(kChunk, n - c0);
-    uint64_t v[kSortBatches];
-    uint32_t ix[kSortBatches], lk[kSortBatches];
-    uint32_t bmin = 0xFFFFFFFFu, bmax = 0;
-#pragma unroll
-    for (int k = 0; k < kSortBatches; ++k) {
-      const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
-      if (e < m) {
-        v[k] = sorted_q[c0 + e];
-        ix[k] = idx[c0 + e];
-        lk[k] = f(v[k]);
-        bmin = min(bmin, lk[k]);
-        bmax = max(bmax, lk[k]);
-      } else {
-        v[k] = 0;
-        ix[k] = 0;
-        lk[k] = 0;
-      }
-    }
-    bmin = __reduce_min_sync(kFull, bmin);
-    bmax = __reduce_max_sync(kFull, bmax);
-    if (lane == 0) {
-      s_mm[0][warp] = bmin;
-      s_mm[1][warp] = bmax;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int w = 0; w < kSortWarps; ++w) {
-      bmin = min(bmin, s_mm[0][w]);
-      bmax = max(bmax, s_mm[1][w]);
-    }
-    uint32_t sh = 0;
-    while (((bmax - bmin) >> sh) >= (1u << kLocalBits)) ++sh;
-#pragma unroll
-    for (int k = 0; k < kSortBatches; ++k) lk[k] = (lk[k] - bmin) >> sh;
-    lsd_pass<kLoBits, 0>(v, ix, lk, m, wcnt, bin_start, tmp, s_q, s_i, s_k);
-    lsd_pass<kHiBits, kLoBits>(v, ix, lk, m, wcnt, bin_start, tmp, s_q, s_i, s_k);
-#pragma unroll
-    for (int k = 0; k < kSortBatches; ++k) {  // write back (coalesced)
-      const uint32_t e = warp * (32 * kSortBatches) + k * 32 + lane;
-      if (e < m) {
-        sorted_q[c0 + e] = v[k];
-        idx[c0 + e] = ix[k];
-      }
-    }
-  }
-}
-
 constexpr int kLocalBins = 1 << kLocalBits;
 // local histogram, sorted keys + positions, and (prefetch) the next chunk's staged queries
 template <int kCh>
@@ -1040,22 +901,17 @@ harmonia_status route_partition2(const uint64_t* q, uint64_t n, const BucketSpli
 }
 
 harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& f, int nb, const PsaWs& ws, int sm,
-                               cudaStream_t st, int level2, bool local, bool wide, uint32_t chunk) {
+                               cudaStream_t st, int level2, bool local, uint32_t chunk) {
   harmonia_status s;
-  if (wide) {  // staged-return mode only (no idx)
-    const uint32_t b1 = (uint32_t)std::min(nb, Wide::BITS);
-    s = coarse_partition<Wide>(q, n, CoarseDigit{f, (uint32_t)nb - b1}, ws, ws.sorted_q, nullptr, sm, st, nullptr,
-                               0);
-  } else {
+  {
     const uint32_t b1 = (uint32_t)std::min(nb, Narrow::BITS);
     s = coarse_partition<Narrow>(q, n, CoarseDigit{f, (uint32_t)nb - b1}, ws, ws.sorted_q, local ? nullptr : ws.idx,
                                  sm, st, nullptr, 0);
   }
   if (s != HARMONIA_OK) return s;
-  if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation / fused chunk sort)
+  if (level2 == 2) return HARMONIA_OK;  // coarse partition only (ablation)
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);  // reported in the "scan" class: level-2 sort
-    HM_CUDA(smem_attr(k_psa2_local_sort, kSortSmem));
     HM_CUDA(smem_attr(k_psa2_count_sort<false, kChunk>, count_sort_smem<kChunk>()));
     HM_CUDA(smem_attr(k_psa2_count_sort<true, kChunk>, count_sort_smem<kChunk>()));
     HM_CUDA(smem_attr(k_psa2_count_sort<true, (int)kPsaChunkMax>, count_sort_smem<kPsaChunkMax>()));
@@ -1068,9 +924,7 @@ harmonia_status psa_partition2(const uint64_t* q, uint64_t n, const BucketBits& 
 #endif
     const int cps = ch == kPsaChunkMax ? HM_SORT_CTAS_PER_SM_8K : HM_SORT_CTAS_PER_SM;
     const int g = (int)std::min<uint64_t>(ceil_div(n, ch), (uint64_t)sm * cps);
-    if (level2 == 1)  // two stable LSD passes of ballot multisplit (ablation)
-      k_psa2_local_sort<<<std::max(g, 1), kSortThreads, kSortSmem, st>>>(ws.sorted_q, ws.idx, n, f);
-    else if (local && ch == kPsaChunkMax)  // 8192-query chunks (denser key ranges per warp)
+    if (local && ch == kPsaChunkMax)  // 8192-query chunks (denser key ranges per warp)
       k_psa2_count_sort<true, (int)kPsaChunkMax>
           <<<std::max(g, 1), kSortThreads, count_sort_smem<kPsaChunkMax>(), st>>>(ws.sorted_q, ws.idx, n, f, nullptr,
                                                                                  nullptr, ws.cbounds);
@@ -1157,9 +1011,9 @@ harmonia_status psa_compact_l2(const PsaWs& ws, uint64_t* out, int sm, cudaStrea
 }
 
 harmonia_status psa_unpartition2(const PsaWs& ws, const uint64_t* res1, uint64_t n, uint64_t* out, int sm,
-                                 cudaStream_t st, bool wide) {
+                                 cudaStream_t st) {
   if (n == 0) return HARMONIA_OK;
-  return wide ? unpartition<Wide>(ws, res1, n, out, sm, st) : unpartition<Narrow>(ws, res1, n, out, sm, st);
+  return unpartition<Narrow>(ws, res1, n, out, sm, st);
 }
 
 }  // namespace hm

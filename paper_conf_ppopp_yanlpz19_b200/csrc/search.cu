@@ -913,152 +913,6 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
   }
 }
 
-// ---- level-2 PSA fused with the G = 1 search (default search path) -----------------------
-// Each CTA takes chunks of kFuseChunk queries of the level-1 (coarse) PSA order, sorts the
-// chunk by its full Nb-bit bucket with a shared-memory counting sort (the same arithmetic as
-// k_psa2_count_sort) and searches the sorted chunk straight from shared memory: the chunk
-// never goes back to L2/HBM between the sort and the search.
-constexpr int kFuseThreads = 1024, kFusePer = 4, kFuseChunk = kFuseThreads * kFusePer;  // 4096
-constexpr int kFuseBins = 2048;
-constexpr uint32_t kFuseSmem = kFuseBins * 4 + kFuseChunk * 12;  // + the staged tree top
-
-// kStaged (staged return): the chunk's own positions are the level-1 offsets, so idx is not
-// read; results are permuted back to chunk order in shared memory (over the sorted queries,
-// after every lane has read its queries) and written contiguously.
-template <int F, bool kStaged>
-__global__ void __launch_bounds__(kFuseThreads, 2) k_sort_search(const SearchArgs a) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ __align__(8) uint64_t bar;
-  __shared__ uint32_t tmp[kFuseThreads / 32 + 1], s_mm[2][kFuseThreads / 32];
-  stage_top(smem, a.ps, a.ps_smem_bytes, a.keys, a.smem_nodes * F * 8, &bar);
-  const uint32_t* s_ps = reinterpret_cast<const uint32_t*>(smem);
-  const uint64_t* s_keys = reinterpret_cast<const uint64_t*>(smem + a.ps_smem_bytes);
-  const uint32_t top = a.ps_smem_bytes + a.smem_nodes * F * 8;  // multiple of 16
-  uint64_t* sq = reinterpret_cast<uint64_t*>(smem + top);
-  uint32_t* si = reinterpret_cast<uint32_t*>(smem + top + kFuseChunk * 8);
-  uint32_t* hist = reinterpret_cast<uint32_t*>(smem + top + kFuseChunk * 12);
-  const bool ps_smem = a.ps_smem_bytes != 0;
-  const bool leaf_smem = a.h - 1 < a.smem_levels;
-  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (uint64_t c0 = (uint64_t)blockIdx.x * kFuseChunk; c0 < a.n; c0 += (uint64_t)gridDim.x * kFuseChunk) {
-    const uint32_t m = (uint32_t)((a.n - c0) < (uint64_t)kFuseChunk ? (a.n - c0) : (uint64_t)kFuseChunk);
-    // ---- load and bucket (sort by the most significant Nb bits)
-    uint64_t v[kFusePer];
-    uint32_t ix[kFusePer], b[kFusePer], rk[kFusePer];
-    uint32_t bmin = 0xFFFFFFFFu, bmax = 0;
-#pragma unroll
-    for (int k = 0; k < kFusePer; ++k) {
-      const uint32_t e = k * kFuseThreads + threadIdx.x;
-      v[k] = 0;
-      ix[k] = 0;
-      b[k] = 0;
-      if (e < m) {
-        v[k] = ld_stream(a.q + c0 + e);
-        ix[k] = kStaged ? e : ld_stream32(a.idx + c0 + e);
-        b[k] = a.bucket(v[k]);
-        bmin = min(bmin, b[k]);
-        bmax = max(bmax, b[k]);
-      }
-    }
-    bmin = __reduce_min_sync(kFull, bmin);
-    bmax = __reduce_max_sync(kFull, bmax);
-    if (lane == 0) {
-      s_mm[0][warp] = bmin;
-      s_mm[1][warp] = bmax;
-    }
-    for (uint32_t i = threadIdx.x; i < kFuseBins; i += kFuseThreads) hist[i] = 0;
-    __syncthreads();
-#pragma unroll 4
-    for (int w = 0; w < kFuseThreads / 32; ++w) {
-      bmin = min(bmin, s_mm[0][w]);
-      bmax = max(bmax, s_mm[1][w]);
-    }
-    uint32_t sh = 0;
-    while (((bmax - bmin) >> sh) >= (uint32_t)kFuseBins) ++sh;
-#pragma unroll
-    for (int k = 0; k < kFusePer; ++k) {
-      const uint32_t e = k * kFuseThreads + threadIdx.x;
-      if (e < m) {
-        b[k] = (b[k] - bmin) >> sh;
-        rk[k] = atomicAdd(&hist[b[k]], 1u);
-      }
-    }
-    __syncthreads();
-    // ---- exclusive scan of the 2048 counters (2 per thread)
-    const uint32_t h0 = hist[2 * threadIdx.x], h1 = hist[2 * threadIdx.x + 1];
-    uint32_t inc = h0 + h1;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t y = __shfl_up_sync(kFull, inc, d);
-      if (lane >= (unsigned)d) inc += y;
-    }
-    if (lane == 31) tmp[warp] = inc;
-    __syncthreads();
-    if (warp == 0) {
-      const uint32_t w = tmp[lane];
-      uint32_t wi = w;
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y = __shfl_up_sync(kFull, wi, d);
-        if (lane >= (unsigned)d) wi += y;
-      }
-      tmp[lane] = wi - w;
-    }
-    __syncthreads();
-    const uint32_t ex = tmp[warp] + inc - (h0 + h1);
-    hist[2 * threadIdx.x] = ex;
-    hist[2 * threadIdx.x + 1] = ex + h0;
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < kFusePer; ++k) {
-      const uint32_t e = k * kFuseThreads + threadIdx.x;
-      if (e < m) {
-        const uint32_t dst = hist[b[k]] + rk[k];
-        sq[dst] = v[k];
-        si[dst] = ix[k];
-      }
-    }
-    __syncthreads();
-    // ---- search the sorted chunk: warp w takes positions [w*128, w*128+128), 2 per lane per round
-    uint64_t rr[kFusePer];
-    uint32_t ro[kFusePer];
-    bool ra[kFusePer];
-#pragma unroll
-    for (int rd = 0; rd < kFusePer / 2; ++rd) {
-      uint64_t q0[2], o[2];
-      bool act[2];
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const uint32_t p = warp * (32 * kFusePer) + (rd * 2 + u) * 32 + lane;
-        act[u] = p < m;
-        q0[u] = act[u] ? sq[p] : kPad;
-        o[u] = act[u] ? si[p] : 0;
-      }
-      uint64_t res[2];
-      lane_core<F, 2>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        if constexpr (kStaged) {
-          rr[rd * 2 + u] = res[u];
-          ro[rd * 2 + u] = (uint32_t)o[u];
-          ra[rd * 2 + u] = act[u];
-        } else if (act[u]) {
-          a.out[o[u]] = res[u];
-        }
-      }
-    }
-    if constexpr (kStaged) {
-      __syncthreads();  // every lane has read its queries: sq becomes the result stage
-#pragma unroll
-      for (int k = 0; k < kFusePer; ++k)
-        if (ra[k]) sq[ro[k]] = rr[k];
-      __syncthreads();
-      for (uint32_t i = threadIdx.x; i < m; i += kFuseThreads) a.out[c0 + i] = sq[i];
-    }
-    __syncthreads();  // the chunk buffers are reused
-  }
-}
-
 // Range scan: descend with lo, then walk leaf slots in key-region order.  One CTA per SM
 // (64 registers): at two CTAs the 32-register cap spilled 16-40 bytes per thread.
 template <int F, int G, int MODE>
@@ -1404,24 +1258,6 @@ harmonia_status launch_range_warp_f(const harmonia_tree* t, const Plan& p, const
 }
 
 template <int F>
-harmonia_status launch_sort_search_f(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
-  auto kern = a.staged ? k_sort_search<F, true> : k_sort_search<F, false>;
-  const uint32_t smem = p.smem_bytes + kFuseSmem;
-  HM_CUDA(smem_attr(kern, smem));
-  int per_sm = 0;
-  HM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kFuseThreads, smem));
-  per_sm = std::max(per_sm, 1);
-  const uint64_t need = ceil_div(a.n, kFuseChunk);
-  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)t->sm_count * per_sm));
-  {
-    ProfScope ps_(HARMONIA_PROF_SEARCH, st);
-    HM_CUDA(launch_win(kern, dim3(grid), dim3(kFuseThreads), smem, st, p, a));
-  }
-  HM_LAUNCHED();
-  return HARMONIA_OK;
-}
-
-template <int F>
 harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
   const int U = p.lane_ilp;
   auto kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true> : (U == 2 ? k_lane_search_c<F, 2, true> : k_lane_search_c<F, 1, true>))
@@ -1594,20 +1430,6 @@ harmonia_status launch_range_lane(const harmonia_tree* t, const Plan& p, const R
     case 64: return launch_range_lane_f<64>(t, p, ra, sa, st);
     case 128: return launch_range_lane_f<128>(t, p, ra, sa, st);
     case 256: return launch_range_lane_f<256>(t, p, ra, sa, st);
-  }
-  return HARMONIA_ERR_INVALID_ARG;
-}
-
-harmonia_status launch_sort_search(const harmonia_tree* t, const Plan& p, const SearchArgs& a, cudaStream_t st) {
-  if (a.n == 0) return HARMONIA_OK;
-  switch (t->F) {
-    case 4: return launch_sort_search_f<4>(t, p, a, st);
-    case 8: return launch_sort_search_f<8>(t, p, a, st);
-    case 16: return launch_sort_search_f<16>(t, p, a, st);
-    case 32: return launch_sort_search_f<32>(t, p, a, st);
-    case 64: return launch_sort_search_f<64>(t, p, a, st);
-    case 128: return launch_sort_search_f<128>(t, p, a, st);
-    case 256: return launch_sort_search_f<256>(t, p, a, st);
   }
   return HARMONIA_ERR_INVALID_ARG;
 }

@@ -131,15 +131,23 @@ def test_lane_search_queries_per_lane(hm, orc, F, lane_queries):
     t = tree(hm, keys, vals, F)
     q = np.concatenate([gen.uniform_queries(keys, 50003, miss_frac=0.4), gen.edge_queries(keys)])
     exp = orc.sorted_search(keys, vals, q)
-    for kw in ({}, {"psa_bits": -1}, {"window": 3072}, {"smem_levels": -1}, {"flags": hm.QF_FUSE_SORT},
-               {"flags": hm.QF_FUSE_SORT, "window": 5120, "smem_levels": 1}, {"flags": hm.QF_SCATTER_RETURN},
+    for kw in ({}, {"psa_bits": -1}, {"window": 3072}, {"smem_levels": -1}, {"flags": hm.QF_SCATTER_RETURN},
                {"flags": hm.QF_SCATTER_RETURN, "window": 7168}, {"window": 7168, "smem_levels": -1},
-               {"flags": hm.QF_PSA_WIDE}, {"flags": hm.QF_PSA_WIDE, "window": 13312},
+               {"flags": hm.QF_PSA_L16, "psa_bits": 17}, {"flags": hm.QF_PSA_L16, "psa_bits": 17, "window": 13312},
                {"flags": hm.QF_PER_LANE}, {"flags": hm.QF_PER_LANE, "window": 7168, "smem_levels": -1},
                {"sort_chunk": 8192}, {"sort_chunk": 8192, "window": 13312}, {"sort_chunk": 4096},
                {"sort_chunk": 8192, "smem_levels": -1}, {"sort_chunk": 8192, "flags": hm.QF_PER_LANE}):
         got = host(t.search(cu(q), group_size=1, lane_queries=lane_queries, **kw))
         assert np.array_equal(got, exp), kw
+
+
+def test_removed_ablation_flags_rejected(hm):
+    """ABI 2 retired three ablation flags (64, 128, 512): they are INVALID_ARG, not ignored."""
+    keys = gen.uniform_keys(1000)
+    t = tree(hm, keys, gen.values_for(keys), 16)
+    for f in (64, 128, 512):
+        with pytest.raises(hm.HarmoniaError):
+            t.search(cu(keys), flags=f)
 
 
 @pytest.mark.parametrize("F", [4, 16, 64, 128])

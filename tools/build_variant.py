@@ -1,5 +1,5 @@
-"""Build an ablation variant of libharmonia.so with extra -D macros into gpurun_variants/<name>.so
-(run with HARMONIA_LIB=gpurun_variants/<name>.so).  Used only for A/B measurements.
+"""Build an ablation variant of libharmonia.so with extra -D macros into tools/bin/<name>.so
+(run with HARMONIA_LIB=tools/bin/<name>.so; tools/bin travels with gpurun).  Used only for A/B measurements.
 
     python tools/build_variant.py NAME [-DMACRO[=V] ...]
 """
@@ -11,7 +11,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ppopp_yanlpz19_b200 import _build as b  # noqa: E402
 
 name, defs = sys.argv[1], sys.argv[2:]
-out_dir = os.path.join(b.ROOT, "gpurun_variants")
+out_dir = os.path.join(b.ROOT, "tools", "bin")
 tmp = os.path.join(out_dir, "obj_" + name)
 os.makedirs(tmp, exist_ok=True)
 procs, objs = [], []
