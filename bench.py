@@ -36,8 +36,10 @@ CONFIGS = {
     # config 5: 2^32 keys range-partitioned over 8 shards of 2^29 (rank p holds shard p), queries
     # uniform over the running ranks' keys and routed, update batches of 2^22 ops (5 % insert,
     # 5 % delete, 90 % update) interleaved 1:1 with the query batches
-    5: dict(name="c5_T2^32_8shards_F64_Q2^27_uniform_partitioned_updates", T=1 << 32, F=64, Q=1 << 27,
-            dist="uniform", shards=8, ops=1 << 22),
+    # The shard is bulk-loaded at fill 0.69, the occupancy of the paper's insertion-built trees
+    # ("half full", P:L592 fn 3; C-A6), so update batches go in place when leaves have room.
+    5: dict(name="c5_T2^32_8shards_F64_fill0.69_Q2^27_uniform_partitioned_updates", T=1 << 32, F=64, Q=1 << 27,
+            dist="uniform", shards=8, ops=1 << 22, fill=0.69),
 }
 METRIC = "point queries/sec (G q/s) at 1/2/4/8 B200; % of L2/HBM roofline"
 UNIT = "G q/s"
@@ -437,7 +439,8 @@ def run_config5(a, c, hm, dev, world, rank, local, pg):
     sp = [int(x) & ((1 << 64) - 1) for x in gen.keys_at_t(T, torch.tensor([p * S for p in range(1, P)],
                                                                             dtype=torch.int64)).tolist()]
     t_build = time.perf_counter()
-    pt = PartitionedTree(lk.view(torch.uint64), gen.values_for_t(lk).view(torch.uint64), sp, fanout=F, device=dev)
+    pt = PartitionedTree(lk.view(torch.uint64), gen.values_for_t(lk).view(torch.uint64), sp, fanout=F,
+                         fill=c.get("fill", 1.0), device=dev)
     torch.cuda.synchronize()
     t_build = time.perf_counter() - t_build
     del lk
@@ -515,15 +518,28 @@ def run_config5(a, c, hm, dev, world, rank, local, pg):
     breakdown = {k: {"ms_per_step": v[0] / a.steps, "launches_per_step": v[1] / a.steps,
                      "share": v[0] / max(1e-9, sum(x[0] for x in prof.values()))} for k, v in prof.items()}
     roof = None
-    if "update" in prof:  # the rebuild: read records (16 B), write merged records (16 B),
-        # write the key region + leaf values (16 B x F/(F-1)) per record of the shard
-        n_rec = info["n_keys"]
-        byt = n_rec * (16 + 16 + 16 * F / (F - 1))
+    dom = max(prof.items(), key=lambda kv: kv[1][0]) if prof else None
+    mode = {1: "in place", 2: "full rebuild"}.get(t.last_update_mode(), "?")
+    if dom and dom[0] == "update":
         avg = prof["update"][0] / prof["update"][1]
-        roof = {"bound": "hbm", "kernel": "harmonia_update_batch (sort, merge, layout rebuild)",
-                "achieved": byt / (avg / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
-                "frac": byt / (avg / 1e3) / 1e9 / hbm_peak, "traffic": None, "peak_source": peak_src,
-                "algorithmic_bytes_per_launch": byt, "avg_launch_ms": avg}
+        if mode == "full rebuild":  # read records (16 B), write merged records (16 B), write the
+            # key region + leaf values (16 B x F/(F-1)) per record of the shard
+            byt = info["n_keys"] * (16 + 16 + 16 * F / (F - 1))
+            what = "harmonia_update_batch (sort, merge, layout rebuild)"
+        else:  # batch in (17 B/op) + key sort (2 x 12 B/op) + winners/locate/classify (~40 B/op)
+            # + the changed leaves re-packed (2 x 1 KiB read + write per changed leaf, <= 1 per insert/delete)
+            byt = c["ops"] * (17 + 24 + 40 + 0.1 * 2 * 2 * F * 8)
+            what = "harmonia_update_batch in place (sort, locate, re-pack changed leaves)"
+        roof = {"bound": "hbm", "kernel": what, "achieved": byt / (avg / 1e3) / 1e9, "peak": hbm_peak,
+                "unit": "GB/s", "frac": byt / (avg / 1e3) / 1e9 / hbm_peak, "traffic": None,
+                "peak_source": peak_src, "algorithmic_bytes_per_launch": byt, "avg_launch_ms": avg}
+    elif dom and dom[0] == "search":
+        avg = dom[1][0] / dom[1][1]
+        plan5 = t.plan(c["Q"])
+        byt, _ = roofline_model(info, plan5, c["Q"], 0)
+        roof = {"bound": "hbm", "kernel": "k_lane_search_c", "achieved": byt / (avg / 1e3) / 1e9, "peak": hbm_peak,
+                "unit": "GB/s", "frac": byt / (avg / 1e3) / 1e9 / hbm_peak, "traffic": None,
+                "peak_source": peak_src, "algorithmic_bytes_per_launch": byt, "avg_launch_ms": avg}
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
         "warmup": max(3, a.warmup), "ms_per_step": ms_max / a.steps,
@@ -534,7 +550,7 @@ def run_config5(a, c, hm, dev, world, rank, local, pg):
                    "queries": "uniform over the running shards' keys", "mode": "partitioned",
                    "l2_flush": "inputs_larger_than_L2 (2^27 queries + a 2^29-key shard per GPU)",
                    "plan": t.plan(c["Q"]), "height": info["height"], "build_s": t_build},
-        "updates_per_s": {"value": ups, "unit": "G ops/s"},
+        "updates_per_s": {"value": ups, "unit": "G ops/s", "mode": mode},
         "roofline": roof, "cpu_baseline": None, "e2e": e2e, "gpu_launches": int(launches),
         "clocks": clk.summary(), "kernel_breakdown": breakdown, "parity_sample_ok": parity_ok,
     }

@@ -217,17 +217,22 @@ harmonia_status harmonia_range_batch(const harmonia_tree* tree, const uint64_t* 
  *   1 = delete: remove if present), d_keys[n], d_values[n] (ignored for deletes).
  *   Sequential semantics in batch order: the last op on a key wins.  Keys equal to
  *   HARMONIA_KEY_PAD or upsert values equal to HARMONIA_NOT_FOUND are rejected
- *   (HARMONIA_ERR_RESERVED, tree unchanged).  The whole layout is rebuilt from the merged
- *   record sequence: re-packed leaves, internal levels and PS recomputed (the paper's
- *   post-batch "movement", as bulk-synchronous device passes; a rebuild from the
- *   first affected leaf costs the same passes on the GPU, and the full rebuild keeps the
- *   layout bit-identical to a fresh harmonia_build, invariant I8).  The batch sort and scans
- *   use CUB (a library primitive, like cuBLAS for a GEMM; not on the query path).  A tree of
- *   2^31 - 1 or more records after the batch is HARMONIA_ERR_TOO_LARGE (32-bit scan counts).
- *   May reallocate the tree's arrays; synchronises `stream`.
+ *   (HARMONIA_ERR_RESERVED, tree unchanged).  In place when the leaves have room: if every
+ *   leaf the batch changes keeps between ceil((F-1)/2) and F-1 records (trees built with fill
+ *   < 1), values are overwritten, the changed leaves re-packed where the separators route their
+ *   keys and the leaf record counts recomputed; the key region, PS and internal levels keep
+ *   their positions (separators still bound their subtrees, I5, but need not equal subtree
+ *   minima after deletes).  Otherwise the whole layout is rebuilt from the merged record
+ *   sequence (the paper's post-batch "movement", as bulk-synchronous device passes;
+ *   bit-identical to a fresh harmonia_build, invariant I8).  harmonia_update_last_mode tells
+ *   which (1 in place, 2 rebuilt).  The batch sort and scans use CUB (a library primitive,
+ *   like cuBLAS for a GEMM; not on the query path).  A tree of 2^31 - 1 or more records after
+ *   the batch is HARMONIA_ERR_TOO_LARGE (32-bit scan counts).  May reallocate the tree's
+ *   arrays; synchronises `stream`.
  *   d_workspace must hold harmonia_update_workspace_bytes(tree, n).
  * ------------------------------------------------------------------------------------- */
 size_t harmonia_update_workspace_bytes(const harmonia_tree* tree, uint64_t n);
+int harmonia_update_last_mode(const harmonia_tree* tree); /* 0 none yet, 1 in place, 2 rebuilt */
 harmonia_status harmonia_update_batch(harmonia_tree* tree, const uint8_t* d_ops,
                                       const uint64_t* d_keys, const uint64_t* d_values,
                                       uint64_t n, void* d_workspace, size_t workspace_bytes,

@@ -78,6 +78,8 @@ def lib():
             "orc_layout_build": (C.c_int, [u64p, u64p, C.c_uint64, C.c_uint32, C.c_double, u64p, u32p, u64p]),
             "orc_layout_check": (C.c_int, [u64p, u32p, u64p, C.c_uint32, C.c_uint32, u64p, u64p, u64p,
                                            C.c_uint64, C.c_char_p, C.c_int]),
+            "orc_layout_check2": (C.c_int, [u64p, u32p, u64p, C.c_uint32, C.c_uint32, u64p, u64p, u64p,
+                                            C.c_uint64, C.c_char_p, C.c_int, C.c_int]),
             "orc_layout_search": (None, [u64p, u32p, u64p, C.c_uint32, C.c_uint32, u64p, u64p, C.c_uint64, u64p]),
             "orc_layout_range": (None, [u64p, u32p, u64p, C.c_uint32, C.c_uint32, u64p, u64p, u64p, C.c_uint64,
                                         C.c_uint32, u64p, u64p, u32p]),
@@ -256,11 +258,14 @@ class Layout:
     def n_internal(self):
         return int(self.level_start[self.h - 1])
 
-    def check(self, keys, vals):
+    def check(self, keys, vals, strict_separators: bool = True):
+        """I1-I7 against the record set; strict_separators=False drops the equality half of I5
+        (separator == subtree minimum), which only a fresh build guarantees."""
         keys, vals = _u64(keys), _u64(vals)
         msg = C.create_string_buffer(256)
-        r = lib().orc_layout_check(_p64(self.key_region), _p32(self.ps), _p64(self.leaf_vals), self.F, self.h,
-                                   _p64(self.level_start), _p64(keys), _p64(vals), keys.shape[0], msg, 256)
+        r = lib().orc_layout_check2(_p64(self.key_region), _p32(self.ps), _p64(self.leaf_vals), self.F, self.h,
+                                    _p64(self.level_start), _p64(keys), _p64(vals), keys.shape[0], msg, 256,
+                                    1 if strict_separators else 0)
         return int(r), msg.value.decode()
 
     def search(self, q) -> np.ndarray:

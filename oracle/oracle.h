@@ -102,6 +102,12 @@ int      orc_layout_check(const uint64_t* key_region, const uint32_t* ps,
                           const uint64_t* level_start /* h+1 entries */,
                           const uint64_t* keys, const uint64_t* vals, uint64_t n,
                           char* msg, int msglen);
+/* The same with strict_sep = 0: the equality half of I5 (separator == subtree minimum, a
+ * property of a fresh build) is not required -- for layouts updated in place. */
+int      orc_layout_check2(const uint64_t* key_region, const uint32_t* ps,
+                           const uint64_t* leaf_vals, uint32_t fanout, uint32_t height,
+                           const uint64_t* level_start, const uint64_t* keys, const uint64_t* vals,
+                           uint64_t n, char* msg, int msglen, int strict_sep);
 /* Scalar Eq-1 interpreter: child_idx = PrefixSum[node_idx] + i - 1. */
 void     orc_layout_search(const uint64_t* key_region, const uint32_t* ps,
                            const uint64_t* leaf_vals, uint32_t fanout, uint32_t height,

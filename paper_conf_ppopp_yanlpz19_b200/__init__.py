@@ -103,6 +103,7 @@ def lib():
             "harmonia_update_batch": (C.c_int, [_vp, _vp, _vp, _vp, _u64, _vp, _sz, _vp]),
             "harmonia_update_batch_seq": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _u64, _vp, _sz, _vp]),
             "harmonia_update_validate": (C.c_int, [_vp, _vp, _vp, _u64, _vp, _vp]),
+            "harmonia_update_last_mode": (C.c_int, [_vp]),
             "harmonia_route_update_payload": (C.c_int, [_vp, _vp, _vp, _u64, C.c_uint32, _vp, _vp, _vp, _vp]),
             "harmonia_route_workspace_bytes": (_sz, [C.c_uint32, _u64]),
             "harmonia_route_partition": (C.c_int, [_vp, C.c_uint32, _vp, _u64, _vp, _vp, _vp, _vp, _sz, _vp]),
@@ -392,6 +393,10 @@ class Tree:
                                           ws.data_ptr() if ws is not None else None, ws_b, C.byref(o), st),
                "harmonia_range_batch")
         return ko, vo, cnt
+
+    def last_update_mode(self) -> int:
+        """1 if the last update batch ran in place, 2 if it rebuilt the layout (0: none yet)."""
+        return int(lib().harmonia_update_last_mode(self._h))
 
     def update(self, ops, keys, values, seq=None, stream=None):
         """Batched upsert (op 0) / delete (op 1), sequential semantics in batch order (or in

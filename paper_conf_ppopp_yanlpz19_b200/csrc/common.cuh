@@ -179,6 +179,7 @@ struct harmonia_tree {
   size_t l2_bytes = 0;
   size_t l2_persist_max = 0, l2_window_max = 0;  // device limits for the access-policy window
   size_t l2_persist_set = 0;                     // cudaLimitPersistingL2CacheSize this tree set
+  int last_update_mode = 0;                      // 1 in place, 2 full rebuild (last update batch)
   // host-pipeline streams/events (harmonia_search_batch_host)
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
   cudaEvent_t ev_start = nullptr, ev_in[2] = {}, ev_done[2] = {}, ev_out[2] = {};
@@ -419,7 +420,9 @@ struct RangeArgs {
 };
 harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeArgs& a,
                              cudaStream_t st);
-// short ranges (cap < 128, PSA-ordered lo): one lane per range on the warp-shared descent
+// in-place update: out[i] = (leaf index << 32) | #keys <= q[i] in that leaf (q sorted)
+harmonia_status launch_locate(const harmonia_tree* t, const uint64_t* q, uint64_t n, uint64_t* out, cudaStream_t st);
+// short ranges (cap < 512, PSA-ordered lo): one lane per range on the warp-shared descent
 harmonia_status launch_range_lane(const harmonia_tree* t, const Plan& p, const RangeArgs& ra, const SearchArgs& sa,
                                   cudaStream_t st);
 

@@ -1135,6 +1135,26 @@ __global__ void __launch_bounds__(1024, 1) k_range_warp(const RangeArgs a) {
   }
 }
 
+// ---- key location for the in-place update: (leaf << 32) | #keys <= q in that leaf ----------
+// The batch keys arrive sorted (the update's stable key sort), so the warp-shared descent
+// applies as for PSA-ordered queries.
+template <int F>
+__global__ void __launch_bounds__(256) k_locate(const SearchArgs a, const uint64_t* __restrict__ q, uint64_t n,
+                                                uint64_t* __restrict__ out) {
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t base = warp * 32; base < n; base += nwarps * 32) {
+    const uint64_t j = base + lane;
+    const bool act = j < n;
+    uint64_t q0[1] = {act ? q[j] : kPad};
+    bool live[1] = {act && q0[0] != kPad};
+    uint64_t res[1];
+    warp_core<F, 1, true>(a, nullptr, nullptr, false, false, q0, live, res);
+    if (act) out[j] = res[0];
+  }
+}
+
 // ---- short ranges (cap < 512): one lane per range ------------------------------------------
 // The ranges arrive PSA-ordered by lo, so a warp's 32 ranges lie in a narrow key interval and
 // share the warp's descent (warp_core): every lane ranks lo - 1 and hi at once (two chains per
@@ -1417,6 +1437,34 @@ harmonia_status launch_range(const harmonia_tree* t, const Plan& p, const RangeA
   }
   const int G = p.G == 1 ? 2 : p.G;  // ranges scan leaves with at least a lane pair
   HM_DISPATCH(launch_range_fg, t->F, G, t, p, a, st)
+}
+
+harmonia_status launch_locate(const harmonia_tree* t, const uint64_t* q, uint64_t n, uint64_t* out, cudaStream_t st) {
+  if (n == 0) return HARMONIA_OK;
+  SearchArgs a{};
+  a.keys = t->d_keys;
+  a.ps = t->d_ps;
+  a.vals = t->d_vals;
+  a.leaf_start = t->level_start[t->h - 1];
+  a.h = t->h;
+  a.coop = 1;
+  a.kmin = t->min_key;
+  a.kmax = t->max_key;
+  const uint32_t span = t->min_key < t->max_key ? 64 - __builtin_clzll(t->min_key ^ t->max_key) : 0;
+  a.cshift = span > 32 ? span - 32 : 0;
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(n, 256), (uint64_t)t->sm_count * 8));
+  switch (t->F) {
+#define HM_LOC(F_)                                        \
+  case F_:                                                \
+    k_locate<F_><<<grid, 256, 0, st>>>(a, q, n, out);     \
+    break;
+    HM_LOC(4) HM_LOC(8) HM_LOC(16) HM_LOC(32) HM_LOC(64) HM_LOC(128) HM_LOC(256)
+#undef HM_LOC
+    default:
+      return HARMONIA_ERR_INVALID_ARG;
+  }
+  HM_LAUNCHED();
+  return HARMONIA_OK;
 }
 
 harmonia_status launch_range_lane(const harmonia_tree* t, const Plan& p, const RangeArgs& ra, const SearchArgs& sa,

@@ -153,3 +153,79 @@ def test_route_update_payload(hm):
     assert np.array_equal(o.cpu().numpy(), ops[pos])
     assert np.array_equal(v.cpu().numpy(), vals[pos])
     assert np.array_equal(s.cpu().numpy(), (np.uint64(5) << np.uint64(32)) | pos.astype(np.uint64))
+
+
+def check_tree_relaxed(hm, orc, t, F, ref_keys, ref_vals, probe):
+    """After in-place batches: I1-I7 with routing separators (the equality half of I5 only
+    holds for a fresh build), results equal to the std::map oracle."""
+    info, kr, ps, lv = t.export_layout()
+    assert info["n_keys"] == ref_keys.shape[0]
+    assert info["min_key"] == int(ref_keys[0]) and info["max_key"] == int(ref_keys[-1])
+    code, msg = orc.Layout(F, info["height"], info["level_start"], kr, ps, lv).check(ref_keys, ref_vals,
+                                                                                    strict_separators=False)
+    assert code == 0, msg
+    out = t.search(cu(probe)).cpu().numpy()
+    assert np.array_equal(out, orc.sorted_search(ref_keys, ref_vals, probe))
+    for cap in (8, 300):  # the lane and the warp range kernels (counts from the recomputed leaf_base)
+        lo, hi = gen.random_ranges(ref_keys, 500, max_width_keys=3 * cap)
+        ko, vo, cnt = t.range(cu(lo), cu(hi), cap)
+        eko, evo, ecnt = orc.sorted_range(ref_keys, ref_vals, lo, hi, cap)
+        assert np.array_equal(cnt.cpu().numpy(), ecnt)
+        m = np.minimum(ecnt.astype(np.int64), cap)
+        mask = np.arange(cap)[None, :] < m[:, None]
+        assert np.array_equal(ko.cpu().numpy()[mask], eko[mask]) and np.array_equal(vo.cpu().numpy()[mask], evo[mask])
+
+
+@pytest.mark.parametrize("F,fill,in_place", [(8, 0.69, False), (16, 0.69, True), (32, 0.69, True), (64, 0.69, True),
+                                             (128, 0.75, True)])
+def test_update_in_place(hm, orc, F, fill, in_place):
+    """Trees with room (fill < 1): the paper's 5 % insert + 5 % delete + 90 % update batches
+     go in place; values, re-packed leaves and leaf_base match the oracle after every
+    batch, including keys below the minimum / above the maximum and repeated keys."""
+    keys = gen.uniform_keys(60000)
+    vals = gen.values_for(keys)
+    t = hm.Tree(cu(keys), cu(vals), fanout=F, fill=fill)
+    ref = orc.UpdateMap(keys, vals)
+    touched = []
+    modes = []
+    for b in range(5):
+        rk, _ = ref.dump()
+        ops, ks, vs = gen.update_ops(rk, 3000, insert_frac=0.05, delete_frac=0.05, seed=gen.SEED_OPS + 7 * b + F)
+        ops = np.concatenate([ops, ops[:200] ^ np.uint8(1), np.zeros(2, dtype=np.uint8)])
+        ks = np.concatenate([ks, ks[:200], np.array([b + 1, MAX - 1 - b], dtype=np.uint64)])
+        vs = np.concatenate([vs, vs[:200] + np.uint64(3), np.array([5, 6], dtype=np.uint64)])
+        t.update(ops, cu(ks), cu(vs))
+        modes.append(t.last_update_mode())
+        ref.apply(ops, ks, vs)
+        touched.append(ks)
+        rk, rv = ref.dump()
+        probe = np.concatenate([np.concatenate(touched), gen.uniform_queries(rk, 20000, miss_frac=0.3),
+                                gen.edge_queries(rk)])
+        check_tree_relaxed(hm, orc, t, F, rk, rv, probe)
+    # in place unless a leaf ran out of room (F = 8 at fill 0.69 builds minimum-occupancy
+    # leaves of 4 records: any delete there underflows, so those batches rebuild)
+    assert modes.count(1) >= 2 if in_place else modes.count(2) >= 1, modes
+
+
+def test_update_in_place_overflow_falls_back(hm, orc):
+    """A batch that overfills one leaf (many inserts into one key gap) takes the full rebuild,
+    whose layout is the closed form again; in-place batches resume afterwards."""
+    keys = (np.arange(1, 20001, dtype=np.uint64) * np.uint64(1000))
+    vals = gen.values_for(keys)
+    F = 16
+    t = hm.Tree(cu(keys), cu(vals), fanout=F, fill=0.69)
+    ref = orc.UpdateMap(keys, vals)
+    ks = np.arange(5001, 5001 + 40, dtype=np.uint64)  # 40 keys into the gap after key 5000
+    ops = np.zeros(ks.shape[0], dtype=np.uint8)
+    vs = gen.values_for(ks)
+    t.update(ops, cu(ks), cu(vs))
+    ref.apply(ops, ks, vs)
+    assert t.last_update_mode() == 2
+    rk, rv = ref.dump()
+    check_tree_relaxed(hm, orc, t, F, rk, rv, np.concatenate([ks, gen.uniform_queries(rk, 5000, miss_frac=0.3)]))
+    ops2, ks2, vs2 = gen.update_ops(rk, 500, insert_frac=0.0, delete_frac=0.02, seed=99)
+    t.update(ops2, cu(ks2), cu(vs2))
+    ref.apply(ops2, ks2, vs2)
+    assert t.last_update_mode() == 1
+    rk, rv = ref.dump()
+    check_tree_relaxed(hm, orc, t, F, rk, rv, np.concatenate([ks2, gen.uniform_queries(rk, 5000, miss_frac=0.3)]))

@@ -172,3 +172,29 @@ def test_shape_fill_below_one():
         n, F, fill, levels = 1 << int(f[0]), int(f[1]), float(f[2]), [int(x) for x in f[3:]]
         h, ln_ = oracle.layout_shape(n, F, fill)
         assert h == len(levels) and ln_.tolist() == levels, (n, F, fill)
+
+
+def test_relaxed_separator_check(orc):
+    """strict_separators=False accepts a layout whose leaf lost its minimum (a delete applied in
+    place) but still rejects keys outside the separator bounds (I5 routing)."""
+    keys = gen.uniform_keys(3000)
+    vals = gen.values_for(keys)
+    lay = orc.layout_build(keys, vals, 8, 1.0)  # 7 records per leaf: one can go (I3 >= 4)
+    I, F = lay.n_internal, lay.F
+    leaf = I + 5  # a leaf with a separator in its parent (not the first child)
+    kr, lv = lay.key_region.copy(), lay.leaf_vals.copy()
+    cnt = int((kr[leaf * F:(leaf + 1) * F] != np.uint64(PAD)).sum())
+    gone = kr[leaf * F]
+    kr[leaf * F:leaf * F + cnt - 1] = kr[leaf * F + 1:leaf * F + cnt]
+    kr[leaf * F + cnt - 1] = np.uint64(PAD)
+    lv[(leaf - I) * F:(leaf - I) * F + cnt - 1] = lv[(leaf - I) * F + 1:(leaf - I) * F + cnt]
+    lv[(leaf - I) * F + cnt - 1] = np.uint64(PAD)
+    keep = keys != gone
+    mut = orc.Layout(F, lay.h, lay.level_start.copy(), kr, lay.ps.copy(), lv)
+    assert cnt - 1 >= F // 2
+    assert mut.check(keys[keep], vals[keep])[0] == 5                      # strict: separator != min
+    assert mut.check(keys[keep], vals[keep], strict_separators=False)[0] == 0
+    bad = orc.Layout(F, lay.h, lay.level_start.copy(), kr.copy(), lay.ps.copy(), lv)
+    bad.key_region[leaf * F] = np.uint64(1)                              # below its separator
+    kk = np.sort(np.concatenate([keys[keep & (keys != kr[leaf * F])], np.array([1], dtype=np.uint64)]))
+    assert bad.check(kk, gen.values_for(kk), strict_separators=False)[0] != 0

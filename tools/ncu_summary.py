@@ -102,7 +102,7 @@ if __name__ == "__main__":
     json.dump(res, open(a.out + ".json", "w"), indent=1)
     # per-launch figures for bench.py's roofline (profiles/ncu_r2.json): traffic, L2 bytes,
     # sectors per request (memory divergence), warp coherence (P:L654 fn 4)
-    tr_path = os.path.join(os.path.dirname(a.out), "ncu_r2.json")
+    tr_path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "ncu_r2.json")
     tr = json.load(open(tr_path)) if os.path.exists(tr_path) else {}
     for d in res.get("full_capture", []):
         k = d["kernel"].split("<")[0]

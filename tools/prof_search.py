@@ -25,18 +25,18 @@ ap.add_argument("--flags", type=int, default=0)
 ap.add_argument("--range-len", type=int, default=0)
 a = ap.parse_args()
 
-keys = gen.uniform_keys(1 << a.keys)
-vals = gen.values_for(keys)
-t = hm.Tree(torch.from_numpy(keys).cuda(), torch.from_numpy(vals).cuda(), fanout=a.fanout)
+kt = gen.uniform_keys_t(1 << a.keys, "cuda")  # device generators (= the numpy streams, tests/test_gen.py)
+t = hm.Tree(kt.view(torch.uint64), gen.values_for_t(kt).view(torch.uint64), fanout=a.fanout)
 o = hm.make_opts(a.group_size, a.psa_bits, a.smem_levels, a.window, a.flags)
 if a.range_len:
+    keys = kt.cpu().numpy().view(np.uint64)
     lo, hi = gen.ranges(keys, 1 << a.queries, a.range_len)
     lo, hi = torch.from_numpy(lo).cuda(), torch.from_numpy(hi).cuda()
     for _ in range(a.calls):
         t.range(lo, hi, a.range_len, opts=o)
 else:
-    q = gen.zipf_queries(keys, 1 << a.queries) if a.dist == "zipf" else gen.uniform_queries(keys, 1 << a.queries)
-    q = torch.from_numpy(q).cuda()
+    q = gen.zipf_queries_t(kt, 1 << a.queries) if a.dist == "zipf" else gen.uniform_queries_t(kt, 1 << a.queries)
+    q = q.view(torch.uint64)
     out = torch.empty_like(q)
     for _ in range(a.calls):
         t.search(q, out, opts=o)
