@@ -261,7 +261,9 @@ struct PsaWs {
   uint32_t* cta_counts; // kL1CtaRows: per level-1 CTA bin totals
   uint32_t* cta_base;   // kL1CtaRows: per level-1 CTA first global slot of each bin
   // ---- second MSD level (Plan::psa_levels == 2), inside the level-1 segments
-  uint32_t* seg;        // [0..256] level-1 segment starts, [257..513] first level-2 tile per segment
+  uint32_t* seg;        // [0..256] level-1 segment starts, [257..513] first level-2 tile per segment,
+                        // then 3 x 64 words of the layout's CTA totals
+  uint32_t* l2_scratch; // 3 x 65536 words: the layout's per-group prefixes
   uint32_t* packed2;    // window: level-2 digit | rank-in-tile << 8, at level-1 positions
   uint32_t* tile_counts2;  // level-2 tiles x 256 digit counts
   uint32_t* tile_base2;    // level-2 tiles x 256: level-2 position of each tile's digit run
@@ -309,7 +311,7 @@ inline L2Sizes l2_sizes(uint64_t window, uint32_t chunk) {
 inline uint64_t l2_ws_bytes(uint64_t window, uint32_t chunk) {
   const L2Sizes z = l2_sizes(window, chunk);
   auto r = [](uint64_t b) { return (b + 255) / 256 * 256; };
-  return r(2 * 257 * 4) + r(window * 4) + 2 * r(z.tiles * 256 * 4) + r(kL2Buckets * 4) + r((kL2Buckets + 1) * 4) +
+  return r((2 * 257 + 3 * 64) * 4) + r(3 * kL2Buckets * 4) + r(window * 4) + 2 * r(z.tiles * 256 * 4) + r(kL2Buckets * 4) + r((kL2Buckets + 1) * 4) +
          r(z.chunks * 8) + r(z.chunks * 4) + 256 + 2 * r(z.padded * 8) + r(z.padded * 2);
 }
 size_t psa_ws_bytes(const Plan& p);

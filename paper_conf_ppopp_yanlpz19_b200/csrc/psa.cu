@@ -201,7 +201,9 @@ PsaWs psa_ws_carve(const Plan& p, void* base) {
   if (p.psa_levels == 2) {
     const L2Sizes z = l2_sizes(p.window, p.chunk);
     w.seg = (uint32_t*)c;
-    c += round_up(2 * 257 * 4, 256);
+    c += round_up((2 * 257 + 3 * 64) * 4, 256);  // + the layout's CTA totals
+    w.l2_scratch = (uint32_t*)c;
+    c += round_up(3 * kL2Buckets * 4, 256);
     w.packed2 = (uint32_t*)c;
     c += round_up(p.window * 4, 256);
     w.tile_counts2 = (uint32_t*)c;

@@ -578,45 +578,75 @@ __global__ void __launch_bounds__(256) k_l2_colsum(const uint32_t* __restrict__ 
   comp_cnt[s * 256 + threadIdx.x] = acc;
 }
 
-// level-2 layout (one CTA of 1024 threads): 16-bit buckets in groups of K, every group starts
-// at a multiple of 8; comp_start[b] = level-2 position of bucket b; the chunk table lists each
-// group (split into pieces of <= cap queries when larger); nch[0] = chunks, nch[1] = length.
-__global__ void __launch_bounds__(1024) k_l2_layout(const uint32_t* __restrict__ comp_cnt, uint32_t K, uint32_t cap,
-                                                    uint32_t* __restrict__ comp_start, uint2* __restrict__ chunks,
-                                                    uint32_t* __restrict__ chunk_pos, uint32_t* __restrict__ nch) {
-  __shared__ uint32_t tmp[1024 / 32 + 1];
-  const uint32_t ng = (kL2Buckets + K - 1) / K, gpt = (ng + 1023) / 1024;
-  const uint32_t g0 = min(ng, threadIdx.x * gpt), g1 = min(ng, g0 + gpt);
-  uint32_t padded = 0, pieces = 0, raw = 0;
-  for (uint32_t g = g0; g < g1; ++g) {
-    uint32_t sz = 0;
-    for (uint32_t b = g * K; b < min(kL2Buckets, (g + 1) * K); ++b) sz += comp_cnt[b];
-    padded += (sz + 7) & ~7u;
-    pieces += (sz + cap - 1) / cap;
-    raw += sz;
-  }
-  uint32_t tot_len, tot_ch, tot_raw;
-  uint32_t pos = block_scan<1024>(padded, tmp, &tot_len);
-  uint32_t ci = block_scan<1024>(pieces, tmp, &tot_ch);
-  uint32_t rpos = block_scan<1024>(raw, tmp, &tot_raw);
-  for (uint32_t g = g0; g < g1; ++g) {
-    uint32_t run = pos;
-    for (uint32_t b = g * K; b < min(kL2Buckets, (g + 1) * K); ++b) {
-      comp_start[b] = run;
-      run += comp_cnt[b];
-    }
-    const uint32_t sz = run - pos;
-    for (uint32_t o = 0; o < sz; o += cap) {
-      chunks[ci] = make_uint2(pos + o, min(cap, sz - o));
-      chunk_pos[ci++] = rpos + o;
-    }
-    pos += (sz + 7) & ~7u;
-    rpos += sz;
+// level-2 layout: 16-bit buckets in groups of K, every group starts at a multiple of 8;
+// comp_start[b] = level-2 position of bucket b; the chunk table lists each group (split into
+// pieces of <= cap queries when larger); nch[0] = chunks, nch[1] = padded length.  Three short
+// kernels (one thread per group): per-CTA scans, a scan of the CTA totals, then the writes.
+constexpr int kLayNT = 1024;
+__device__ __forceinline__ uint32_t l2_group_size(const uint32_t* __restrict__ comp_cnt, uint32_t g, uint32_t K) {
+  uint32_t sz = 0;
+  const uint32_t b1 = min(kL2Buckets, (g + 1) * K);
+  for (uint32_t b = g * K; b < b1; ++b) sz += __ldg(comp_cnt + b);
+  return sz;
+}
+// pass 1: per group (thread) its padded size, pieces and size; CTA-local exclusive prefixes
+// of the three go to gpre[3 x ng], the CTA totals to ctot[3 x nctas]
+__global__ void __launch_bounds__(kLayNT) k_l2_layout_a(const uint32_t* __restrict__ comp_cnt, uint32_t K, uint32_t cap,
+                                                        uint32_t* __restrict__ gpre, uint32_t* __restrict__ ctot) {
+  __shared__ uint32_t tmp[kLayNT / 32 + 1];
+  const uint32_t ng = (kL2Buckets + K - 1) / K, g = blockIdx.x * kLayNT + threadIdx.x;
+  const uint32_t sz = g < ng ? l2_group_size(comp_cnt, g, K) : 0;
+  uint32_t t0, t1, t2;
+  const uint32_t p0 = block_scan<kLayNT>((sz + 7) & ~7u, tmp, &t0);
+  const uint32_t p1 = block_scan<kLayNT>((sz + cap - 1) / cap, tmp, &t1);
+  const uint32_t p2 = block_scan<kLayNT>(sz, tmp, &t2);
+  if (g < ng) {
+    gpre[g] = p0;
+    gpre[ng + g] = p1;
+    gpre[2 * ng + g] = p2;
   }
   if (threadIdx.x == 0) {
-    comp_start[kL2Buckets] = tot_len;
-    nch[0] = tot_ch;
-    nch[1] = tot_len;
+    ctot[blockIdx.x] = t0;
+    ctot[gridDim.x + blockIdx.x] = t1;
+    ctot[2 * gridDim.x + blockIdx.x] = t2;
+  }
+}
+// pass 2 (one CTA): exclusive scans of the CTA totals in place; the grand totals to nch
+__global__ void __launch_bounds__(kLayNT) k_l2_layout_b(uint32_t* __restrict__ ctot, uint32_t nctas,
+                                                        uint32_t* __restrict__ nch) {
+  __shared__ uint32_t tmp[kLayNT / 32 + 1];
+  for (int k = 0; k < 3; ++k) {
+    const uint32_t v = threadIdx.x < nctas ? ctot[k * nctas + threadIdx.x] : 0;
+    uint32_t tot;
+    const uint32_t ex = block_scan<kLayNT>(v, tmp, &tot);
+    if (threadIdx.x < nctas) ctot[k * nctas + threadIdx.x] = ex;
+    if (threadIdx.x == 0 && k == 0) nch[1] = tot;
+    if (threadIdx.x == 0 && k == 1) nch[0] = tot;
+  }
+}
+// pass 3: bucket positions and the group's chunk entries
+__global__ void __launch_bounds__(kLayNT) k_l2_layout_c(const uint32_t* __restrict__ comp_cnt, uint32_t K, uint32_t cap,
+                                                        const uint32_t* __restrict__ gpre,
+                                                        const uint32_t* __restrict__ ctot,
+                                                        uint32_t* __restrict__ comp_start, uint2* __restrict__ chunks,
+                                                        uint32_t* __restrict__ chunk_pos, const uint32_t* __restrict__ nch) {
+  const uint32_t ng = (kL2Buckets + K - 1) / K, g = blockIdx.x * kLayNT + threadIdx.x;
+  if (g == 0) comp_start[kL2Buckets] = nch[1];
+  if (g >= ng) return;
+  const uint32_t nct = gridDim.x;
+  const uint32_t pos = gpre[g] + ctot[blockIdx.x];
+  uint32_t ci = gpre[ng + g] + ctot[nct + blockIdx.x];
+  const uint32_t rpos = gpre[2 * ng + g] + ctot[2 * nct + blockIdx.x];
+  uint32_t run = pos;
+  const uint32_t b1 = min(kL2Buckets, (g + 1) * K);
+  for (uint32_t b = g * K; b < b1; ++b) {
+    comp_start[b] = run;
+    run += __ldg(comp_cnt + b);
+  }
+  const uint32_t sz = run - pos;
+  for (uint32_t o = 0; o < sz; o += cap) {
+    chunks[ci] = make_uint2(pos + o, min(cap, sz - o));
+    chunk_pos[ci++] = rpos + o;
   }
 }
 
@@ -960,7 +990,13 @@ harmonia_status psa_partition2_l2(const uint64_t* q, uint64_t n, const BucketBit
   {
     ProfScope ps_(HARMONIA_PROF_PSA_SCAN, st);
     k_l2_colsum<<<256, 256, 0, st>>>(ws.seg, ws.tile_counts2, ws.comp_cnt);
-    k_l2_layout<<<1, 1024, 0, st>>>(ws.comp_cnt, K, cap, ws.comp_start, ws.chunks, ws.chunk_pos, ws.nchunks);
+    const uint32_t ng = (kL2Buckets + K - 1) / K, nct = (ng + kLayNT - 1) / kLayNT;  // nct <= 64
+    uint32_t* gpre = ws.l2_scratch;
+    uint32_t* ctot = ws.seg + 2 * 257;
+    k_l2_layout_a<<<nct, kLayNT, 0, st>>>(ws.comp_cnt, K, cap, gpre, ctot);
+    k_l2_layout_b<<<1, kLayNT, 0, st>>>(ctot, nct, ws.nchunks);
+    k_l2_layout_c<<<nct, kLayNT, 0, st>>>(ws.comp_cnt, K, cap, gpre, ctot, ws.comp_start, ws.chunks, ws.chunk_pos,
+                                          ws.nchunks);
     k_l2_tilebase<<<256, 256, 0, st>>>(ws.seg, ws.tile_counts2, ws.comp_start, ws.tile_base2);
   }
   HM_LAUNCHED();

@@ -408,3 +408,29 @@ def test_l2_access_policy_window(hm, orc):
     ko, vo, cnt = t.range(cu(lo), cu(hi), 64)
     eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, 64)
     assert np.array_equal(host(cnt), ecnt) and np.array_equal(host(ko), eko) and np.array_equal(host(vo), evo)
+
+
+def test_concurrent_streams_separate_workspaces(hm, orc):
+    """Searches on two streams at once each get their own workspace (the C ABI needs one per
+    stream): interleaved calls on the same Tree return exact results on both streams."""
+    import torch
+
+    keys = gen.uniform_keys(1 << 18)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 64)
+    qa = gen.uniform_queries(keys, (1 << 21) + 3, miss_frac=0.2)
+    qb = gen.uniform_queries(keys, (1 << 20) + 11, seed=gen.SEED_QUERY + 5, miss_frac=0.3)
+    da, db = cu(qa), cu(qb)
+    sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    outs = []
+    for _ in range(3):
+        with torch.cuda.stream(sa):
+            oa = t.search(da, stream=sa)
+        with torch.cuda.stream(sb):
+            ob = t.search(db, stream=sb)
+        outs.append((oa, ob))
+    torch.cuda.synchronize()
+    ea, eb = orc.sorted_search(keys, vals, qa), orc.sorted_search(keys, vals, qb)
+    for oa, ob in outs:
+        assert np.array_equal(host(oa), ea) and np.array_equal(host(ob), eb)

@@ -1,7 +1,9 @@
 #!/bin/bash
-for lt in 23 26; do
-  AB_ROOT=tools/bin/r1repo PYTHONPATH=tools/bin/r1repo python tools/ab_search.py $lt 26 r1
-  python tools/ab_search.py $lt 26 cur
+# A/B of library variants (tools/bin/*.so, tools/build_variant.py) on one box: c2 and c4 step
+# and kernel times.   bash tools/gpu_ab.sh "variant1 variant2 ..."
+for v in cur $1; do
+  for cfg in c2 c4; do
+    if [ "$v" = cur ]; then python tools/exp_l16.py $cfg 2>&1 | grep auto | sed "s/^/$v /";
+    else HARMONIA_LIB=tools/bin/$v.so python tools/exp_l16.py $cfg 2>&1 | grep auto | sed "s/^/$v /"; fi
+  done
 done
-python tools/exp_l16.py c4
-python -m pytest -x -q tests/test_gpu_psa.py tests/test_gpu_search.py 2>&1 | tail -2
