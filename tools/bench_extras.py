@@ -71,7 +71,7 @@ def range_bench(T=1 << 23, F=64, reps=5, groups=(0,), flags=0):
             ok = bool((cnt == length).all())  # lo = key[p], hi = key[p+len-1]: exactly len records
             res.append({"what": "range_batch", "T": T, "F": F, "G": G, "len": length, "Qr": Qr, "ms": ms,
                         "kernel": ("group" if (G or flags & (hm.QF_RANGE_GROUP | hm.QF_NO_RANGE_LANE)) else
-                                   ("lane" if length < 128 else "warp")), "counts_ok": ok,
+                                   ("lane" if length < 512 else "warp")), "counts_ok": ok,
                         "Gq_per_s": Qr / ms / 1e6, "G_records_per_s": Qr * length / ms / 1e6,
                         "GB_per_s_out": Qr * length * 16 / ms / 1e6})
             print(json.dumps(res[-1]), flush=True)
