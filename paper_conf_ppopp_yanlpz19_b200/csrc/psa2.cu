@@ -443,20 +443,26 @@ __global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? HM_UNMOVE_MINB : C::M
     if (HM_UNMOVE_TMA_STORE && threadIdx.x == 0) bulk_store_wait_read();  // st_r free again
     __syncthreads();
     const uint32_t tile_n = (uint32_t)std::min<uint64_t>(C::TILE, n - t0);
-    uint64_t rv[C::PER];
-    uint32_t oo[C::PER];
+    // rounds of <= 8 slots per thread: all loads of a round in flight before its stores (16
+    // per thread at 4096-query tiles spilled past the 64-register cap)
+    constexpr int R = C::PER < 8 ? C::PER : 8;
 #pragma unroll
-    for (int k = 0; k < C::PER; ++k) {  // all loads in flight before the stores
-      const uint32_t i = k * C::NT + threadIdx.x;
-      if (i < tile_n) {
-        const uint32_t od = st_od[i], dd = od >> C::TILE_SHIFT;
-        oo[k] = od & (C::TILE - 1);
-        rv[k] = __ldg(res1 + gbase[dd] + (i - bin_start[dd]));
+    for (int k0 = 0; k0 < C::PER; k0 += R) {
+      uint64_t rv[R];
+      uint32_t oo[R];
+#pragma unroll
+      for (int k = 0; k < R; ++k) {
+        const uint32_t i = (k0 + k) * C::NT + threadIdx.x;
+        if (i < tile_n) {
+          const uint32_t od = st_od[i], dd = od >> C::TILE_SHIFT;
+          oo[k] = od & (C::TILE - 1);
+          rv[k] = __ldg(res1 + gbase[dd] + (i - bin_start[dd]));
+        }
       }
-    }
 #pragma unroll
-    for (int k = 0; k < C::PER; ++k)
-      if (k * C::NT + threadIdx.x < tile_n) st_r[oo[k]] = rv[k];
+      for (int k = 0; k < R; ++k)
+        if ((k0 + k) * C::NT + threadIdx.x < tile_n) st_r[oo[k]] = rv[k];
+    }
     // TMA store of a full tile (one thread, async); the next tile's st_r writes wait above
     const bool tma = HM_UNMOVE_TMA_STORE && tile_n == (uint32_t)C::TILE && ((uintptr_t)(out + t0) & 15) == 0;
     if (tma) fence_proxy_async_smem();
@@ -486,7 +492,12 @@ constexpr size_t unmove_smem() {
 // Plan::l2_group consecutive buckets, each group padded to a multiple of 8 slots), which makes
 // the whole window sorted by all Nb bits.  Tile bases are computed by per-segment column scans
 // (deterministic; no global atomics).
-using L2C = L1Cfg<8, 2048, 256>;
+#ifndef HM_L2_TILE
+#define HM_L2_TILE 4096  // measured: 4096-query tiles (runs of ~16) beat 2048 in the two-level path
+#endif
+using L2C = L1Cfg<8, HM_L2_TILE, 256>;
+// the two-level path's level 1 uses the same tile (its moves gain more than its unmoves lose)
+using Narrow4 = L1Cfg<8, HM_L2_TILE, 256>;
 
 struct L2Digit {
   BucketBits f;
@@ -717,8 +728,9 @@ __global__ void __launch_bounds__(L2C::NT, HM_UNMOVE_MINB) k_psa2_unmove_s(const
                                                                            const uint64_t* __restrict__ res2,
                                                                            uint64_t* __restrict__ res1) {
   __shared__ uint32_t s_seg[2 * 257];
-  __shared__ __align__(16) uint64_t st_r[L2C::TILE];
-  __shared__ uint32_t st_od[L2C::TILE];
+  extern __shared__ __align__(16) unsigned char l2u_smem[];
+  uint64_t* st_r = reinterpret_cast<uint64_t*>(l2u_smem);                      // TILE results
+  uint32_t* st_od = reinterpret_cast<uint32_t*>(l2u_smem + L2C::TILE * 8);     // TILE offsets | digit
   __shared__ uint32_t bin_start[L2C::BINS], gbase[L2C::BINS], tmp[L2C::NT / 32 + 1];
   l2_load_seg(s_seg, seg);
   uint32_t tb, te;
@@ -740,28 +752,33 @@ __global__ void __launch_bounds__(L2C::NT, HM_UNMOVE_MINB) k_psa2_unmove_s(const
 #pragma unroll
     for (int k = 0; k < L2C::PER; ++k) {
       const uint32_t i = k * L2C::NT + threadIdx.x;
-      if (i < len) st_od[bin_start[pk[k] & 255u] + (pk[k] >> 8)] = i | ((pk[k] & 255u) << 11);
+      if (i < len) st_od[bin_start[pk[k] & 255u] + (pk[k] >> 8)] = i | ((pk[k] & 255u) << L2C::TILE_SHIFT);
     }
     __syncthreads();
-    uint64_t rv[L2C::PER];
-    uint32_t oo[L2C::PER];
+    constexpr int R = L2C::PER < 8 ? L2C::PER : 8;  // rounds: loads in flight before the stores
 #pragma unroll
-    for (int k = 0; k < L2C::PER; ++k) {  // all loads in flight before the shared stores
-      const uint32_t i = k * L2C::NT + threadIdx.x;
-      if (i < len) {
-        const uint32_t od = st_od[i], d = od >> 11;
-        oo[k] = od & (L2C::TILE - 1);
-        rv[k] = __ldg(res2 + gbase[d] + (i - bin_start[d]));
+    for (int k0 = 0; k0 < L2C::PER; k0 += R) {
+      uint64_t rv[R];
+      uint32_t oo[R];
+#pragma unroll
+      for (int k = 0; k < R; ++k) {
+        const uint32_t i = (k0 + k) * L2C::NT + threadIdx.x;
+        if (i < len) {
+          const uint32_t od = st_od[i], d = od >> L2C::TILE_SHIFT;
+          oo[k] = od & (L2C::TILE - 1);
+          rv[k] = __ldg(res2 + gbase[d] + (i - bin_start[d]));
+        }
       }
-    }
 #pragma unroll
-    for (int k = 0; k < L2C::PER; ++k)
-      if (k * L2C::NT + threadIdx.x < len) st_r[oo[k]] = rv[k];
+      for (int k = 0; k < R; ++k)
+        if ((k0 + k) * L2C::NT + threadIdx.x < len) st_r[oo[k]] = rv[k];
+    }
     __syncthreads();
     for (uint32_t i = threadIdx.x; i < len; i += L2C::NT) res1[t0 + i] = st_r[i];
     __syncthreads();
   }
 }
+constexpr size_t kUnmoveSSmem = (size_t)L2C::TILE * 12;
 
 // the queries of the level-2 chunks, pads skipped, in the order the search visits them
 // (harmonia_psa_inspect)
@@ -977,7 +994,7 @@ harmonia_status psa_partition2_l2(const uint64_t* q, uint64_t n, const BucketBit
                                   cudaStream_t st, uint32_t K, uint32_t cap) {
   if (nb < 16 || (cap != kPsaChunk && cap != kPsaChunkMax)) return HARMONIA_ERR_INVALID_ARG;
   harmonia_status s =
-      coarse_partition<Narrow>(q, n, CoarseDigit{f, (uint32_t)nb - 8}, ws, ws.sorted_q, nullptr, sm, st, nullptr, 0);
+      coarse_partition<Narrow4>(q, n, CoarseDigit{f, (uint32_t)nb - 8}, ws, ws.sorted_q, nullptr, sm, st, nullptr, 0);
   if (s != HARMONIA_OK) return s;
   const L2Digit dg{f, (uint32_t)nb - 16};
   const int g = l1_grid<L2C>(n + 256ull * L2C::TILE, sm), gm = l1_grid_mv<L2C>(n + 256ull * L2C::TILE, sm);
@@ -1032,11 +1049,12 @@ harmonia_status psa_unpartition2_l2(const PsaWs& ws, const uint64_t* res2, uint6
   if (n == 0) return HARMONIA_OK;
   {
     ProfScope ps_(HARMONIA_PROF_RETURN, st);
-    k_psa2_unmove_s<<<l1_grid_mv<L2C>(n + 256ull * L2C::TILE, sm), L2C::NT, 0, st>>>(
+    HM_CUDA(smem_attr(k_psa2_unmove_s, kUnmoveSSmem));
+    k_psa2_unmove_s<<<l1_grid_mv<L2C>(n + 256ull * L2C::TILE, sm), L2C::NT, kUnmoveSSmem, st>>>(
         ws.seg, ws.packed2, ws.tile_counts2, ws.tile_base2, res2, ws.sorted_q);
   }
   HM_LAUNCHED();
-  return unpartition<Narrow>(ws, ws.sorted_q, n, out, sm, st);
+  return unpartition<Narrow4>(ws, ws.sorted_q, n, out, sm, st);
 }
 
 // harmonia_psa_inspect: the queries of the search's chunks in visiting order (two-level PSA)
