@@ -166,3 +166,39 @@ def test_range_split_assemble_single_process(hm, orc, P, cap):
         gk, gv = _np(ko).reshape(-1, cap), _np(vo).reshape(-1, cap)
         assert np.array_equal(gk[mk], eko.reshape(-1, cap)[mk]) and np.array_equal(gv[mk], evo.reshape(-1, cap)[mk])
         assert np.all(gk[~mk] == np.uint64((1 << 64) - 1))
+
+
+def test_partitioned_single_rank_with_updates(hm, orc):
+    """Config 5's loop at N = 1 on the GPU: a one-rank NCCL group, PartitionedTree (routing
+    bypassed at P = 1) over a fill-0.69 shard, query batches interleaved with 5 % insert / 5 %
+    delete / 90 % update batches (in place), every batch checked against the std::map oracle."""
+    import torch.distributed as dist
+
+    from paper_conf_ppopp_yanlpz19_b200.dist import PartitionedTree
+
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1,
+                            device_id=torch.device("cuda", 0))
+    try:
+        keys = gen.uniform_keys(1 << 18)
+        vals = gen.values_for(keys)
+        pt = PartitionedTree(_u64(keys), _u64(vals), [], fanout=64, fill=0.69, device=torch.device("cuda", 0))
+        ref = orc.UpdateMap(keys, vals)
+        modes = []
+        for b in range(4):
+            rk, rv = ref.dump()
+            q = gen.uniform_queries(rk, 300000, seed=gen.SEED_QUERY + b, miss_frac=0.2)
+            assert np.array_equal(_np(pt.search(_u64(q))), orc.sorted_search(rk, rv, q))
+            ops, ks, vs = gen.update_ops(rk, 20000, insert_frac=0.05, delete_frac=0.05, seed=gen.SEED_OPS + b)
+            pt.update(torch.from_numpy(ops).cuda(), _u64(ks), _u64(vs))
+            modes.append(pt.ops.tree.last_update_mode())
+            ref.apply(ops, ks, vs)
+        rk, rv = ref.dump()
+        q = np.concatenate([rk, gen.edge_queries(rk)])
+        assert np.array_equal(_np(pt.search(_u64(q))), orc.sorted_search(rk, rv, q))
+        assert modes.count(1) >= 3, modes
+    finally:
+        dist.destroy_process_group()
