@@ -457,9 +457,15 @@ __device__ __forceinline__ void ld_quad_global(const uint64_t* p, uint64_t (&k)[
 // then the TL-key block [r, r+TL) is read with TL/4 independent 256-bit loads and counted
 // (keys below r are <= q, keys from r+TL on are > q, so r + #(block <= q) is the rank).
 // log2(F/TL) + 1 dependent round trips instead of log2(F).  best = the last key <= q.
+__device__ __forceinline__ void prefetch_l1(const void* p) { asm volatile("prefetch.global.L1 [%0];" ::"l"(p)); }
+// vrow (leaf probe, two-level PSA kernels): value row of node 0 (values of node n at vrow + n*F);
+// once the rank is known to a 16-slot block, that block's value line is prefetched into L1 so
+// the final value load does not wait for another L2 round trip (measured: c4 search −5 %; with
+// one PSA level the extra L1 requests cost more than the saved round trip, c2 +2 %, c3 +10 %)
 template <int F, int U, int TL>
 __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint32_t (&node)[U],
-                                               const uint64_t (&q)[U], uint32_t (&r)[U], uint64_t (&best)[U]) {
+                                               const uint64_t (&q)[U], uint32_t (&r)[U], uint64_t (&best)[U],
+                                               const uint64_t* vrow = nullptr) {
 #pragma unroll
   for (int s = F / 2; s >= TL; s >>= 1) {
     uint64_t k[U];
@@ -470,6 +476,10 @@ __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint3
       const bool le = k[u] <= q[u];
       r[u] += le ? s : 0;
       best[u] = le ? k[u] : best[u];
+    }
+    if (vrow && s == 16 && F >= 32) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) prefetch_l1(vrow + (uint64_t)node[u] * F + r[u]);
     }
   }
   uint64_t k[U][TL];
@@ -498,7 +508,7 @@ __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint3
 // one lane, U interleaved queries, from level l0 at nodes node[]: descent (Eq 1) + leaf probe
 // RANK: instead of the value, res = (leaf index << 32) | #keys <= q in that leaf (the range
 // kernels turn it into a global record rank with leaf_base)
-template <int F, int U, bool RANK = false>
+template <int F, int U, bool RANK = false, bool PF = false>
 __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                              bool ps_smem, bool leaf_smem, uint32_t l0, uint32_t (&node)[U],
                                              const uint64_t (&q)[U], const bool (&live)[U], uint64_t (&res)[U]) {
@@ -550,7 +560,8 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
   }
 #if HM_LEAF_TAIL > 0
   if (F >= 2 * HM_LEAF_TAIL && !leaf_smem) {
-    lane_rank_tail<F, U, (F >= 2 * HM_LEAF_TAIL ? HM_LEAF_TAIL : 4)>(a.keys, node, q, r, best);
+    lane_rank_tail<F, U, (F >= 2 * HM_LEAF_TAIL ? HM_LEAF_TAIL : 4)>(
+        a.keys, node, q, r, best, PF && !RANK ? a.vals - (uint64_t)a.leaf_start * F : nullptr);
   } else
 #endif
   {
@@ -723,7 +734,7 @@ __device__ __forceinline__ void chunk_path(const SearchArgs& a, const uint64_t* 
   }
 }
 
-template <int F, int U, bool RANK = false>
+template <int F, int U, bool RANK = false, bool PF = false>
 __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
                                           bool ps_smem, bool leaf_smem, const uint64_t (&q0)[U],
                                           const bool (&act)[U], uint64_t (&res)[U], uint32_t node0 = 0,
@@ -772,7 +783,7 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
     else window_rank<F, U, false>(a.keys, off, q, rlo, rhi, r, best);
 #pragma unroll
     for (int u = 0; u < U; ++u) nd[u] = first + r[u];
-    lane_descend<F, U, RANK>(a, s_keys, s_ps, ps_smem, leaf_smem, l + 1, nd, q, live, res);
+    lane_descend<F, U, RANK, PF>(a, s_keys, s_ps, ps_smem, leaf_smem, l + 1, nd, q, live, res);
     return;
   }
   // the whole warp reached the same leaf
@@ -872,7 +883,7 @@ __global__ void __launch_bounds__(HM_SEARCH_NT, 2) k_lane_search_c(const SearchA
       }
       uint64_t res[U];
       if constexpr (COOP && TAB) {
-        warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res, node0, lev0);
+        warp_core<F, U, false, true>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res, node0, lev0);
       } else if constexpr (COOP) {
         warp_core<F, U>(a, s_keys, s_ps, ps_smem, leaf_smem, q0, act, res);
       } else {
