@@ -31,6 +31,15 @@ namespace hm {
 #ifndef HM_UNMOVE_MINB
 #define HM_UNMOVE_MINB 4
 #endif
+// 4096-query tiles (the two-level path, both levels): 3 resident CTAs per SM, so the 16
+// queries per thread fit in registers (at 4 the 64-register cap spilled; c4 move 1.16 -> 1.08
+// ms, return 1.41 -> 1.27 ms; the 2048-query tiles of the one-level path keep 4)
+#ifndef HM_MOVE_MINB4
+#define HM_MOVE_MINB4 3
+#endif
+#ifndef HM_UNMOVE_MINB4
+#define HM_UNMOVE_MINB4 3
+#endif
 #ifndef HM_L1_WAVES
 #define HM_L1_WAVES 6
 #endif
@@ -40,20 +49,12 @@ namespace hm {
 
 namespace {
 
-constexpr int kBatches = 8;                              // 32-query batches per warp per tile
-constexpr int kCoarseTile = kBlock * kBatches;           // 2048 queries per scatter tile
 #ifndef HM_SORT_THREADS
 #define HM_SORT_THREADS 512
 #endif
-constexpr int kSortThreads = HM_SORT_THREADS, kSortWarps = kSortThreads / 32;
+constexpr int kSortThreads = HM_SORT_THREADS;
 constexpr int kChunk = (int)kPsaChunk;                   // queries per chunk-sort chunk (4096)
 constexpr int kLocalBits = 11;                           // chunk sort: 2048 local buckets
-
-__device__ __forceinline__ unsigned lane_lt() {
-  unsigned m;
-  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
-  return m;
-}
 
 // exclusive scan of one value per thread (NT threads); `tmp` needs NT/32 + 1 words
 template <int NT>
@@ -246,7 +247,7 @@ __global__ void __launch_bounds__(C::NT, C::MINB) k_psa2_rank(const uint64_t* __
 // straight into the receive buffer of rank d (a peer-mapped device pointer, NVLink stores),
 // push_dst[d] = address of this rank's segment there; nothing is written locally.
 template <class Digit, class C, bool kIdx, bool kPush = false>
-__global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? HM_MOVE_MINB : C::MINB)) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
+__global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? (C::TILE == 4096 ? HM_MOVE_MINB4 : HM_MOVE_MINB) : C::MINB)) k_psa2_move(const uint64_t* __restrict__ q, uint64_t n, Digit dg,
                                                               const uint32_t* __restrict__ counts,
                                                               uint32_t* __restrict__ cursor,
                                                               const uint32_t* __restrict__ tile_counts,
@@ -379,7 +380,7 @@ constexpr size_t move_smem() {
 // gbase rebuilt from the CTA base, so res1 is read in runs and out[] written contiguously --
 // no scattered global access on either side.
 template <class C>
-__global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? HM_UNMOVE_MINB : C::MINB)) k_psa2_unmove(const uint32_t* __restrict__ tile_counts,
+__global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? (C::TILE == 4096 ? HM_UNMOVE_MINB4 : HM_UNMOVE_MINB) : C::MINB)) k_psa2_unmove(const uint32_t* __restrict__ tile_counts,
                                                                 const uint32_t* __restrict__ cta_base,
                                                                 const uint32_t* __restrict__ packed,
                                                                 const uint64_t* __restrict__ res1, uint64_t n,
@@ -445,7 +446,10 @@ __global__ void __launch_bounds__(C::NT, (C::BINS == 256 ? HM_UNMOVE_MINB : C::M
     const uint32_t tile_n = (uint32_t)std::min<uint64_t>(C::TILE, n - t0);
     // rounds of <= 8 slots per thread: all loads of a round in flight before its stores (16
     // per thread at 4096-query tiles spilled past the 64-register cap)
-    constexpr int R = C::PER < 8 ? C::PER : 8;
+#ifndef HM_UNMOVE_R
+#define HM_UNMOVE_R 8
+#endif
+    constexpr int R = C::PER < HM_UNMOVE_R ? C::PER : HM_UNMOVE_R;
 #pragma unroll
     for (int k0 = 0; k0 < C::PER; k0 += R) {
       uint64_t rv[R];
@@ -676,7 +680,7 @@ __global__ void __launch_bounds__(256) k_l2_tilebase(const uint32_t* __restrict_
 }
 
 // staged move of every level-2 tile: level-1 order -> level-2 order (runs by consecutive lanes)
-__global__ void __launch_bounds__(L2C::NT, HM_MOVE_MINB) k_psa2_move_s(const uint64_t* __restrict__ q1, L2Digit dg,
+__global__ void __launch_bounds__(L2C::NT, (L2C::TILE == 4096 ? HM_MOVE_MINB4 : HM_MOVE_MINB)) k_psa2_move_s(const uint64_t* __restrict__ q1, L2Digit dg,
                                                                        const uint32_t* __restrict__ seg,
                                                                        const uint32_t* __restrict__ packed2,
                                                                        const uint32_t* __restrict__ tile_counts2,
@@ -721,7 +725,7 @@ __global__ void __launch_bounds__(L2C::NT, HM_MOVE_MINB) k_psa2_move_s(const uin
 
 // inverse of k_psa2_move_s: res1[level-1 position] = res2[level-2 position]; reads res2 in
 // runs, writes res1 contiguously
-__global__ void __launch_bounds__(L2C::NT, HM_UNMOVE_MINB) k_psa2_unmove_s(const uint32_t* __restrict__ seg,
+__global__ void __launch_bounds__(L2C::NT, (L2C::TILE == 4096 ? HM_UNMOVE_MINB4 : HM_UNMOVE_MINB)) k_psa2_unmove_s(const uint32_t* __restrict__ seg,
                                                                            const uint32_t* __restrict__ packed2,
                                                                            const uint32_t* __restrict__ tile_counts2,
                                                                            const uint32_t* __restrict__ tile_base2,
