@@ -353,7 +353,9 @@ class Tree:
         return out
 
     def search_host(self, q_host, out_host=None, *, opts: QueryOpts | None = None, stream=None, **kw):
-        """End-to-end point queries from host memory (pinned CPU tensors for overlap)."""
+        """End-to-end point queries from host memory (pinned CPU tensors for overlap).
+        Asynchronous on `stream`, like harmonia_search_batch_host: synchronise the stream
+        before reading the returned host buffer."""
         torch = _torch()
         if isinstance(q_host, np.ndarray):
             q_host = torch.from_numpy(np.ascontiguousarray(q_host.astype(np.uint64, copy=False)))
