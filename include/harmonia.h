@@ -299,6 +299,18 @@ harmonia_status harmonia_scatter_results(const uint64_t* d_routed_values, const 
  *   handle_out) for the other ranks; harmonia_peer_open maps a peer's handle into this
  *   process (cudaIpcOpenMemHandle, lazy peer access); harmonia_peer_close unmaps it;
  *   harmonia_peer_free releases an own buffer.  Setup-time calls, never on a query path.
+ *   Buffers from harmonia_peer_alloc are zero-filled.
+ * harmonia_peer_barrier: device-side barrier of the P ranks of the fused routing (steps 4's
+ *   "barrier"; no host thread waits).  d_flag_addrs[P] (device array): the address of rank p's
+ *   flag array (P uint64, a harmonia_peer_alloc buffer, mapped into this process with
+ *   harmonia_peer_open; this rank's own for p = me); d_my_flags: this rank's own flag array.
+ *   Every rank calls it with the same strictly increasing epoch (1, 2, ...).  The kernel
+ *   stores `epoch` to slot `me` of every rank's flags (system-scope fence + release store, so
+ *   the stores of this rank's earlier work on `stream` -- its pushed runs -- are visible
+ *   first) and returns when every rank's slot in d_my_flags holds >= epoch (system-scope
+ *   acquire), so the work queued after it on `stream` sees every peer's pushes.  After
+ *   timeout_ns (0: 30 s) without all flags, it sets *d_error = 1 and returns (the caller
+ *   checks d_error; the batch's results are then invalid).  Asynchronous; P <= 256.
  * ------------------------------------------------------------------------------------- */
 harmonia_status harmonia_route_count(const uint64_t* d_splitters, uint32_t P, const uint64_t* d_queries,
                                      uint64_t n, uint64_t* h_counts, void* d_workspace,
@@ -348,6 +360,8 @@ harmonia_status harmonia_peer_alloc(size_t bytes, void** d_ptr, void* handle_out
 harmonia_status harmonia_peer_open(const void* handle, void** d_ptr);
 harmonia_status harmonia_peer_close(void* d_ptr);
 harmonia_status harmonia_peer_free(void* d_ptr);
+harmonia_status harmonia_peer_barrier(uint32_t P, uint32_t me, const uint64_t* d_flag_addrs, uint64_t* d_my_flags,
+                                      uint64_t epoch, uint32_t* d_error, uint64_t timeout_ns, void* stream);
 
 /* The plan a search/range call with these options would use (for reporting). */
 typedef struct {

@@ -123,6 +123,7 @@ def lib():
             "harmonia_peer_open": (C.c_int, [_vp, C.POINTER(_vp)]),
             "harmonia_peer_close": (C.c_int, [_vp]),
             "harmonia_peer_free": (C.c_int, [_vp]),
+            "harmonia_peer_barrier": (C.c_int, [C.c_uint32, C.c_uint32, _vp, _vp, _u64, _vp, _u64, _vp]),
             "harmonia_psa_bits_auto": (C.c_int32, [_u64]),
             "harmonia_ntg_choose": (C.c_int, [_vp, _vp, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
                                               C.c_uint32, C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
@@ -548,6 +549,14 @@ class PeerBuffer:
         if self.ptr.value:
             _check(lib().harmonia_peer_free(self.ptr), "harmonia_peer_free")
             self.ptr = C.c_void_p()
+
+
+def peer_barrier(P: int, me: int, flag_addrs, my_flags_addr: int, epoch: int, error, timeout_ns: int = 0,
+                 stream=None):
+    """harmonia_peer_barrier: device-side barrier of the fused routing (asynchronous; `flag_addrs`
+    a device uint64 tensor of the P ranks' flag-array addresses, `error` a device int32[1])."""
+    _check(lib().harmonia_peer_barrier(P, me, flag_addrs.data_ptr(), my_flags_addr, epoch, error.data_ptr(),
+                                       timeout_ns, _stream_ptr(stream, error.device)), "harmonia_peer_barrier")
 
 
 # ----------------------------------------------------------------------------- range routing

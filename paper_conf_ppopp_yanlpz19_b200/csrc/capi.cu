@@ -704,6 +704,11 @@ extern "C" harmonia_status harmonia_peer_alloc(size_t bytes, void** d_ptr, void*
     return HARMONIA_ERR_OUT_OF_MEMORY;
   }
   HM_CUDA(e);
+  e = cudaMemset(p, 0, bytes);  // zero-filled (the peer barrier's flags start at epoch 0)
+  if (e != cudaSuccess) {
+    cudaFree(p);
+    return cuda_fail(e);
+  }
   cudaIpcMemHandle_t h;
   e = cudaIpcGetMemHandle(&h, p);
   if (e != cudaSuccess) {
@@ -712,6 +717,54 @@ extern "C" harmonia_status harmonia_peer_alloc(size_t bytes, void** d_ptr, void*
   }
   std::memcpy(handle_out, &h, sizeof(h));
   *d_ptr = p;
+  return HARMONIA_OK;
+}
+
+// ---- device-side barrier over peer memory (replaces the host barrier of the fused routing) ----
+// Thread p (< P) publishes `epoch` into slot `me` of rank p's flag array (fence.sc.sys, then a
+// system-scope release store: every store this rank's earlier kernels made on the stream --
+// the pushed runs -- is visible to p before the flag), then spins with system-scope acquire
+// loads until rank p's flag in this rank's array reaches `epoch`.  The kernels after it on the
+// stream (the search of the receive buffer, the inverse partition) therefore see every peer's
+// pushes, and no host thread waits.  A wait longer than timeout_ns sets *d_error = 1 and ends
+// the kernel instead of hanging the device.
+namespace hm_peer {
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__global__ void __launch_bounds__(256) k_peer_barrier(uint32_t P, uint32_t me, const uint64_t* __restrict__ flag_addrs,
+                                                      const uint64_t* my_flags, uint64_t epoch, uint32_t* err,
+                                                      uint64_t timeout_ns) {
+  const uint32_t p = threadIdx.x;
+  if (p >= P) return;
+  uint64_t* f = reinterpret_cast<uint64_t*>(flag_addrs[p]) + me;
+  asm volatile("fence.sc.sys;" ::: "memory");
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(epoch) : "memory");
+  const uint64_t t0 = globaltimer_ns();
+  for (;;) {
+    uint64_t v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(my_flags + p) : "memory");
+    if (v >= epoch) break;
+    if (globaltimer_ns() - t0 > timeout_ns) {
+      atomicExch(err, 1u);
+      break;
+    }
+    __nanosleep(256);
+  }
+}
+}  // namespace hm_peer
+
+extern "C" harmonia_status harmonia_peer_barrier(uint32_t P, uint32_t me, const uint64_t* d_flag_addrs,
+                                                 uint64_t* d_my_flags, uint64_t epoch, uint32_t* d_error,
+                                                 uint64_t timeout_ns, void* stream) {
+  if (P == 0 || P > 256 || me >= P || !d_flag_addrs || !d_my_flags || !d_error || epoch == 0)
+    return HARMONIA_ERR_INVALID_ARG;
+  hm_peer::k_peer_barrier<<<1, 256, 0, (cudaStream_t)stream>>>(P, me, d_flag_addrs, d_my_flags, epoch, d_error,
+                                                      timeout_ns ? timeout_ns : 30ull * 1000000000ull);
+  count_launch();
+  HM_CUDA(cudaGetLastError());
   return HARMONIA_OK;
 }
 

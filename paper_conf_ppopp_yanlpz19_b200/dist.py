@@ -13,10 +13,12 @@ PartitionedTree  rank p owns the keys in [splitter[p-1], splitter[p]) (key quant
 PeerPartitionedTree  the same shards with the exchange fused into the kernels over peer memory
                  (no NCCL data collective): harmonia_route_count -> all_gather of the P x P count
                  matrix -> harmonia_route_push writes every destination's run straight into
-                 that rank's receive buffer (CUDA IPC mapping, NVLink stores) -> barrier ->
-                 local search of the receive buffer -> harmonia_segments_push returns every
-                 source's results into its "back" buffer -> barrier -> harmonia_route_return
-                 (inverse partition) restores the caller's order.
+                 that rank's receive buffer (CUDA IPC mapping, NVLink stores) -> device
+                 barrier -> local search of the receive buffer -> harmonia_segments_push
+                 returns every source's results into its "back" buffer -> device barrier ->
+                 harmonia_route_return (inverse partition) restores the caller's order.  The
+                 barriers are harmonia_peer_barrier kernels (flags in peer memory, system-scope
+                 release/acquire): the only host wait per batch is the count matrix.
 
 The per-device steps go through a small `ops` object so that the exchange logic can be
 tested on CPU with a gloo group (tests/test_dist.py injects CPU stand-ins); the default ops
@@ -310,13 +312,19 @@ def peer_offsets(M, me: int):
 class CudaPeerOps:
     """Device steps and peer buffers of PeerPartitionedTree (libharmonia.so kernels, CUDA IPC)."""
 
-    def __init__(self, tree: Tree, splitters: torch.Tensor, P: int, group=None):
+    def __init__(self, tree: Tree, splitters: torch.Tensor, P: int, group=None, device_barrier: bool = True):
         self.tree, self.split, self.P, self.group = tree, splitters, P, group
         self.dev = tree.device
         self.recv = self.back = None
         self.recv_addr, self.back_addr = [], []
         self.cap_recv = self.cap_back = 0
         self.ws, self.ws_n = None, -1
+        self.device_barrier = device_barrier
+        self.flags = None           # this rank's flag array (PeerBuffer, P uint64)
+        self.flag_addrs = None      # device uint64[P]: every rank's flag array, mapped here
+        self.flag_maps = []
+        self.epoch = 0
+        self.err = None
 
     # buffers --------------------------------------------------------------------------
     def ensure_capacity(self, cap_recv: int, cap_back: int):
@@ -335,6 +343,20 @@ class CudaPeerOps:
         self.recv_addr = [self.recv.addr if p == me else PeerBuffer.open(allh[p][0]) for p in range(self.P)]
         self.back_addr = [self.back.addr if p == me else PeerBuffer.open(allh[p][1]) for p in range(self.P)]
         self.cap_recv, self.cap_back = cap_recv, cap_back
+        if self.device_barrier and self.flags is None:  # once: flags outlive buffer growth
+            self.flags = PeerBuffer(8 * self.P)
+            allf = [None] * self.P
+            dist.all_gather_object(allf, self.flags.handle_bytes(), group=self.group)
+            addrs = [self.flags.addr if p == me else PeerBuffer.open(allf[p]) for p in range(self.P)]
+            self.flag_maps = [a for p, a in enumerate(addrs) if p != me]
+            self.flag_addrs = torch.tensor([a - (1 << 64) if a >= (1 << 63) else a for a in addrs],
+                                           dtype=torch.int64, device=self.dev)
+            self.err = torch.zeros(1, dtype=torch.int32, device=self.dev)
+
+    def check(self):
+        """Raise if a device barrier timed out (reads one flag; the caller has synchronised)."""
+        if self.err is not None and int(self.err.item()):
+            raise HarmoniaError(5, "harmonia_peer_barrier: timed out waiting for a peer")
 
     def close(self):
         from . import PeerBuffer
@@ -348,10 +370,15 @@ class CudaPeerOps:
             if p != me:
                 PeerBuffer.close_mapping(self.recv_addr[p])
                 PeerBuffer.close_mapping(self.back_addr[p])
+        for a in self.flag_maps:
+            PeerBuffer.close_mapping(a)
         dist.barrier(group=self.group)  # every mapping closed before the owners free
         self.recv.free()
         self.back.free()
-        self.recv = self.back = None
+        if self.flags is not None:
+            self.flags.free()
+        self.recv = self.back = self.flags = None
+        self.flag_maps, self.flag_addrs = [], None
         self.cap_recv = self.cap_back = 0
 
     # steps ----------------------------------------------------------------------------
@@ -393,6 +420,17 @@ class CudaPeerOps:
     def fence(self):
         torch.cuda.current_stream(self.dev).synchronize()  # the pushes of this rank are complete
 
+    def barrier(self):
+        """Every rank's pushes so far are visible to the work queued after this on the stream."""
+        if not self.device_barrier:
+            self.fence()
+            dist.barrier(group=self.group)
+            return
+        from . import peer_barrier
+
+        self.epoch += 1
+        peer_barrier(self.P, dist.get_rank(self.group), self.flag_addrs, self.flags.addr, self.epoch, self.err)
+
     def route_update(self, ops, keys, values, rank: int):
         rk, pos, counts = route_partition(self.split, self.P, keys)
         ro, rv, rs = route_update_payload(ops, values, pos, rank)
@@ -408,7 +446,7 @@ class PeerPartitionedTree:
     buffer and the results come back the same way."""
 
     def __init__(self, local_keys, local_values, splitters, fanout: int = 64, fill: float = 1.0, group=None,
-                 ops=None, device=None):
+                 ops=None, device=None, device_barrier: bool = True):
         self.group = group
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
@@ -416,7 +454,8 @@ class PeerPartitionedTree:
         if ops is None:
             dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
             tree = Tree(local_keys, local_values, fanout=fanout, fill=fill, device=dev)
-            ops = CudaPeerOps(tree, _u64_words(splitters, dev).view(torch.uint64), self.world, group)
+            ops = CudaPeerOps(tree, _u64_words(splitters, dev).view(torch.uint64), self.world, group,
+                              device_barrier=device_barrier)
         self.ops = ops
         self.splitters = list(splitters)
 
@@ -432,24 +471,34 @@ class PeerPartitionedTree:
     def search(self, q: torch.Tensor) -> torch.Tensor:
         P, me, n = self.world, self.rank, q.numel()
         counts = self.ops.route_count(q)                       # kernel: destination ranks
-        M = self._count_matrix(counts)                         # P x P ints
+        M = self._count_matrix(counts)                         # P x P ints (the host wait)
+        if hasattr(self.ops, "check"):
+            self.ops.check()                                   # the previous batch's barriers
         push_off, recv_off, recv_n, back_off = peer_offsets(M, me)
         need_recv = max(sum(M[p][d] for p in range(P)) for d in range(P))
         need_back = max(sum(row) for row in M)
         self.ops.ensure_capacity(need_recv, need_back)         # collective, same numbers everywhere
         self.ops.route_push(q, [(d, push_off[d]) for d in range(P)])  # kernel: NVLink stores
-        self.ops.fence()
-        dist.barrier(group=self.group)                         # every run has arrived
+        self._barrier()                                        # every run has arrived
         vals = self.ops.search_recv(recv_n)                    # local Harmonia search
         self.ops.segments_push(vals, [(recv_off[p], M[p][me], p, back_off[p]) for p in range(P)])
-        self.ops.fence()
-        dist.barrier(group=self.group)                         # every result has arrived
+        self._barrier()                                        # every result has arrived
         return self.ops.route_return(n)                        # kernel: caller's order
+
+    def _barrier(self):
+        if hasattr(self.ops, "barrier"):
+            self.ops.barrier()                                 # device-side (peer-memory flags)
+        else:
+            self.ops.fence()
+            dist.barrier(group=self.group)
 
     def update(self, ops, keys, values):
         """Batched upsert (op 0) / delete (op 1) routed to the owning shards (collective)."""
         _routed_update(self, ops, keys, values)
 
     def close(self):
+        if hasattr(self.ops, "check"):
+            torch.cuda.synchronize()
+            self.ops.check()
         if hasattr(self.ops, "close"):
             self.ops.close()

@@ -77,7 +77,7 @@ def _free_port():
     return p
 
 
-def _ipc_worker(rank, world, port, T, result_q):
+def _ipc_worker(rank, world, port, T, result_q, device_barrier=True):
     import torch.distributed as dist
 
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
@@ -92,7 +92,8 @@ def _ipc_worker(rank, world, port, T, result_q):
         sp = key_splitters(keys, world)
         bnd = [0] + [int(np.searchsorted(keys, np.uint64(s))) for s in sp] + [T]
         lk, lv = keys[bnd[rank]:bnd[rank + 1]], vals[bnd[rank]:bnd[rank + 1]]
-        pt = PeerPartitionedTree(_u64(lk), _u64(lv), sp, fanout=16, device=torch.device("cuda", 0))
+        pt = PeerPartitionedTree(_u64(lk), _u64(lv), sp, fanout=16, device=torch.device("cuda", 0),
+                                 device_barrier=device_barrier)
         ok = True
         for b, nq in enumerate((3000, 0, 70000, 5000)):  # growth of the buffers, an empty batch
             nq = nq + 111 * rank if nq else (0 if rank == 0 else 900)
@@ -108,14 +109,16 @@ def _ipc_worker(rank, world, port, T, result_q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_peer_partitioned_two_processes_ipc(world):
+@pytest.mark.parametrize("world,device_barrier", [(2, True), (3, True), (2, False)])
+def test_peer_partitioned_two_processes_ipc(world, device_barrier):
+    """device_barrier: the batch's two barriers are harmonia_peer_barrier kernels (flags in
+    IPC-mapped peer memory); False: stream synchronise + host barrier."""
     import torch.multiprocessing as mp
 
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_ipc_worker, args=(r, world, port, 60000, q)) for r in range(world)]
+    procs = [ctx.Process(target=_ipc_worker, args=(r, world, port, 60000, q, device_barrier)) for r in range(world)]
     for p in procs:
         p.start()
     res = [q.get(timeout=300) for _ in range(world)]
@@ -123,6 +126,28 @@ def test_peer_partitioned_two_processes_ipc(world):
         p.join(timeout=120)
     for rank, ok, err in res:
         assert ok, f"rank {rank}: {err or 'peer-routed results differ from the oracle'}"
+
+
+@pytest.mark.parametrize("P", [1, 3, 8])
+def test_peer_barrier_single_process(hm, P):
+    """harmonia_peer_barrier with P virtual ranks in one process, each on its own stream: every
+    kernel returns only when all P have arrived, with every flag at the epoch; a rank whose
+    peers never arrive times out and reports it instead of hanging."""
+    bufs = [torch.zeros(P, dtype=torch.int64, device="cuda") for _ in range(P)]  # rank me's flag array
+    addrs = torch.tensor([b.data_ptr() for b in bufs], dtype=torch.int64, device="cuda")
+    err = torch.zeros(1, dtype=torch.int32, device="cuda")
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    for epoch in (1, 2, 3):
+        for me in range(P):
+            hm.peer_barrier(P, me, addrs, bufs[me].data_ptr(), epoch, err, stream=streams[me])
+        torch.cuda.synchronize()
+        assert int(err.item()) == 0
+        for b in bufs:
+            assert b.cpu().tolist() == [epoch] * P
+    if P > 1:  # only rank 0 arrives at epoch 4: it must time out (1 ms), not hang
+        hm.peer_barrier(P, 0, addrs, bufs[0].data_ptr(), 4, err, timeout_ns=1_000_000)
+        torch.cuda.synchronize()
+        assert int(err.item()) == 1
 
 
 @pytest.mark.parametrize("P,cap", [(1, 16), (3, 0), (4, 64), (16, 32)])
