@@ -591,6 +591,7 @@ def main():
             os.environ.setdefault("MASTER_PORT", str(29500 + os.getpid() % 1000))
             os.environ.setdefault("RANK", "0")
             os.environ.setdefault("WORLD_SIZE", "1")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")  # NCCL's banner/log off stdout (the JSON line)
         dist.init_process_group("nccl", device_id=dev)
         pg = dist
 
