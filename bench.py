@@ -591,8 +591,19 @@ def main():
             os.environ.setdefault("MASTER_PORT", str(29500 + os.getpid() % 1000))
             os.environ.setdefault("RANK", "0")
             os.environ.setdefault("WORLD_SIZE", "1")
-        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")  # NCCL's banner/log off stdout (the JSON line)
-        dist.init_process_group("nccl", device_id=dev)
+        # NCCL prints its version banner on the C-level stdout at communicator creation; route
+        # fd 1 to stderr meanwhile so stdout carries only the JSON line
+        sys.stdout.flush()
+        saved = os.dup(1)
+        os.dup2(2, 1)
+        try:
+            dist.init_process_group("nccl", device_id=dev)
+            dist.barrier()
+            torch.cuda.synchronize()
+        finally:
+            sys.stdout.flush()
+            os.dup2(saved, 1)
+            os.close(saved)
         pg = dist
 
     def barrier():
