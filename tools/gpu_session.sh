@@ -11,7 +11,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
     python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu --no-extra > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_lane_search_c|k_psa2" -s 15 -c 5 \
     -o gpurun_out/${T}_c2 python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu --no-extra > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_lane_search_c|k_psa2|k_l2" -s 40 -c 12 \
+ncu --set full --clock-control none --import-source on -k regex:"k_lane_search_c|k_psa2|k_l2" -s 40 -c 16 \
     -o gpurun_out/${T}_c4 python tools/prof_search.py --keys 28 --queries 27 --calls 4 > /dev/null 2>&1
 ls -la gpurun_out | grep $T
 # summaries on the box (gpurun brings back at most 64 MiB): keep the c2 report, drop c4's
