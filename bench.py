@@ -328,14 +328,14 @@ def step_model(info, plan, nq, l2_cap, hbm_gbs, l2_gbs, psa=True):
             "reuse_aware": {"B_hbm": r_hbm, "B_l2": r_l2, "bound_gqs": rbound}}
 
 
-def ncu_stats(workload, kernel):
+def ncu_stats(workload, kernel, whole=False):
     """Per-launch ncu figures of `kernel` for `workload` from the committed capture summary
     (profiles/ncu_r2.json, tools/ncu_summary.py): DRAM and L2 bytes, sectors per request
     (the paper's memory divergence), warp coherence = active threads per
     executed instruction / 32 (P:L654 fn 4), branch uniformity."""
     try:
         d = json.load(open(os.path.join(ROOT, "profiles", "ncu_r2.json")))
-        return d.get(workload, {}).get(kernel)
+        return d.get(workload, {}) if whole else d.get(workload, {}).get(kernel)
     except Exception:
         return None
 
@@ -807,6 +807,30 @@ def main():
         if "l1_wavefront_pct" in st:  # the on-chip limiter of the search
             roof["limiter"] = {"resource": "L1 data-pipe (LSU) wavefronts", "frac": st["l1_wavefront_pct"] / 100,
                                "source": st.get("source")}
+        # the same limiter as a roofline on the live launch time: the kernel's LSU wavefronts
+        # per launch (committed capture) against 1 wavefront per cycle per SM at the median SM
+        # clock sampled during the timed region; and for the whole step (every kernel of the
+        # step, one launch each), the LSU-bound step time against the measured one
+        mhz = clk.summary().get("sm_mhz")
+        nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+        if st.get("lsu_wavefronts") and mhz:
+            lpeak = nsm * mhz * 1e6
+            ach = st["lsu_wavefronts"] / (roof["avg_launch_ms"] / 1e3)
+            roof["lsu"] = {"achieved": ach / 1e9, "peak": lpeak / 1e9, "unit": "G wavefronts/s",
+                           "frac": ach / lpeak, "wavefronts_per_launch": st["lsu_wavefronts"],
+                           "shared_wavefronts_per_launch": st.get("lsu_wavefronts_shared"),
+                           "peak_source": f"1 L1 data-pipe wavefront / cycle / SM x {nsm} SMs x {mhz:.0f} MHz "
+                                          "(median SM clock in the timed region)",
+                           "source": st.get("source")}
+            step_k = ("k_psa2_rank", "k_psa2_move", "k_psa2_count_sort", "k_lane_search_c", "k_psa2_unmove")
+            allk = (ncu_stats(c["name"], None, whole=True) or {})
+            if plan.get("staged_return") and plan.get("psa_levels") == 1 and all(
+                    allk.get(k, {}).get("lsu_wavefronts") for k in step_k):
+                wsum = sum(allk[k]["lsu_wavefronts"] for k in step_k)
+                bound_ms = wsum / lpeak * 1e3
+                roof["step_lsu"] = {"wavefronts_per_step": wsum, "bound_ms": bound_ms,
+                                    "measured_ms": ms_max / a.steps, "frac": bound_ms / (ms_max / a.steps),
+                                    "kernels": list(step_k), "source": st.get("source")}
     if roof is not None and l2_peak:
         sm_ = step_model(info, plan, c["Q"] * 1, l2_bytes, hbm_peak, l2_peak, psa=plan["psa_bits"] > 0)
         sm_["frac"] = value / world / sm_["bound_gqs"]

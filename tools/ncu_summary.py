@@ -26,6 +26,7 @@ METRICS = [
     "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed",
     "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
     "lts__t_sectors.sum", "lts__t_sectors_srcunit_tex.sum", "lts__t_sectors_srcunit_ltcfabric.sum",
+    "l1tex__data_pipe_lsu_wavefronts.sum", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
 ]
 
 
@@ -136,6 +137,13 @@ if __name__ == "__main__":
         if isinstance(tv, float):
             ent["ncu_time_s"] = tv * {"ns": 1e-9, "nsecond": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3,
                                       "msecond": 1e-3, "s": 1.0, "second": 1.0}.get(tu, 1e-9)
+        # L1 data-pipe (LSU) wavefronts per launch: global/local loads and stores, shared-memory
+        # accesses, atomics and shuffles all pass this pipe (1 wavefront per cycle per SM)
+        for key, m in (("lsu_wavefronts", "l1tex__data_pipe_lsu_wavefronts.sum"),
+                       ("lsu_wavefronts_shared", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")):
+            v = d.get(m)
+            if isinstance(v, float):
+                ent[key] = v
         st = d.get("stall_share")
         if isinstance(st, dict) and "long_scoreboard" in st:
             ent["long_scoreboard_stall_share"] = st["long_scoreboard"]
