@@ -91,3 +91,31 @@ def test_config5_shard_full_size(hm):
     info = t.info()
     assert info["n_keys"] == S and info["key_region_bytes"] > (1 << 32)  # byte offsets beyond 32 bits
     _check_device(hm, t, keys_t, 1 << 26, seed=gen.SEED_QUERY + 5)
+
+
+@pytest.mark.parametrize("fanout,fill", [(8, 1.0), (16, 1.0), (32, 1.0), (128, 1.0), (8, 0.69), (32, 0.69),
+                                         (64, 0.69), (128, 0.69)])
+def test_config3_fanout_sweep_full_size(hm, orc, fanout, fill):
+    """c3's fanout sweep at its full size (2^26 keys, F in 8..128, fill
+    1.0 and 0.69, 2^26 Zipfian queries), in the launch configuration the bench's sweep times:
+    every hit checked on the device by the key-derived values, key+1 misses, and 2^18 sampled
+    queries element by element against the oracle."""
+    import torch
+
+    T, Q = 1 << 26, 1 << 26
+    keys_t = gen.uniform_keys_t(T, "cuda")
+    t = hm.Tree(keys_t.view(torch.uint64), gen.values_for_t(keys_t).view(torch.uint64), fanout=fanout, fill=fill)
+    q = gen.zipf_queries_t(keys_t, Q)
+    out = t.search(q.view(torch.uint64)).view(torch.int64)
+    assert int((out != gen.values_for_t(q)).sum()) == 0
+    _check_device(hm, t, keys_t, 1 << 22, seed=gen.SEED_QUERY + fanout)
+    keys = keys_t.cpu().numpy().view(np.uint64)
+    sel = torch.from_numpy((gen._stream(13 + fanout, 0, 1 << 18) % np.uint64(Q)).astype(np.int64)).cuda()
+    qs = q[sel].cpu().numpy().view(np.uint64)
+    assert np.array_equal(out[sel].cpu().numpy().view(np.uint64), orc.sorted_search(keys, gen.values_for(keys), qs))
+    vals = gen.values_for(keys)
+    lo, hi = gen.ranges(keys, 1 << 12, 64)
+    ko, vo, cnt = t.range(torch.from_numpy(lo).cuda(), torch.from_numpy(hi).cuda(), 64)
+    eko, evo, ecnt = orc.sorted_range(keys, vals, lo, hi, 64)
+    assert np.array_equal(cnt.cpu().numpy(), ecnt)
+    assert np.array_equal(ko.cpu().numpy(), eko) and np.array_equal(vo.cpu().numpy(), evo)
