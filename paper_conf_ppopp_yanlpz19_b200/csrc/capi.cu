@@ -425,10 +425,14 @@ extern "C" harmonia_status harmonia_psa_inspect(const harmonia_tree* t, const ui
 }
 
 // ---- host-buffer pipeline --------------------------------------------------------------
+#ifndef HM_HOST_CHUNK_LOG
+#define HM_HOST_CHUNK_LOG 22
+#endif
 static uint64_t host_chunk(const Plan& p, uint64_t n) {
   // 4M-query chunks: the copies (PCIe-bound) dominate, so a deeper pipeline beats larger
   // PSA windows here
-  uint64_t c = std::min<uint64_t>(p.psa ? p.window : (1ull << 22), 1ull << 22);
+  constexpr uint64_t kC = 1ull << HM_HOST_CHUNK_LOG;
+  uint64_t c = std::min<uint64_t>(p.psa ? p.window : kC, kC);
   return std::max<uint64_t>(1024, std::min<uint64_t>(c, round_up(std::max<uint64_t>(n, 1), 1024)));
 }
 
