@@ -453,6 +453,9 @@ __device__ __forceinline__ void ld_quad_global(const uint64_t* p, uint64_t (&k)[
 #ifndef HM_LEAF_TAIL
 #define HM_LEAF_TAIL 4  // measured: 4 > 8 > 16 > off at c2 and c3
 #endif
+#ifndef HM_TAIL3
+#define HM_TAIL3 1
+#endif
 // Per-lane rank in a global node with a vector tail: binary-lifting steps down to TL keys,
 // then the TL-key block [r, r+TL) is read with TL/4 independent 256-bit loads and counted
 // (keys below r are <= q, keys from r+TL on are > q, so r + #(block <= q) is the rank).
@@ -462,7 +465,7 @@ __device__ __forceinline__ void prefetch_l1(const void* p) { asm volatile("prefe
 // once the rank is known to a 16-slot block, that block's value line is prefetched into L1 so
 // the final value load does not wait for another L2 round trip (measured: c4 search −5 %; with
 // one PSA level the extra L1 requests cost more than the saved round trip, c2 +2 %, c3 +10 %)
-template <int F, int U, int TL>
+template <int F, int U, int TL, bool T3 = false>
 __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint32_t (&node)[U],
                                                const uint64_t (&q)[U], uint32_t (&r)[U], uint64_t (&best)[U],
                                                const uint64_t* vrow = nullptr) {
@@ -482,6 +485,30 @@ __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint3
       for (int u = 0; u < U; ++u) prefetch_l1(vrow + (uint64_t)node[u] * F + r[u]);
     }
   }
+#if HM_TAIL3
+  if constexpr (TL == 4 && T3) {
+    // the rank lies in [r, r+4): keys r, r+1 (one 128-bit load, 16-byte aligned) and r+2 (one
+    // 64-bit load) decide it; key r+3 is known to be > q.  Two loads, one round trip, and
+    // fewer L1 data-pipe wavefronts than one 256-bit load per lane (ncu: 21.5 per warp-row).
+    // Measured: two-level (chunk-table) kernel c4 search 1.833 -> 1.765 ms; the one-level
+    // kernel loses (c2 0.865 -> 0.872, 2^26 keys 1.71 -> 1.83), so T3 = that kernel only.
+    ulonglong2 k01[U];
+    uint64_t k2[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t* b = keys + (uint64_t)node[u] * F + r[u];
+      k01[u] = ld_pair_global(b);
+      k2[u] = ld_key_global(b + 2);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool l0 = k01[u].x <= q[u], l1 = k01[u].y <= q[u], l2 = k2[u] <= q[u];
+      r[u] += (l0 ? 1u : 0u) + (l1 ? 1u : 0u) + (l2 ? 1u : 0u);
+      best[u] = l2 ? k2[u] : (l1 ? k01[u].y : (l0 ? k01[u].x : best[u]));
+    }
+    return;
+  }
+#endif
   uint64_t k[U][TL];
 #pragma unroll
   for (int u = 0; u < U; ++u)
@@ -560,7 +587,7 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
   }
 #if HM_LEAF_TAIL > 0
   if (F >= 2 * HM_LEAF_TAIL && !leaf_smem) {
-    lane_rank_tail<F, U, (F >= 2 * HM_LEAF_TAIL ? HM_LEAF_TAIL : 4)>(
+    lane_rank_tail<F, U, (F >= 2 * HM_LEAF_TAIL ? HM_LEAF_TAIL : 4), PF && !RANK>(
         a.keys, node, q, r, best, PF && !RANK ? a.vals - (uint64_t)a.leaf_start * F : nullptr);
   } else
 #endif
