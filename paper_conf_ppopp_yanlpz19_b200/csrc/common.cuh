@@ -323,6 +323,10 @@ harmonia_status psa_partition(const uint64_t* q, uint64_t n, const Bucket& f, ui
                               const PsaWs& ws, int sm_count, cudaStream_t st,
                               uint64_t* h_counts /* optional: sync copy of counts */);
 
+// rank-mode results (update locate, short ranges): (leaf << 32) | #keys <= q | kRankHit when
+// the leaf holds q (the in-place update needs no second read of the key)
+constexpr uint32_t kRankHit = 0x80000000u;
+
 struct SearchArgs {
   const uint64_t* keys;
   const uint32_t* ps;

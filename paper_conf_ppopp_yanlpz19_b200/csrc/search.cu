@@ -533,7 +533,8 @@ __device__ __forceinline__ void lane_rank_tail(const uint64_t* keys, const uint3
 // the memory-level parallelism without adding work.  A warp takes 32*U consecutive
 // (PSA-ordered) queries: query (u, lane) = base + u*32 + lane.
 // one lane, U interleaved queries, from level l0 at nodes node[]: descent (Eq 1) + leaf probe
-// RANK: instead of the value, res = (leaf index << 32) | #keys <= q in that leaf (the range
+// RANK: instead of the value, res = (leaf index << 32) | #keys <= q in that leaf | kRankHit when
+// the leaf holds q itself (the range
 // kernels turn it into a global record rank with leaf_base)
 template <int F, int U, bool RANK = false, bool PF = false>
 __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t* s_keys, const uint32_t* s_ps,
@@ -610,7 +611,8 @@ __device__ __forceinline__ void lane_descend(const SearchArgs& a, const uint64_t
 #pragma unroll
   for (int u = 0; u < U; ++u) {
     if constexpr (RANK) {
-      res[u] = ((uint64_t)(node[u] - a.leaf_start) << 32) | r[u];
+      const bool ex = live[u] && r[u] > 0 && best[u] == q[u];
+      res[u] = ((uint64_t)(node[u] - a.leaf_start) << 32) | r[u] | (ex ? kRankHit : 0u);
     } else {
       res[u] = kNotFound;
       if (live[u] && r[u] > 0 && best[u] == q[u])
@@ -873,7 +875,8 @@ __device__ __forceinline__ void warp_core(const SearchArgs& a, const uint64_t* s
 #pragma unroll
   for (int u = 0; u < U; ++u) {
     if constexpr (RANK) {
-      res[u] = ((uint64_t)(node - a.leaf_start) << 32) | r[u];
+      const bool ex = live[u] && r[u] > rlo && best[u] == q[u];
+      res[u] = ((uint64_t)(node - a.leaf_start) << 32) | r[u] | (ex ? kRankHit : 0u);
     } else {
       res[u] = kNotFound;
       if (live[u] && r[u] > rlo && best[u] == q[u]) res[u] = __ldg(vrow + (r[u] - 1));
@@ -1239,14 +1242,20 @@ __global__ void __launch_bounds__(256) k_locate(const SearchArgs a, const uint64
   const unsigned lane = threadIdx.x & 31;
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t base = warp * 32; base < n; base += nwarps * 32) {
-    const uint64_t j = base + lane;
-    const bool act = j < n;
-    uint64_t q0[1] = {act ? q[j] : kPad};
-    bool live[1] = {act && q0[0] != kPad};
-    uint64_t res[1];
-    warp_core<F, 1, true>(a, nullptr, nullptr, false, false, q0, live, res);
-    if (act) out[j] = res[0];
+  for (uint64_t base = warp * 64; base < n; base += nwarps * 64) {  // two sorted keys per lane
+    uint64_t q0[2];
+    bool live[2];
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const uint64_t j = base + u * 32 + lane;
+      q0[u] = j < n ? q[j] : kPad;
+      live[u] = j < n && q0[u] != kPad;
+    }
+    uint64_t res[2];
+    warp_core<F, 2, true>(a, nullptr, nullptr, false, false, q0, live, res);
+#pragma unroll
+    for (int u = 0; u < 2; ++u)
+      if (base + u * 32 + lane < n) out[base + u * 32 + lane] = res[u];
   }
 }
 
@@ -1288,9 +1297,9 @@ __global__ void __launch_bounds__(1024, 1) k_range_lane(const RangeArgs ra, cons
     if (valid) {
       if (qa[0]) {
         leaf = (uint32_t)(res[0] >> 32);
-        r0 = __ldg(ra.leaf_base + leaf) + (uint32_t)res[0];
+        r0 = __ldg(ra.leaf_base + leaf) + ((uint32_t)res[0] & ~kRankHit);
       }
-      const uint64_t r1 = __ldg(ra.leaf_base + (res[1] >> 32)) + (uint32_t)res[1];
+      const uint64_t r1 = __ldg(ra.leaf_base + (res[1] >> 32)) + ((uint32_t)res[1] & ~kRankHit);
       count = r1 > r0 ? r1 - r0 : 0;
     }
     const uint32_t ncopy = (uint32_t)(count < cap ? count : cap);
@@ -1547,7 +1556,7 @@ harmonia_status launch_locate(const harmonia_tree* t, const uint64_t* q, uint64_
   a.kmax = t->max_key;
   const uint32_t span = t->min_key < t->max_key ? 64 - __builtin_clzll(t->min_key ^ t->max_key) : 0;
   a.cshift = span > 32 ? span - 32 : 0;
-  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(n, 256), (uint64_t)t->sm_count * 8));
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(ceil_div(n, 512), (uint64_t)t->sm_count * 8));
   switch (t->F) {
 #define HM_LOC(F_)                                        \
   case F_:                                                \

@@ -184,8 +184,8 @@ __global__ void k_upd_ip_classify(const uint64_t* __restrict__ wk, const uint8_t
                                   uint32_t F, int32_t* __restrict__ ldelta, uint8_t* __restrict__ lflag,
                                   uint32_t* __restrict__ wleaf) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t leaf = (uint32_t)(loc[i] >> 32), r = (uint32_t)loc[i];
-    const bool exists = r > 0 && kr[(leaf_start + leaf) * F + r - 1] == wk[i];
+    const uint32_t leaf = (uint32_t)(loc[i] >> 32), r = (uint32_t)loc[i] & ~kRankHit;
+    const bool exists = ((uint32_t)loc[i] & kRankHit) != 0;  // the locate saw key[r-1] == wk[i]
     wleaf[i] = leaf;
     if (wop[i] == 0) {
       if (exists) {
