@@ -340,6 +340,36 @@ def ncu_stats(workload, kernel, whole=False):
         return None
 
 
+STEP_KERNELS = ("k_psa2_rank", "k_psa2_move", "k_psa2_count_sort", "k_lane_search_c", "k_psa2_unmove")
+
+
+def lsu_roofline(st, allk, nsm, mhz, avg_launch_ms, step_ms, one_level):
+    """The search kernel's L1 data-pipe (LSU) roofline and the step's (DESIGN.md §7 item 4):
+    every global / shared access, shared atomic and shuffle retires through the SM's L1 data
+    pipe at one wavefront per cycle.  `st` / `allk`: per-launch ncu figures of the kernel and of
+    every kernel of the workload (profiles/ncu_r2.json); nsm SMs at mhz (median SM clock in the
+    timed region).  lsu = wavefronts per launch over the live launch time against nsm x clock;
+    step_lsu (one-level staged path: the five kernels of a step, one launch each) = the
+    LSU-bound step time against the measured one.  Returns (lsu, step_lsu), None when absent."""
+    if not st or not st.get("lsu_wavefronts") or not mhz:
+        return None, None
+    lpeak = nsm * mhz * 1e6
+    ach = st["lsu_wavefronts"] / (avg_launch_ms / 1e3)
+    lsu = {"achieved": ach / 1e9, "peak": lpeak / 1e9, "unit": "G wavefronts/s", "frac": ach / lpeak,
+           "wavefronts_per_launch": st["lsu_wavefronts"],
+           "shared_wavefronts_per_launch": st.get("lsu_wavefronts_shared"),
+           "peak_source": f"1 L1 data-pipe wavefront / cycle / SM x {nsm} SMs x {mhz:.0f} MHz "
+                          "(median SM clock in the timed region)",
+           "source": st.get("source")}
+    step = None
+    if one_level and all(allk.get(k, {}).get("lsu_wavefronts") for k in STEP_KERNELS):
+        wsum = sum(allk[k]["lsu_wavefronts"] for k in STEP_KERNELS)
+        bound_ms = wsum / lpeak * 1e3
+        step = {"wavefronts_per_step": wsum, "bound_ms": bound_ms, "measured_ms": step_ms,
+                "frac": bound_ms / step_ms, "kernels": list(STEP_KERNELS), "source": st.get("source")}
+    return lsu, step
+
+
 def load_peaks():
     hbm, src = 6650.0, "fallback (B200_PROFILING.md)"
     try:
@@ -813,24 +843,13 @@ def main():
         # step, one launch each), the LSU-bound step time against the measured one
         mhz = clk.summary().get("sm_mhz")
         nsm = torch.cuda.get_device_properties(dev).multi_processor_count
-        if st.get("lsu_wavefronts") and mhz:
-            lpeak = nsm * mhz * 1e6
-            ach = st["lsu_wavefronts"] / (roof["avg_launch_ms"] / 1e3)
-            roof["lsu"] = {"achieved": ach / 1e9, "peak": lpeak / 1e9, "unit": "G wavefronts/s",
-                           "frac": ach / lpeak, "wavefronts_per_launch": st["lsu_wavefronts"],
-                           "shared_wavefronts_per_launch": st.get("lsu_wavefronts_shared"),
-                           "peak_source": f"1 L1 data-pipe wavefront / cycle / SM x {nsm} SMs x {mhz:.0f} MHz "
-                                          "(median SM clock in the timed region)",
-                           "source": st.get("source")}
-            step_k = ("k_psa2_rank", "k_psa2_move", "k_psa2_count_sort", "k_lane_search_c", "k_psa2_unmove")
-            allk = (ncu_stats(c["name"], None, whole=True) or {})
-            if plan.get("staged_return") and plan.get("psa_levels") == 1 and all(
-                    allk.get(k, {}).get("lsu_wavefronts") for k in step_k):
-                wsum = sum(allk[k]["lsu_wavefronts"] for k in step_k)
-                bound_ms = wsum / lpeak * 1e3
-                roof["step_lsu"] = {"wavefronts_per_step": wsum, "bound_ms": bound_ms,
-                                    "measured_ms": ms_max / a.steps, "frac": bound_ms / (ms_max / a.steps),
-                                    "kernels": list(step_k), "source": st.get("source")}
+        one_level = bool(plan.get("staged_return")) and plan.get("psa_levels") == 1
+        lsu, step_lsu = lsu_roofline(st, ncu_stats(c["name"], None, whole=True) or {}, nsm, mhz,
+                                     roof["avg_launch_ms"], ms_max / a.steps, one_level)
+        if lsu:
+            roof["lsu"] = lsu
+        if step_lsu:
+            roof["step_lsu"] = step_lsu
     if roof is not None and l2_peak:
         sm_ = step_model(info, plan, c["Q"] * 1, l2_bytes, hbm_peak, l2_peak, psa=plan["psa_bits"] > 0)
         sm_["frac"] = value / world / sm_["bound_gqs"]

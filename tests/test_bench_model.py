@@ -47,3 +47,28 @@ def test_step_model_hbm_tier():
     m = bench.step_model(info, {"smem_levels": 2}, 1 << 27, 132644864, 6538.0, 17775.2)
     assert m["l2_tier_levels"] == 2 and m["hbm_tier_levels"] == 1
     assert m["B_hbm"] == 88 + 544 and m["B_l2"] == 88 + 3 * 544
+
+
+def test_lsu_roofline_from_committed_capture():
+    """roofline.lsu / step_lsu from the committed c2 capture: the search kernel's wavefronts
+    over its launch time against 1 wavefront / cycle / SM, and the sum over the five kernels
+    of a step as an LSU-bound step time (DESIGN.md §7 item 4)."""
+    import json
+    import os
+
+    d = json.load(open(os.path.join(os.path.dirname(bench.__file__), "profiles", "ncu_r2.json")))
+    allk = d["c2_T2^23_F64_Q2^26_uniform"]
+    st = allk["k_lane_search_c"]
+    lsu, step = bench.lsu_roofline(st, allk, 148, 2000.0, 1.0, 2.0, True)
+    assert abs(lsu["peak"] - 296.0) < 1e-9                      # 148 x 2 GHz x 1 wavefront
+    assert abs(lsu["achieved"] - st["lsu_wavefronts"] / 1e-3 / 1e9) < 1e-9
+    wsum = sum(allk[k]["lsu_wavefronts"] for k in bench.STEP_KERNELS)
+    assert step["wavefronts_per_step"] == wsum
+    assert abs(step["bound_ms"] - wsum / 296e9 * 1e3) < 1e-12
+    assert abs(step["frac"] - step["bound_ms"] / 2.0) < 1e-12
+    # the committed capture: the search alone is the largest share of the step's wavefronts
+    assert st["lsu_wavefronts"] > 0.4 * wsum
+    # absent inputs: no figure, no exception
+    assert bench.lsu_roofline(None, {}, 148, 2000.0, 1.0, 2.0, True) == (None, None)
+    assert bench.lsu_roofline(st, allk, 148, None, 1.0, 2.0, True) == (None, None)
+    assert bench.lsu_roofline(st, allk, 148, 2000.0, 1.0, 2.0, False)[1] is None
