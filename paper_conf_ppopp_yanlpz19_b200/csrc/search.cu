@@ -929,7 +929,7 @@ __global__ void __launch_bounds__(1024, (U <= 2 ? 2 : 1)) k_lane_search_u(const 
 // warp-shared descent every warp starts below its chunk's shared path.  A separate
 // instantiation: the variable start node costs registers at the 32-register cap (8 bytes of
 // spills), which the narrow bucket-aligned chunks repay and the one-level chunks do not.
-// Specializations (HM_SEARCH_SPEC, F = 64): PSS >= 0 makes the staging facts known at launch
+// Specializations (HM_SEARCH_SPEC; heights and the two-level kernel at F = 64 only): PSS >= 0 makes the staging facts known at launch
 // compile-time constants -- whether the PS is in shared memory (PSS), and that the leaves are
 // not -- and H > 0 fixes the tree height and the staged levels (SL) too, so the level loops
 // unroll and every per-level choice between shared and global reads is resolved at compile
@@ -1403,7 +1403,10 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
     kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true, true> : (U == 2 ? k_lane_search_c<F, 2, true, true> : k_lane_search_c<F, 1, true, true>))
                   : (U >= 4 ? k_lane_search_c<F, 4, false, true> : (U == 2 ? k_lane_search_c<F, 2, false, true> : k_lane_search_c<F, 1, false, true>));
 #if HM_SEARCH_SPEC
-  if constexpr (F == 64) {
+  if constexpr (F != 64) {  // other fanouts: the staging facts only, one-level path
+    if (a.coop && U == 2 && !a.ctab && a.h - 1 >= a.smem_levels)
+      kern = a.ps_smem_bytes != 0 ? k_lane_search_c<F, 2, true, false, 1> : k_lane_search_c<F, 2, true, false, 0>;
+  } else {
     if (a.coop && U == 2 && a.h - 1 >= a.smem_levels) {
       const bool pss = a.ps_smem_bytes != 0, tab = a.ctab != nullptr;
       kern = tab ? (pss ? k_lane_search_c<F, 2, true, true, 1> : k_lane_search_c<F, 2, true, true, 0>)
