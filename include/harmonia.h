@@ -119,6 +119,14 @@ typedef struct {
 #define HARMONIA_QF_PSA_L16 8192u /* staged-return PSA: force two MSD levels (8 + 8 bits) and
                                       bucket-aligned chunks, i.e. the whole window in Eq-2
                                       order (default: chosen by the plan, see harmonia_plan) */
+#define HARMONIA_QF_HOST_UNORDERED 65536u /* harmonia_search_batch_host: the caller guarantees that
+                                      h_queries is ready when the call is made (written by the host,
+                                      not by earlier work on `stream`), so the first chunks' H2D
+                                      copies wait only for their device buffers, not for earlier
+                                      work on `stream`: back-to-back calls then overlap one call's
+                                      last D2H copy with the next call's first H2D copy.  Results
+                                      are unchanged; h_values_out stays ordered after the call's
+                                      own work as before. */
 #define HARMONIA_QF_PSA_L8 16384u /* staged-return PSA: force one MSD level (8 bits) + chunk
                                       sort (the window is Eq-2 ordered inside each chunk)    */
 #define HARMONIA_QF_LINEAR     4u  /* in-node search = the paper's linear NTG walk (Fig 9:

@@ -32,6 +32,7 @@ QF_RANGE_GROUP = 2048
 QF_PSA_L16 = 8192
 QF_PSA_L8 = 16384
 QF_NO_RANGE_LANE = 32768
+QF_HOST_UNORDERED = 65536
 _STATUS = {0: "OK", 1: "INVALID_ARG", 2: "UNSORTED", 3: "RESERVED", 4: "OUT_OF_MEMORY", 5: "CUDA",
            6: "DEVICE_MISMATCH", 7: "TOO_LARGE"}
 

@@ -477,15 +477,19 @@ extern "C" harmonia_status harmonia_search_batch_host(const harmonia_tree* tc, c
       HM_CUDA(cudaEventCreateWithFlags(&t->ev_out[i], cudaEventDisableTiming));
     }
   }
-  // order the pipeline after the caller's prior work
+  // order the pipeline after the caller's prior work (the query copies only when the caller
+  // has not declared the host queries ready: HARMONIA_QF_HOST_UNORDERED)
+  const bool unordered = o && (o->flags & HARMONIA_QF_HOST_UNORDERED);
   HM_CUDA(cudaEventRecord(t->ev_start, st));
-  HM_CUDA(cudaStreamWaitEvent(t->s_h2d, t->ev_start, 0));
+  if (!unordered) HM_CUDA(cudaStreamWaitEvent(t->s_h2d, t->ev_start, 0));
   HM_CUDA(cudaStreamWaitEvent(t->s_d2h, t->ev_start, 0));
   const uint64_t chunks = ceil_div(n, C);
   for (uint64_t k = 0; k < chunks; ++k) {
     const int b = (int)(k & 1);
     const uint64_t off = k * C, m = std::min<uint64_t>(C, n - off);
-    if (k >= 2) HM_CUDA(cudaStreamWaitEvent(t->s_h2d, t->ev_done[b], 0));  // din[b] consumed
+    // din[b] consumed: by this call's chunk k-2, or (unordered) by the last chunk of an earlier
+    // call that used it (an event never recorded is complete)
+    if (k >= 2 || unordered) HM_CUDA(cudaStreamWaitEvent(t->s_h2d, t->ev_done[b], 0));
     HM_CUDA(cudaMemcpyAsync(din[b], h_q + off, m * 8, cudaMemcpyHostToDevice, t->s_h2d));
     HM_CUDA(cudaEventRecord(t->ev_in[b], t->s_h2d));
     HM_CUDA(cudaStreamWaitEvent(st, t->ev_in[b], 0));

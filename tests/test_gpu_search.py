@@ -344,6 +344,26 @@ def test_search_host_pipeline(hm, orc):
     assert np.array_equal(out2.numpy(), out.numpy())
 
 
+def test_search_host_unordered_back_to_back(hm, orc):
+    """HARMONIA_QF_HOST_UNORDERED: back-to-back host-buffer calls with different queries and
+    outputs, queued without synchronising in between (the next call's first H2D copies overlap
+    the previous call's last D2H copies); every output equals the oracle's."""
+    import torch
+
+    keys = gen.uniform_keys(1 << 18)
+    vals = gen.values_for(keys)
+    t = tree(hm, keys, vals, 64)
+    n = (1 << 22) * 2 + 777  # three host chunks: both device buffers in use at the call end
+    qs = [gen.uniform_queries(keys, n, seed=gen.SEED_QUERY + i, miss_frac=0.1) for i in range(4)]
+    qh = [torch.from_numpy(q).pin_memory() for q in qs]
+    oh = [torch.empty(n, dtype=torch.uint64, pin_memory=True) for _ in qs]
+    for i in range(4):
+        t.search_host(qh[i], oh[i], flags=hm.QF_HOST_UNORDERED)
+    torch.cuda.synchronize()
+    for i in range(4):
+        assert np.array_equal(oh[i].numpy(), orc.sorted_search(keys, vals, qs[i])), f"call {i}"
+
+
 # ----------------------------------------------------------------------------- routing
 def test_route_partition_and_scatter(hm):
     import torch
