@@ -527,8 +527,7 @@ def run_config5(a, c, hm, dev, world, rank, local, pg):
         hopts = hm.make_opts(a.group_size, a.psa_bits, a.smem_levels, a.window, a.flags | hm.QF_HOST_UNORDERED)
 
         def e2e_step():
-            q.copy_(q_host, non_blocking=True)
-            out_host.copy_(pt.search(q), non_blocking=True)
+            pt.search_host(q_host, out_host, opts=hopts)
             o, k, v = batches[it[0] % nb]
             it[0] += 1
             pt.update(o, k, v)
@@ -543,7 +542,8 @@ def run_config5(a, c, hm, dev, world, rank, local, pg):
             hms = float(tt.item())
         e2e = {"value": c["Q"] * world * k2 / (hms / 1e3) / 1e9, "unit": UNIT,
                "h2d_bytes_per_step": int(c["Q"] * 8), "d2h_bytes_per_step": int(c["Q"] * 8), "steps": k2,
-               "ms_per_step": hms / k2, "api": "PartitionedTree.search + update, pinned query/result copies",
+               "ms_per_step": hms / k2, "api": "PartitionedTree.search_host + update (one shard: the tree's H2D/search/D2H pipeline; "
+                      "several: pinned copies around the routed search)",
                "note": "update batches are device-resident (generated on the device) in both measurements"}
     if rank != 0:
         return

@@ -214,6 +214,17 @@ class PartitionedTree:
                                group=self.group)               # C5: return values
         return self.ops.scatter(_u64(back), pos)               # caller's order
 
+    def search_host(self, q_host: torch.Tensor, out_host: torch.Tensor, **kw) -> torch.Tensor:
+        """Point queries from and to pinned host memory.  One shard: the tree's own three-stage
+        host pipeline (harmonia_search_batch_host, H2D / search / D2H overlapped chunk by
+        chunk); several shards: one H2D copy, the routed search, one D2H copy."""
+        if self.world == 1 and hasattr(self.ops, "tree"):
+            return self.ops.tree.search_host(q_host, out_host, **kw)
+        dev = self.ops.tree.device if hasattr(self.ops, "tree") else q_host.device
+        q = q_host.to(dev, non_blocking=True)
+        out_host.copy_(self.search(q), non_blocking=True)
+        return out_host
+
     def _search_sliced(self, q, slices):
         import contextlib
 

@@ -166,6 +166,10 @@ def _worker(rank, world, port, T, cap, result_q):
         # the sliced exchange (slice i+1 in flight while slice i is searched) gives the same
         got3 = pt.search(qt, slices=3).view(torch.int64).numpy().view(np.uint64)
         ok_pts = ok_pts and bool(np.array_equal(got3, exp))
+        # host buffers in and out (search_host: copies around the routed search)
+        oh = torch.empty(q.shape[0], dtype=torch.uint64)
+        goth = pt.search_host(qt.clone(), oh).view(torch.int64).numpy().view(np.uint64)
+        ok_pts = ok_pts and bool(np.array_equal(goth, exp))
         # ranges: short, long (crossing several shards), empty, lo > hi, full span
         lo1, hi1 = gen.ranges(keys, 200, 40, seed=gen.SEED_RANGE + rank)
         lo2, hi2 = gen.random_ranges(keys, 200, seed=gen.SEED_RANGE + 7 * rank, max_width_keys=T)
