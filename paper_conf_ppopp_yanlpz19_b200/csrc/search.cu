@@ -1403,9 +1403,20 @@ harmonia_status launch_lane_search_c(const harmonia_tree* t, const Plan& p, cons
     kern = a.coop ? (U >= 4 ? k_lane_search_c<F, 4, true, true> : (U == 2 ? k_lane_search_c<F, 2, true, true> : k_lane_search_c<F, 1, true, true>))
                   : (U >= 4 ? k_lane_search_c<F, 4, false, true> : (U == 2 ? k_lane_search_c<F, 2, false, true> : k_lane_search_c<F, 1, false, true>));
 #if HM_SEARCH_SPEC
-  if constexpr (F != 64) {  // other fanouts: the staging facts only, one-level path
-    if (a.coop && U == 2 && !a.ctab && a.h - 1 >= a.smem_levels)
-      kern = a.ps_smem_bytes != 0 ? k_lane_search_c<F, 2, true, false, 1> : k_lane_search_c<F, 2, true, false, 0>;
+  if constexpr (F != 64) {  // other fanouts: the staging facts, one-level path
+    if (a.coop && U == 2 && !a.ctab && a.h - 1 >= a.smem_levels) {
+      const bool pss = a.ps_smem_bytes != 0;
+      kern = pss ? k_lane_search_c<F, 2, true, false, 1> : k_lane_search_c<F, 2, true, false, 0>;
+      // and config 3's geometries (2^26 keys, fill 1.0, the 48 KiB staging budget)
+      if constexpr (F == 8)
+        if (!pss && a.h == 9 && a.smem_levels == 4) kern = k_lane_search_c<F, 2, true, false, 0, 9, 4>;
+      if constexpr (F == 16)
+        if (!pss && a.h == 7 && a.smem_levels == 3) kern = k_lane_search_c<F, 2, true, false, 0, 7, 3>;
+      if constexpr (F == 32)
+        if (!pss && a.h == 6 && a.smem_levels == 3) kern = k_lane_search_c<F, 2, true, false, 0, 6, 3>;
+      if constexpr (F == 128)
+        if (pss && a.h == 4 && a.smem_levels == 1) kern = k_lane_search_c<F, 2, true, false, 1, 4, 1>;
+    }
   } else {
     if (a.coop && U == 2 && a.h - 1 >= a.smem_levels) {
       const bool pss = a.ps_smem_bytes != 0, tab = a.ctab != nullptr;
